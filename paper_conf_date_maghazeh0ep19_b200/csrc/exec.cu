@@ -1,0 +1,926 @@
+// Sub-kernel launcher and the plan/execute half of the C ABI.
+//
+// The paper enforces its schedule "by slightly modifying the source code" so that each
+// sub-kernel launches only its subset of blocks.  Here a sub-kernel is a
+// launch of the op's kernel over a 1-D grid whose blocks map to a list of <= 4 block
+// rects (kernel parameter), so a ragged Alg. 2 fragment is still one launch.  The
+// inter-launch gap the paper measures is removed by:
+//   GRAPH       the launch sequence captured once into a CUDA graph (one host call);
+//   PF_PDL      programmatic dependent launch: the next sub-kernel's CTAs are scheduled
+//               while the previous one drains and wait in griddepcontrol.wait;
+//   PERSISTENT  one launch; CTAs take tiles in schedule order from an atomic ticket and
+//               wait on per-block completion flags (acquire/release at gpu scope) —
+//               deadlock-free because producers always precede consumers in the order.
+// Dead intermediate lines (last reader done) are dropped from L2 with discard.global.L2
+// (no write-back): as the prologue of the next launch (stream/graph modes) or by the
+// last reader tile (persistent mode).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstdlib>
+#include <cstring>
+
+#include "kernels.cuh"
+#include "kt_internal.h"
+
+namespace kt {
+Graph* graph_of(ktiler_graph_t g);
+}
+
+namespace {
+
+using ktd::DBuf;
+constexpr int MAXR = 4, MAXD = 4;
+constexpr int PERSIST_THREADS = 256;
+constexpr int MAXDEAD = 64;
+constexpr int PERSIST_MINB_DEFAULT = 3;
+
+struct LRect {
+  int32_t x0, y0, z0, x1, y1, z1;
+};
+struct DRect {  // whole 128-B lines: row r -> base + z*fs + y*pitch + lb0 + k*128, k < lpr
+  uint8_t* base;
+  int64_t pitch, fstride, lb0, lpr;
+  int32_t y0, y1, z0, z1;
+};
+struct KParams {
+  DBuf in, out;
+  int32_t tw, th;
+  float T;
+  int32_t nrect, ndisc, pdl;
+  LRect r[MAXR];
+  int64_t rpre[MAXR + 1];
+  DRect d[MAXD];
+  int64_t dpre[MAXD + 1];
+};
+
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+__device__ __forceinline__ void do_discards(const KParams& p) {
+  const int64_t total = p.dpre[p.ndisc];
+  const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += nthr) {
+    int k = 0;
+    while (k + 1 < p.ndisc && i >= p.dpre[k + 1]) ++k;
+    const DRect& d = p.d[k];
+    int64_t j = i - p.dpre[k];
+    int64_t row = j / d.lpr, l = j % d.lpr;
+    int64_t h = d.y1 - d.y0;
+    int64_t z = d.z0 + row / h, y = d.y0 + row % h;
+    ktd::discard_line(d.base + z * d.fstride + y * d.pitch + d.lb0 + 128 * l);
+  }
+}
+
+template <int OP, bool SCALAR>
+__global__ void __launch_bounds__(256) op_kernel(const __grid_constant__ KParams p) {
+  if (p.pdl) pdl_wait();
+  if (p.ndisc) do_discards(p);
+  if (p.pdl) pdl_launch();
+  int64_t lin = blockIdx.x;
+  if (lin >= p.rpre[p.nrect]) return;  // discard-only CTAs
+  int k = 0;
+  while (k + 1 < p.nrect && lin >= p.rpre[k + 1]) ++k;
+  const LRect& r = p.r[k];
+  lin -= p.rpre[k];
+  const int64_t w = r.x1 - r.x0, h = r.y1 - r.y0;
+  const int64_t bx = r.x0 + lin % w, by = r.y0 + (lin / w) % h, bz = r.z0 + lin / (w * h);
+  ktd::Tile t;
+  t.z = bz;
+  t.x0 = p.tw * bx;
+  t.y0 = p.th * by;
+  t.x1 = min(t.x0 + p.tw, p.out.W);
+  t.y1 = min(t.y0 + p.th, p.out.H);
+  const int nt = blockDim.x * blockDim.y * blockDim.z;
+  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  extern __shared__ __align__(16) uint8_t ktsm[];
+  ktd::run_tile(OP, SCALAR, p.in, p.out, t, p.T, nt, tid, ktsm);
+}
+
+__global__ void discard_kernel(const __grid_constant__ KParams p) {
+  if (p.pdl) pdl_wait();
+  do_discards(p);
+  if (p.pdl) pdl_launch();
+}
+
+// ------------------------------------------------------------------------------------
+// persistent executor
+// ------------------------------------------------------------------------------------
+struct PNode {
+  DBuf in, out;
+  int32_t op, scalar, tw, th;
+  float T;
+  int32_t gx, gy;
+  int64_t flag0;
+  int32_t pu, disc_in;
+  int64_t rax, ray, rox, roy;
+  int32_t rhl, rhr, rht, rhb;
+  int64_t wax, way;
+  int32_t pgx, pgy;
+  int64_t pflag0;
+  const uint8_t* expect;  // per producer block: number of reader blocks
+  int64_t ptw, pth;       // producer output tile (for discards)
+};
+struct PCtrl {
+  unsigned int ticket, done, epoch, pad;
+};
+// Tile descriptor of ticket t: node (4 bits) | bz (12) | by (24) | bx (24).
+__host__ __device__ inline uint64_t pack_tile(uint64_t node, uint64_t bx, uint64_t by, uint64_t bz) {
+  return (node << 60) | (bz << 48) | (by << 24) | bx;
+}
+struct PParams {
+  const PNode* nodes;
+  const uint64_t* desc;  // one descriptor per ticket, in schedule order
+  int32_t discard;
+  int32_t pad;
+  int64_t total;
+  unsigned int* flags;
+  unsigned int* rc;
+  PCtrl* ctrl;
+  int64_t stage_bytes;  // one staging buffer (the kernel double-buffers)
+};
+
+__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void hit(int64_t a, int64_t o, int64_t hl, int64_t hr, int64_t lo, int64_t hi, int64_t n,
+                                    int64_t& i0, int64_t& i1) {
+  auto fd = [](int64_t x, int64_t b) { int64_t q = x / b; return (x % b != 0 && x < 0) ? q - 1 : q; };
+  i0 = max((int64_t)0, fd(lo - o - hr, a));
+  i1 = min(n, fd(hi - o + hl - 1, a) + 1);
+  if (i1 < i0) i1 = i0;
+}
+
+
+// Decoded ticket: node, block, its output rect, and the producer-block range of its read
+// footprint (the closed-form dependency of the affine maps).
+struct TInfo {
+  const PNode* nd;
+  ktd::Tile t;
+  int64_t bx, by, px0, py0, pw, ndep;
+};
+
+__device__ __forceinline__ TInfo decode(const PParams& p, uint64_t dsc) {
+  TInfo r;
+  r.nd = p.nodes + (dsc >> 60);
+  const PNode& nd = *r.nd;
+  const int64_t bz = (dsc >> 48) & 0xFFF;
+  r.by = (dsc >> 24) & 0xFFFFFF;
+  r.bx = dsc & 0xFFFFFF;
+  r.t.z = bz;
+  r.t.x0 = nd.tw * r.bx;
+  r.t.y0 = nd.th * r.by;
+  r.t.x1 = min(r.t.x0 + nd.tw, nd.out.W);
+  r.t.y1 = min(r.t.y0 + nd.th, nd.out.H);
+  int64_t px0 = 0, px1 = 0, py0 = 0, py1 = 0;
+  if (nd.pu >= 0) {
+    int64_t rx0 = max((int64_t)0, nd.rax * r.bx + nd.rox - nd.rhl), rx1 = min(nd.in.W, nd.rax * (r.bx + 1) + nd.rox + nd.rhr);
+    int64_t ry0 = max((int64_t)0, nd.ray * r.by + nd.roy - nd.rht), ry1 = min(nd.in.H, nd.ray * (r.by + 1) + nd.roy + nd.rhb);
+    hit(nd.wax, 0, 0, 0, rx0, rx1, nd.pgx, px0, px1);
+    hit(nd.way, 0, 0, 0, ry0, ry1, nd.pgy, py0, py1);
+  }
+  r.px0 = px0;
+  r.py0 = py0;
+  r.pw = px1 - px0;
+  r.ndep = r.pw * (py1 - py0);
+  return r;
+}
+
+__device__ __forceinline__ const unsigned int* dep_flag(const PParams& p, const TInfo& a, int64_t i) {
+  const PNode& nd = *a.nd;
+  return p.flags + nd.pflag0 + (a.t.z * nd.pgy + a.py0 + i / a.pw) * nd.pgx + a.px0 + i % a.pw;
+}
+
+// Blocking wait for all producer blocks of a (every thread polls its share), then barrier.
+__device__ __forceinline__ void wait_deps(const PParams& p, const TInfo& a, unsigned epoch, int nt, int tid) {
+  for (int64_t i = tid; i < a.ndep; i += nt) {
+    const unsigned int* f = dep_flag(p, a, i);
+    while (ld_acquire(f) != epoch) __nanosleep(32);
+  }
+  __syncthreads();
+}
+
+// One non-blocking poll of a's producer flags; CTA-uniform result.
+__device__ __forceinline__ bool probe_deps(const PParams& p, const TInfo& a, unsigned epoch, int nt, int tid) {
+  int ok = 1;
+  for (int64_t i = tid; i < a.ndep; i += nt) ok &= (ld_acquire(dep_flag(p, a, i)) == epoch);
+  return __syncthreads_and(ok) != 0;
+}
+
+__device__ __forceinline__ void stage_any(const TInfo& a, uint8_t* sm, int nt, int tid) {
+  if (!a.nd->scalar) ktd::stage_tile(a.nd->op, a.nd->in, a.t, sm, nt, tid);
+}
+
+// Software-pipelined persistent executor.  Per CTA: while tile A is computed from shared
+// buffer `cur`, the input of the next tile B is already streaming into the other buffer
+// (cp.async), provided B's producers are complete (non-blocking probe); otherwise B is
+// staged after A is released, so a CTA never waits on a tile it has not released itself.
+// The ticket queue (A, B, C) lives in shared memory and thread 0 refills it one tile
+// ahead, so no atomic or descriptor load is ever waited on and nothing but the buffer
+// index stays live across a tile's arithmetic.  Deadlock freedom: tickets are taken in
+// schedule order, each CTA processes its tickets in increasing order and producers
+// precede consumers, so the smallest unfinished ticket is always runnable.
+struct PQueue {
+  int64_t tk[3];    // A, B, C
+  uint64_t dsc[3];
+  int64_t fut;      // thread 0's next grab (its descriptor is loaded one tile later)
+  int ndead;
+  int readyB;
+};
+
+__device__ __forceinline__ void release_and_discard(const PParams& p, const TInfo& a, unsigned epoch, PQueue& q,
+                                                    int64_t* dead, int nt, int tid) {
+  const PNode& nd = *a.nd;
+  if (tid == 0) {
+    __threadfence();
+    st_release(p.flags + nd.flag0 + (a.t.z * nd.gy + a.by) * nd.gx + a.bx, epoch);
+  }
+  if (!(p.discard && nd.disc_in)) return;
+  // last reader of a producer block drops its lines from L2 (no write-back)
+  for (int64_t i = tid; i < a.ndep; i += nt) {
+    const int64_t pl = (a.t.z * nd.pgy + a.py0 + i / a.pw) * nd.pgx + a.px0 + i % a.pw;
+    unsigned int old = atomicAdd(p.rc + nd.pflag0 + pl, 1u);
+    if (old + 1 == nd.expect[pl]) {
+      p.rc[nd.pflag0 + pl] = 0;
+      int k = atomicAdd(&q.ndead, 1);
+      if (k < MAXDEAD) dead[k] = pl;
+    }
+  }
+  __syncthreads();
+  const int nd_dead = min(q.ndead, MAXDEAD);
+  const int64_t eb = nd.op == 4 ? 4 : 1;  // element bytes of the producer output (= our input)
+  for (int k = 0; k < nd_dead; ++k) {
+    const int64_t pl = dead[k];
+    const int64_t qx = pl % nd.pgx, qy = (pl / nd.pgx) % nd.pgy;
+    const int64_t ax0 = nd.ptw * qx, ax1 = min(ax0 + nd.ptw, nd.in.W);
+    const int64_t ay0 = nd.pth * qy, ay1 = min(ay0 + nd.pth, nd.in.H);
+    const uint64_t fb = (uint64_t)(nd.in.p + a.t.z * nd.in.fstride);
+    // lines fully inside [ax0*eb, ax1*eb) of each row (the buffer pitch is a multiple of 128)
+    const int64_t l0 = (ax0 * eb + 127) >> 7, l1 = (ax1 * eb) >> 7, lpr = l1 > l0 ? l1 - l0 : 0;
+    const int64_t n = lpr * (ay1 - ay0);
+    for (int64_t j = tid; j < n; j += nt) {
+      const int64_t yy = ay0 + j / lpr, l = l0 + j % lpr;
+      ktd::discard_line((const void*)(fb + yy * nd.in.pitch + 128 * l));
+    }
+  }
+}
+
+template <int MINB>
+__global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const __grid_constant__ PParams p) {
+  __shared__ PQueue q;
+  __shared__ unsigned int s_epoch;
+  __shared__ int64_t s_dead[MAXDEAD];
+  extern __shared__ __align__(16) uint8_t ktsm[];
+  const int nt = blockDim.x, tid = threadIdx.x;
+  if (tid == 0) {
+    s_epoch = *(volatile unsigned int*)&p.ctrl->epoch;
+    for (int k = 0; k < 3; ++k) {
+      const int64_t t = atomicAdd(&p.ctrl->ticket, 1u);
+      q.tk[k] = t;
+      q.dsc[k] = t < p.total ? p.desc[t] : 0;
+    }
+    q.fut = q.tk[2] < p.total ? (int64_t)atomicAdd(&p.ctrl->ticket, 1u) : p.total;
+  }
+  __syncthreads();
+  const unsigned int epoch = s_epoch;
+  int cur = 0;
+  if (q.tk[0] < p.total) {
+    const TInfo a = decode(p, q.dsc[0]);
+    wait_deps(p, a, epoch, nt, tid);
+    stage_any(a, ktsm, nt, tid);
+  }
+  ktd::cp_async_commit();
+  while (q.tk[0] < p.total) {
+    uint8_t* const bufA = ktsm + (cur ? p.stage_bytes : 0);
+    uint8_t* const bufB = ktsm + (cur ? 0 : p.stage_bytes);
+    // ---- start B's staging if its producers are done ----
+    bool readyB = false;
+    if (q.tk[1] < p.total) {
+      const TInfo b = decode(p, q.dsc[1]);
+      readyB = probe_deps(p, b, epoch, nt, tid);
+      if (readyB) stage_any(b, bufB, nt, tid);
+    }
+    ktd::cp_async_commit();
+    // ---- thread 0: grab the ticket behind C (lands in q.fut while A computes) ----
+    int64_t fut = p.total;
+    uint64_t fdsc = 0;
+    if (tid == 0 && q.fut < p.total) {
+      fut = atomicAdd(&p.ctrl->ticket, 1u);
+      fdsc = p.desc[q.fut];
+    }
+    // ---- compute A ----
+    ktd::cp_async_wait<1>();
+    __syncthreads();
+    {
+      const TInfo a = decode(p, q.dsc[0]);
+      const PNode& nd = *a.nd;
+      if (nd.scalar) ktd::scalar_tile(nd.op, nd.in, nd.out, a.t, nd.T, nt, tid);
+      else ktd::compute_tile(nd.op, nd.out, a.t, bufA, nd.T, nt, tid);
+    }
+    if (tid == 0) q.ndead = 0;
+    __syncthreads();
+    release_and_discard(p, decode(p, q.dsc[0]), epoch, q, s_dead, nt, tid);
+    __syncthreads();
+    // ---- shift the queue: B -> A, C -> B, fut -> C ----
+    if (tid == 0) {
+      const int64_t c = q.fut;
+      q.tk[0] = q.tk[1]; q.dsc[0] = q.dsc[1];
+      q.tk[1] = q.tk[2]; q.dsc[1] = q.dsc[2];
+      q.tk[2] = c;       q.dsc[2] = fdsc;
+      q.fut = fut;
+      q.readyB = readyB;
+    }
+    __syncthreads();
+    if (q.tk[0] < p.total && !q.readyB) {
+      const TInfo b = decode(p, q.dsc[0]);
+      wait_deps(p, b, epoch, nt, tid);
+      stage_any(b, bufB, nt, tid);
+      ktd::cp_async_commit();
+    }
+    cur ^= 1;
+  }
+  ktd::cp_async_wait<0>();
+  if (tid == 0) {
+    __threadfence();
+    unsigned int old = atomicAdd(&p.ctrl->done, 1u);
+    if (old == gridDim.x - 1) {
+      p.ctrl->ticket = 0;
+      p.ctrl->done = 0;
+      __threadfence();
+      atomicAdd(&p.ctrl->epoch, 1u);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------
+
+// ------------------------------------------------------------------------------------
+// host side
+// ------------------------------------------------------------------------------------
+typedef void (*kfn_t)(KParams);
+
+kfn_t vec_kernel(int op) {
+  switch (op) {
+    case 0: return op_kernel<0, false>;
+    case 1: return op_kernel<1, false>;
+    case 2: return op_kernel<2, false>;
+    case 3: return op_kernel<3, false>;
+    default: return op_kernel<4, false>;
+  }
+}
+kfn_t scalar_kernel(int op) {
+  switch (op) {
+    case 0: return op_kernel<0, true>;
+    case 1: return op_kernel<1, true>;
+    case 2: return op_kernel<2, true>;
+    case 3: return op_kernel<3, true>;
+    default: return op_kernel<4, true>;
+  }
+}
+
+struct Launch {
+  int node = -1;  // -1: discard-only
+  kt::Node* n = nullptr;
+  KParams kp;
+  int64_t blocks = 0;
+  dim3 block;
+  int smem = 0;
+  std::vector<int32_t> crects;  // OP_CUSTOM rect list
+};
+
+}  // namespace
+
+struct ktiler_plan_s {
+  kt::Graph g;
+  kt::Schedule s;
+  ktiler_fragment_policy pol{};
+  double plan_ms = 0;
+  std::vector<Launch> launches;
+  int device = -1;
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  // persistent state
+  void* dmem = nullptr;
+  PParams pp{};
+  int pctas = 0;
+  int psmem = 0;
+  void (*pfn)(PParams) = nullptr;
+  int64_t skew = 0;
+  bool has_custom = false;
+  ~ktiler_plan_s() {
+    if (exec) cudaGraphExecDestroy(exec);
+    if (graph) cudaGraphDestroy(graph);
+    if (dmem) cudaFree(dmem);
+  }
+};
+
+namespace {
+
+using kt::fail;
+
+DBuf dbuf(const kt::Buffer& b) {
+  return DBuf{(uint8_t*)b.d.base, b.d.width, b.d.height, b.d.pitch_bytes, b.d.frame_stride_bytes};
+}
+
+bool discardable(const kt::Buffer& b) { return (b.d.pitch_bytes % 128 == 0) && (b.d.frame_stride_bytes % 128 == 0); }
+
+DRect drect(const kt::Graph& g, const kt::Discard& d) {
+  const kt::Buffer& b = g.bufs[d.buf];
+  DRect r;
+  r.base = (uint8_t*)b.d.base;
+  r.pitch = b.d.pitch_bytes;
+  r.fstride = b.d.frame_stride_bytes;
+  r.lb0 = (d.xb0 + 127) & ~127ll;
+  int64_t lb1 = d.xb1 & ~127ll;
+  r.lpr = lb1 > r.lb0 ? (lb1 - r.lb0) / 128 : 0;
+  r.y0 = d.y0; r.y1 = d.y1; r.z0 = d.z0; r.z1 = d.z1;
+  return r;
+}
+
+void build_launches(ktiler_plan_s* P) {
+  const kt::Graph& g = P->g;
+  const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
+  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
+  std::vector<DRect> pending;
+  auto flush_disc_only = [&](size_t keep) {
+    while (pending.size() > keep) {
+      Launch L;
+      std::memset(&L.kp, 0, sizeof(L.kp));
+      L.kp.pdl = pdl;
+      size_t n = std::min<size_t>(MAXD, pending.size());
+      L.kp.ndisc = (int32_t)n;
+      L.kp.dpre[0] = 0;
+      for (size_t i = 0; i < n; ++i) {
+        L.kp.d[i] = pending[i];
+        L.kp.dpre[i + 1] = L.kp.dpre[i] + L.kp.d[i].lpr * (int64_t)(pending[i].y1 - pending[i].y0) * (pending[i].z1 - pending[i].z0);
+      }
+      pending.erase(pending.begin(), pending.begin() + n);
+      int64_t lines = L.kp.dpre[n];
+      L.blocks = std::max<int64_t>(1, std::min<int64_t>(1184, (lines + 255) / 256));
+      L.block = dim3(256);
+      P->launches.push_back(L);
+    }
+  };
+  for (size_t si = 0; si < P->s.subs.size(); ++si) {
+    const kt::SubKernel& sk = P->s.subs[si];
+    const kt::Node& n = g.nodes[sk.node];
+    if (n.op == KTILER_OP_CUSTOM) {
+      flush_disc_only(0);
+      Launch L;
+      L.node = sk.node;
+      L.n = const_cast<kt::Node*>(&n);
+      for (auto& r : sk.rects) {
+        int32_t v[6] = {r.x0, r.y0, r.z0, r.x1, r.y1, r.z1};
+        L.crects.insert(L.crects.end(), v, v + 6);
+      }
+      P->launches.push_back(L);
+    } else {
+      const kt::Access& w = n.acc[n.wacc];
+      const kt::Access& r = n.acc[n.racc];
+      for (size_t c = 0; c < sk.rects.size(); c += MAXR) {
+        if (pending.size() > (size_t)MAXD) flush_disc_only(MAXD);
+        Launch L;
+        std::memset(&L.kp, 0, sizeof(L.kp));
+        L.node = sk.node;
+        L.n = const_cast<kt::Node*>(&n);
+        L.kp.in = dbuf(g.bufs[r.buf]);
+        L.kp.out = dbuf(g.bufs[w.buf]);
+        L.kp.tw = (int32_t)w.ax;
+        L.kp.th = (int32_t)w.ay;
+        L.kp.T = n.T;
+        L.kp.pdl = pdl;
+        size_t m = std::min<size_t>(MAXR, sk.rects.size() - c);
+        L.kp.nrect = (int32_t)m;
+        L.kp.rpre[0] = 0;
+        for (size_t i = 0; i < m; ++i) {
+          const kt::Rect6& q = sk.rects[c + i];
+          L.kp.r[i] = {q.x0, q.y0, q.z0, q.x1, q.y1, q.z1};
+          L.kp.rpre[i + 1] = L.kp.rpre[i] + q.count();
+        }
+        L.blocks = L.kp.rpre[m];
+        if (c == 0 && !pending.empty()) {
+          size_t nd = std::min<size_t>(MAXD, pending.size());
+          L.kp.ndisc = (int32_t)nd;
+          L.kp.dpre[0] = 0;
+          for (size_t i = 0; i < nd; ++i) {
+            L.kp.d[i] = pending[i];
+            L.kp.dpre[i + 1] = L.kp.dpre[i] + pending[i].lpr * (int64_t)(pending[i].y1 - pending[i].y0) * (pending[i].z1 - pending[i].z0);
+          }
+          pending.erase(pending.begin(), pending.begin() + nd);
+        }
+        L.block = dim3(n.block[0], n.block[1], n.block[2]);
+        L.smem = n.scalar ? 0 : ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay);
+        P->launches.push_back(L);
+      }
+    }
+    if (disc)
+      for (auto& d : P->s.discards[si]) {
+        if (!discardable(g.bufs[d.buf])) continue;
+        DRect dr = drect(g, d);
+        if (dr.lpr > 0) pending.push_back(dr);
+      }
+  }
+  flush_disc_only(0);
+}
+
+ktiler_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(KTILER_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
+  for (auto& L : P->launches) {
+    if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
+      L.n->launch(L.n->user, L.crects.data(), (int32_t)(L.crects.size() / 6), (void*)st);
+      continue;
+    }
+    kfn_t fn = L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
+    int64_t grid = std::max<int64_t>(L.blocks, 1);
+    if (L.kp.ndisc) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = L.block;
+    cfg.dynamicSmemBytes = (size_t)L.smem;
+    if (L.smem > 48 * 1024) {
+      cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
+      if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
+    }
+    cfg.stream = st;
+    cudaLaunchAttribute attr[2];
+    int na = 0;
+    if (L.kp.pdl) {
+      attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[na].val.programmaticStreamSerializationAllowed = 1;
+      ++na;
+    }
+    if (P->pol.exec_mode == KTILER_EXEC_GRAPH_PERSIST_L2 && L.node >= 0) {
+      // the sub-kernel's output region persists in L2 for its consumer; input streams
+      const DBuf& o = L.kp.out;
+      const LRect& r0 = L.kp.r[0];
+      const LRect& r1 = L.kp.r[L.kp.nrect - 1];
+      int64_t eb = L.n->op == 3 ? 4 : 1;
+      uint64_t lo = (uint64_t)(o.p + r0.z0 * o.fstride + (int64_t)r0.y0 * L.kp.th * o.pitch);
+      uint64_t hi = (uint64_t)(o.p + (r1.z1 - 1) * o.fstride + std::min<int64_t>((int64_t)r1.y1 * L.kp.th, o.H) * o.pitch);
+      (void)eb;
+      attr[na].id = cudaLaunchAttributeAccessPolicyWindow;
+      attr[na].val.accessPolicyWindow.base_ptr = (void*)lo;
+      attr[na].val.accessPolicyWindow.num_bytes = (size_t)std::min<uint64_t>(hi - lo, 64ull << 20);
+      attr[na].val.accessPolicyWindow.hitRatio = 1.0f;
+      attr[na].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      attr[na].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      ++na;
+    }
+    cfg.attrs = na ? attr : nullptr;
+    cfg.numAttrs = na;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, fn, L.kp);
+    if (e != cudaSuccess) return cuda_fail(e, "sub-kernel launch");
+  }
+  return KTILER_OK;
+}
+
+ktiler_status setup_persistent(ktiler_plan_s* P) {
+  const kt::Graph& g = P->g;
+  const int nn = (int)g.nodes.size();
+  for (auto& n : g.nodes)
+    if (n.op == KTILER_OP_CUSTOM) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode runs built-in ops only");
+  // flags: one u32 per block of every node; rc: reader counters, same indexing
+  std::vector<int64_t> flag0(nn);
+  int64_t nflags = 0;
+  for (int v = 0; v < nn; ++v) {
+    flag0[v] = nflags;
+    nflags += g.nodes[v].nblocks;
+  }
+  // expected reader counts per producer block (u8)
+  std::vector<uint8_t> expect(nflags, 0);
+  for (int u = 0; u < nn; ++u) {
+    const kt::Node& n = g.nodes[u];
+    for (int64_t l = 0; l < n.nblocks; ++l) {
+      int64_t px = l % n.gx(), py = (l / n.gx()) % n.gy();
+      int64_t cnt = 0;
+      for (auto& c : g.out_ch[u]) {
+        kt::BRange r = g.consumers(c, px, py);
+        cnt += (r.x1 - r.x0) * (r.y1 - r.y0);
+      }
+      expect[flag0[u] + l] = (uint8_t)std::min<int64_t>(cnt, 255);
+    }
+  }
+  std::vector<PNode> pn(nn);
+  for (int v = 0; v < nn; ++v) {
+    const kt::Node& n = g.nodes[v];
+    const kt::Access& w = n.acc[n.wacc];
+    const kt::Access& r = n.acc[n.racc];
+    PNode& q = pn[v];
+    std::memset(&q, 0, sizeof(q));
+    q.in = dbuf(g.bufs[r.buf]);
+    q.out = dbuf(g.bufs[w.buf]);
+    q.op = n.op;
+    q.scalar = n.scalar;
+    q.tw = (int32_t)w.ax;
+    q.th = (int32_t)w.ay;
+    q.T = n.T;
+    q.gx = (int32_t)n.gx();
+    q.gy = (int32_t)n.gy();
+    q.flag0 = flag0[v];
+    q.pu = -1;
+    for (auto& c : g.in_ch[v]) {
+      const kt::Node& u = g.nodes[c.u];
+      const kt::Access& uw = u.acc[c.w];
+      q.pu = c.u;
+      q.rax = r.ax; q.ray = r.ay; q.rox = r.ox; q.roy = r.oy;
+      q.rhl = r.hl; q.rhr = r.hr; q.rht = r.ht; q.rhb = r.hb;
+      q.wax = uw.ax; q.way = uw.ay;
+      q.pgx = (int32_t)u.gx(); q.pgy = (int32_t)u.gy();
+      q.pflag0 = flag0[c.u];
+      q.ptw = uw.ax; q.pth = uw.ay;
+      const kt::Buffer& ib = g.bufs[c.buf];
+      q.disc_in = (ib.d.flags & KTILER_BUF_INTERNAL) && discardable(ib);
+    }
+  }
+  int nsm = 0, occ = 0;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+  {
+    // registers vs CTAs per SM (KTILER_PERSIST_MINB = 2, 3 or 4 minimum resident CTAs)
+    const char* ev = getenv("KTILER_PERSIST_MINB");
+    int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
+    P->pfn = mb >= 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>);
+  }
+  P->psmem = 0;
+  for (auto& n : g.nodes) {
+    const kt::Access& w = n.acc[n.wacc];
+    if (!n.scalar) P->psmem = std::max(P->psmem, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
+  }
+  P->pp.stage_bytes = P->psmem;
+  P->psmem *= 2;
+  if (P->psmem > 48 * 1024) {
+    cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
+    if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
+  }
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, P->pfn, PERSIST_THREADS, P->psmem);
+  P->pctas = P->pol.persistent_ctas > 0 ? P->pol.persistent_ctas : nsm * std::max(1, occ);
+  // Ticket order.  skew < 0: the emitted (fragment-major) order.  skew = k > 0: software
+  // pipeline over fragments — the sub-kernel of fragment f at node depth d is issued at
+  // step f + d*k, deepest node first within a step.  A consumer's producers sit in
+  // fragments <= f at smaller depth, hence at strictly earlier steps: still a valid total
+  // order, and about k fragments of tiles separate a tile from its
+  // producers, so a CTA rarely waits.
+  std::vector<int> depth(nn, 0);
+  int dmax = 0;
+  for (int v : g.topo)
+    for (auto& c : g.in_ch[v]) depth[v] = std::max(depth[v], depth[c.u] + 1);
+  for (int v = 0; v < nn; ++v) dmax = std::max(dmax, depth[v]);
+  const int64_t nfrag = P->s.nfrag;
+  std::vector<std::vector<int>> by_frag(nfrag, std::vector<int>(nn, -1));
+  int64_t tiles = 0;
+  for (size_t i = 0; i < P->s.subs.size(); ++i) {
+    by_frag[P->s.subs[i].frag][P->s.subs[i].node] = (int)i;
+    tiles += P->s.subs[i].nblocks;
+  }
+  int64_t k = P->pol.pipeline_skew;
+  if (k == 0) {
+    int64_t per_frag = std::max<int64_t>(1, tiles / std::max<int64_t>(1, nfrag));
+    k = std::max<int64_t>(1, (3 * (int64_t)P->pctas + 2 * per_frag - 1) / (2 * per_frag));
+  }
+  P->skew = k;
+  std::vector<int> order;
+  if (k < 0) {
+    for (size_t i = 0; i < P->s.subs.size(); ++i) order.push_back((int)i);
+  } else {
+    std::vector<int> rtopo(g.topo.rbegin(), g.topo.rend());
+    for (int64_t s = 0; s < nfrag + dmax * k; ++s)
+      for (int v : rtopo) {
+        int64_t f = s - depth[v] * k;
+        if (f >= 0 && f < nfrag && by_frag[f][v] >= 0) order.push_back(by_frag[f][v]);
+      }
+  }
+  // per-ticket tile descriptors, in ticket order (blocks of one sub-kernel in rect order)
+  std::vector<uint64_t> desc;
+  desc.reserve(tiles);
+  for (int oi : order) {
+    const kt::SubKernel& sk = P->s.subs[oi];
+    if (g.nodes[sk.node].gz() > 4096 || g.nodes[sk.node].gy() >= (1 << 24) || g.nodes[sk.node].gx() >= (1 << 24) || nn > 16)
+      return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: grid exceeds the tile descriptor (16 nodes, 4096 frames, 2^24 blocks per axis)");
+    for (auto& r : sk.rects)
+      for (int64_t z = r.z0; z < r.z1; ++z)
+        for (int64_t y = r.y0; y < r.y1; ++y)
+          for (int64_t x = r.x0; x < r.x1; ++x) desc.push_back(pack_tile(sk.node, x, y, z));
+  }
+  const int64_t t0 = (int64_t)desc.size();
+  // one device allocation: ctrl | flags | rc | expect | nodes | desc
+  auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  size_t o_ctrl = 0, o_flags = al(sizeof(PCtrl)), o_rc = o_flags + al(nflags * 4), o_exp = o_rc + al(nflags * 4);
+  size_t o_nodes = o_exp + al(nflags), o_desc = o_nodes + al(pn.size() * sizeof(PNode));
+  size_t total = o_desc + al(desc.size() * sizeof(uint64_t));
+  char* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, total);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (persistent tables)");
+  P->dmem = d;
+  for (auto& q : pn) q.expect = (const uint8_t*)(d + o_exp) + q.pflag0;
+  PCtrl c0{0, 0, 1, 0};
+  if ((e = cudaMemset(d, 0, total)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
+  cudaMemcpy(d + o_ctrl, &c0, sizeof(c0), cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_exp, expect.data(), expect.size(), cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_nodes, pn.data(), pn.size() * sizeof(PNode), cudaMemcpyHostToDevice);
+  if ((e = cudaMemcpy(d + o_desc, desc.data(), desc.size() * sizeof(uint64_t), cudaMemcpyHostToDevice)) != cudaSuccess)
+    return cuda_fail(e, "cudaMemcpy (persistent tables)");
+  // expect for nodes is indexed by the producer's local id: expect base + pflag0 was set
+  // above; the kernel adds the producer-local index.
+  P->pp.nodes = (const PNode*)(d + o_nodes);
+  P->pp.desc = (const uint64_t*)(d + o_desc);
+  P->pp.discard = (P->pol.flags & KTILER_PF_DISCARD_DEAD) ? 1 : 0;
+  P->pp.total = t0;
+  P->pp.flags = (unsigned int*)(d + o_flags);
+  P->pp.rc = (unsigned int*)(d + o_rc);
+  P->pp.ctrl = (PCtrl*)(d + o_ctrl);
+  return KTILER_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fragment_policy* pol, ktiler_plan_t* out) {
+  if (!gh || !pol || !out) return fail(KTILER_E_INVALID, "NULL argument");
+  *out = nullptr;
+  kt::Graph* G = kt::graph_of(gh);
+  ktiler_status s = G->finalize();
+  if (s) return s;
+  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_PERSISTENT)
+    return fail(KTILER_E_INVALID, "unknown exec_mode");
+  if (cache_bytes == 0) {
+    int dev = 0, l2 = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    if (e != cudaSuccess || l2 <= 0) return cuda_fail(e, "cache_bytes = 0 needs a CUDA device to query the L2 size");
+    cache_bytes = (size_t)l2;
+  }
+  auto t0 = std::chrono::steady_clock::now();
+  ktiler_plan_s* P = nullptr;
+  try {
+    P = new ktiler_plan_s();
+    P->g = *G;
+    P->pol = *pol;
+    s = kt::build_schedule(P->g, (int64_t)cache_bytes, *pol, P->s);
+    if (s) {
+      delete P;
+      return s;
+    }
+    kt::compute_discards(P->g, P->s);
+    build_launches(P);
+  } catch (const std::bad_alloc&) {
+    delete P;
+    return fail(KTILER_E_NOMEM, "host allocation failed while planning");
+  }
+  P->plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  for (auto& n : P->g.nodes) P->has_custom |= (n.op == KTILER_OP_CUSTOM);
+  *out = P;
+  kt::clear_error();
+  return KTILER_OK;
+}
+
+void ktiler_plan_destroy(ktiler_plan_t p) { delete p; }
+
+ktiler_status ktiler_plan_num_subkernels(ktiler_plan_t p, int64_t* n) {
+  if (!p || !n) return fail(KTILER_E_INVALID, "NULL argument");
+  *n = (int64_t)p->s.subs.size();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_num_fragments(ktiler_plan_t p, int64_t* n) {
+  if (!p || !n) return fail(KTILER_E_INVALID, "NULL argument");
+  *n = p->s.nfrag;
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_get_subkernel(ktiler_plan_t p, int64_t i, ktiler_subkernel* out, int32_t* rects, int32_t cap) {
+  if (!p || !out) return fail(KTILER_E_INVALID, "NULL argument");
+  if (i < 0 || i >= (int64_t)p->s.subs.size()) return fail(KTILER_E_INVALID, "sub-kernel index out of range");
+  const kt::SubKernel& sk = p->s.subs[i];
+  out->node = sk.node;
+  out->fragment = sk.frag;
+  out->n_blocks = sk.nblocks;
+  out->n_rects = (int32_t)sk.rects.size();
+  out->pad = 0;
+  out->footprint_bytes = sk.footprint;
+  if (rects)
+    for (int32_t k = 0; k < cap && k < (int32_t)sk.rects.size(); ++k) {
+      const kt::Rect6& r = sk.rects[k];
+      int32_t v[6] = {r.x0, r.y0, r.z0, r.x1, r.y1, r.z1};
+      std::memcpy(rects + 6 * k, v, sizeof(v));
+    }
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_get_stats(ktiler_plan_t p, ktiler_plan_stats* out) {
+  if (!p || !out) return fail(KTILER_E_INVALID, "NULL argument");
+  std::memset(out, 0, sizeof(*out));
+  out->n_subkernels = (int64_t)p->s.subs.size();
+  out->n_fragments = p->s.nfrag;
+  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT ? 1 : (int64_t)p->launches.size();
+  out->n_discard_lines = (p->pol.flags & KTILER_PF_DISCARD_DEAD) ? p->s.discard_lines : 0;
+  out->budget_bytes = p->s.budget;
+  out->max_footprint_bytes = p->s.max_footprint;
+  out->plan_ms = p->plan_ms;
+  out->exec_mode = p->pol.exec_mode;
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
+  if (!p) return fail(KTILER_E_INVALID, "NULL plan");
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e;
+  if (p->device < 0) {
+    if ((e = cudaGetDevice(&p->device)) != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    if (p->pol.exec_mode == KTILER_EXEC_GRAPH_PERSIST_L2) {
+      int maxp = 0;
+      cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, p->device);
+      if (maxp > 0) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp);
+    }
+    if (p->pol.exec_mode == KTILER_EXEC_PERSISTENT) {
+      ktiler_status s = setup_persistent(p);
+      if (s) return s;
+    }
+  }
+  switch (p->pol.exec_mode) {
+    case KTILER_EXEC_STREAM: {
+      ktiler_status s = enqueue(p, st);
+      if (s) return s;
+      break;
+    }
+    case KTILER_EXEC_GRAPH:
+    case KTILER_EXEC_GRAPH_PERSIST_L2: {
+      if (!p->exec) {
+        cudaStream_t cs;
+        if ((e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking)) != cudaSuccess) return cuda_fail(e, "cudaStreamCreate");
+        if ((e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal)) != cudaSuccess) {
+          cudaStreamDestroy(cs);
+          return cuda_fail(e, "cudaStreamBeginCapture");
+        }
+        ktiler_status s = enqueue(p, cs);
+        cudaGraph_t gr = nullptr;
+        cudaError_t e2 = cudaStreamEndCapture(cs, &gr);
+        cudaStreamDestroy(cs);
+        if (s) {
+          if (gr) cudaGraphDestroy(gr);
+          return s;
+        }
+        if (e2 != cudaSuccess) return cuda_fail(e2, "cudaStreamEndCapture");
+        p->graph = gr;
+        if ((e = cudaGraphInstantiate(&p->exec, gr, 0)) != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+      }
+      if ((e = cudaGraphLaunch(p->exec, st)) != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
+      break;
+    }
+    case KTILER_EXEC_PERSISTENT: {
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3((unsigned)p->pctas);
+      cfg.blockDim = dim3(PERSIST_THREADS);
+      cfg.dynamicSmemBytes = (size_t)p->psmem;
+      cfg.stream = st;
+      if ((e = cudaLaunchKernelEx(&cfg, p->pfn, p->pp)) != cudaSuccess) return cuda_fail(e, "persistent launch");
+      break;
+    }
+  }
+  if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "launch");
+  kt::clear_error();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_execute_host(ktiler_plan_t p, const ktiler_host_copy* in, int32_t nin, const ktiler_host_copy* outc,
+                                  int32_t nout, void* stream) {
+  if (!p) return fail(KTILER_E_INVALID, "NULL plan");
+  cudaStream_t st = (cudaStream_t)stream;
+  auto copy = [&](const ktiler_host_copy& c, bool h2d) -> ktiler_status {
+    if (c.buf_id < 0 || c.buf_id >= (int32_t)p->g.bufs.size()) return fail(KTILER_E_INVALID, "host copy buffer id out of range");
+    const kt::Buffer& b = p->g.bufs[c.buf_id];
+    int64_t f0 = c.frame0, nf = c.frames ? c.frames : b.d.frames - f0;
+    if (f0 < 0 || f0 + nf > b.d.frames || !c.host) return fail(KTILER_E_INVALID, "host copy frame range");
+    const int64_t rowb = b.d.width * b.d.elem_bytes;
+    for (int64_t z = f0; z < f0 + nf; ++z) {
+      char* dev = (char*)b.d.base + z * b.d.frame_stride_bytes;
+      char* host = (char*)c.host + (z - f0) * rowb * b.d.height;
+      cudaError_t e = h2d ? cudaMemcpy2DAsync(dev, b.d.pitch_bytes, host, rowb, rowb, b.d.height, cudaMemcpyHostToDevice, st)
+                          : cudaMemcpy2DAsync(host, rowb, dev, b.d.pitch_bytes, rowb, b.d.height, cudaMemcpyDeviceToHost, st);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMemcpy2DAsync");
+    }
+    return KTILER_OK;
+  };
+  for (int i = 0; i < nin; ++i) {
+    ktiler_status s = copy(in[i], true);
+    if (s) return s;
+  }
+  ktiler_status s = ktiler_execute(p, stream);
+  if (s) return s;
+  for (int i = 0; i < nout; ++i) {
+    s = copy(outc[i], false);
+    if (s) return s;
+  }
+  return KTILER_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,268 @@
+"""Thin ctypes binding of libktiler.so (include/ktiler.h) — argument marshalling only.
+
+Every step of the hot path (planning, dependency analysis, partitioning, emission,
+launching, the kernels themselves) runs inside libktiler.so.  There is no Python or
+CPU fallback: if the shared library is missing this module raises on import of the
+library, and every ABI error is raised as KtilerError with the library's message.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libktiler.so")
+
+# ---- enums (mirror include/ktiler.h) ----
+OK, E_INVALID, E_CYCLE, E_UNTILEABLE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = range(8)
+BUF_INTERNAL = 1
+READ, WRITE = 1, 2
+OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM = range(6)
+FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE = range(4)
+EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT = range(4)
+PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL = 1, 2, 4
+
+EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
+              "persistent": EXEC_PERSISTENT}
+FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE}
+
+
+class KtilerError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        self.status = status
+        super().__init__(f"{_status_name(status)}: {msg}")
+
+
+class BufferDesc(ctypes.Structure):
+    _fields_ = [("base", ctypes.c_void_p), ("width", ctypes.c_int64), ("height", ctypes.c_int64),
+                ("frames", ctypes.c_int64), ("pitch_bytes", ctypes.c_int64), ("frame_stride_bytes", ctypes.c_int64),
+                ("elem_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+
+
+class Access(ctypes.Structure):
+    _fields_ = [("buf_id", ctypes.c_int32), ("mode", ctypes.c_int32), ("ax", ctypes.c_int64), ("ay", ctypes.c_int64),
+                ("ox", ctypes.c_int64), ("oy", ctypes.c_int64), ("halo_l", ctypes.c_int32),
+                ("halo_r", ctypes.c_int32), ("halo_t", ctypes.c_int32), ("halo_b", ctypes.c_int32)]
+
+
+LAUNCH_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.POINTER(ctypes.c_int32), ctypes.c_int32, ctypes.c_void_p)
+
+
+class KernelDesc(ctypes.Structure):
+    _fields_ = [("op", ctypes.c_int32), ("grid", ctypes.c_uint32 * 3), ("block", ctypes.c_uint32 * 3),
+                ("n_access", ctypes.c_int32), ("access", ctypes.POINTER(Access)), ("params", ctypes.c_void_p),
+                ("params_bytes", ctypes.c_size_t), ("launch", LAUNCH_FN), ("user", ctypes.c_void_p)]
+
+
+class Policy(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("l2_fraction", ctypes.c_double), ("rows", ctypes.c_int64),
+                ("exec_mode", ctypes.c_int32), ("flags", ctypes.c_uint32), ("persistent_ctas", ctypes.c_int32),
+                ("pipeline_skew", ctypes.c_int32)]
+
+
+class SubKernelInfo(ctypes.Structure):
+    _fields_ = [("node", ctypes.c_int32), ("fragment", ctypes.c_int32), ("n_blocks", ctypes.c_int64),
+                ("n_rects", ctypes.c_int32), ("pad", ctypes.c_int32), ("footprint_bytes", ctypes.c_int64)]
+
+
+class PlanStats(ctypes.Structure):
+    _fields_ = [("n_subkernels", ctypes.c_int64), ("n_fragments", ctypes.c_int64), ("n_launches", ctypes.c_int64),
+                ("n_discard_lines", ctypes.c_int64), ("budget_bytes", ctypes.c_int64),
+                ("max_footprint_bytes", ctypes.c_int64), ("plan_ms", ctypes.c_double), ("exec_mode", ctypes.c_int32),
+                ("pad", ctypes.c_int32)]
+
+
+class HostCopy(ctypes.Structure):
+    _fields_ = [("buf_id", ctypes.c_int32), ("pad", ctypes.c_int32), ("host", ctypes.c_void_p),
+                ("frame0", ctypes.c_int64), ("frames", ctypes.c_int64)]
+
+
+EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktiler_graph_create",
+           "ktiler_graph_destroy", "ktiler_add_buffer", "ktiler_add_kernel", "ktiler_add_edge",
+           "ktiler_graph_block_deps", "ktiler_graph_block_lines", "ktiler_plan", "ktiler_plan_destroy",
+           "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
+           "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host"]
+
+_LIB = None
+
+
+def lib() -> ctypes.CDLL:
+    global _LIB
+    if _LIB is not None:
+        return _LIB
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+                           "(there is no fallback path)")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i32, i64, P = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.POINTER
+    st = ctypes.c_int
+    sig = {
+        "ktiler_status_str": ([st], ctypes.c_char_p),
+        "ktiler_last_error": ([], ctypes.c_char_p),
+        "ktiler_abi_version": ([], i32),
+        "ktiler_graph_create": ([P(vp)], st),
+        "ktiler_graph_destroy": ([vp], None),
+        "ktiler_add_buffer": ([vp, P(BufferDesc), P(i32)], st),
+        "ktiler_add_kernel": ([vp, P(KernelDesc), P(i32)], st),
+        "ktiler_add_edge": ([vp, i32, i32, i32, ctypes.c_float], st),
+        "ktiler_graph_block_deps": ([vp, i32, i32, i32, i32, P(i32), i64, P(i64)], st),
+        "ktiler_graph_block_lines": ([vp, i32, i32, i32, i32, P(i64), i64, P(i64)], st),
+        "ktiler_plan": ([vp, ctypes.c_size_t, P(Policy), P(vp)], st),
+        "ktiler_plan_destroy": ([vp], None),
+        "ktiler_plan_num_subkernels": ([vp, P(i64)], st),
+        "ktiler_plan_num_fragments": ([vp, P(i64)], st),
+        "ktiler_plan_get_subkernel": ([vp, i64, P(SubKernelInfo), P(i32), i32], st),
+        "ktiler_plan_get_stats": ([vp, P(PlanStats)], st),
+        "ktiler_execute": ([vp, vp], st),
+        "ktiler_execute_host": ([vp, P(HostCopy), i32, P(HostCopy), i32, vp], st),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+    if L.ktiler_abi_version() != 1:
+        raise RuntimeError("libktiler ABI version mismatch")
+    _LIB = L
+    return L
+
+
+def _status_name(s: int) -> str:
+    try:
+        return lib().ktiler_status_str(s).decode()
+    except Exception:  # pragma: no cover
+        return str(s)
+
+
+def _check(s: int) -> None:
+    if s != OK:
+        raise KtilerError(s, lib().ktiler_last_error().decode())
+
+
+class Graph:
+    """Owning wrapper of a ktiler_graph_t."""
+
+    def __init__(self):
+        h = ctypes.c_void_p()
+        _check(lib().ktiler_graph_create(ctypes.byref(h)))
+        self._h = h
+        self._keep = []
+
+    def close(self):
+        if self._h:
+            lib().ktiler_graph_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def add_buffer(self, base: int, width: int, height: int, elem_bytes: int, frames: int = 1,
+                   pitch_bytes: int | None = None, frame_stride_bytes: int = 0, internal: bool = False) -> int:
+        pitch = pitch_bytes if pitch_bytes is not None else width * elem_bytes
+        d = BufferDesc(base, width, height, frames, pitch, frame_stride_bytes, elem_bytes,
+                       BUF_INTERNAL if internal else 0)
+        out = ctypes.c_int32()
+        _check(lib().ktiler_add_buffer(self._h, ctypes.byref(d), ctypes.byref(out)))
+        return out.value
+
+    def add_kernel(self, op: int, grid, block, accesses, params: bytes | None = None, launch=None) -> int:
+        acc = (Access * len(accesses))()
+        for i, a in enumerate(accesses):
+            acc[i] = Access(a["buf"], a["mode"], a["ax"], a["ay"], a.get("ox", 0), a.get("oy", 0),
+                            a.get("hl", 0), a.get("hr", 0), a.get("ht", 0), a.get("hb", 0))
+        pbuf = ctypes.create_string_buffer(params) if params else None
+        fn = LAUNCH_FN(launch) if launch is not None else LAUNCH_FN()
+        if launch is not None:
+            self._keep.append(fn)
+        d = KernelDesc(op, (ctypes.c_uint32 * 3)(*grid), (ctypes.c_uint32 * 3)(*block), len(accesses), acc,
+                       ctypes.cast(pbuf, ctypes.c_void_p) if pbuf else None, len(params) if params else 0, fn, None)
+        out = ctypes.c_int32()
+        _check(lib().ktiler_add_kernel(self._h, ctypes.byref(d), ctypes.byref(out)))
+        return out.value
+
+    def add_edge(self, src: int, dst: int, buf: int, weight: float = 1.0) -> None:
+        _check(lib().ktiler_add_edge(self._h, src, dst, buf, weight))
+
+    def block_deps(self, node: int, bx: int, by: int, bz: int = 0):
+        n = ctypes.c_int64()
+        _check(lib().ktiler_graph_block_deps(self._h, node, bx, by, bz, None, 0, ctypes.byref(n)))
+        arr = (ctypes.c_int32 * (4 * max(1, n.value)))()
+        _check(lib().ktiler_graph_block_deps(self._h, node, bx, by, bz, arr, n.value, ctypes.byref(n)))
+        return [tuple(arr[4 * i:4 * i + 4]) for i in range(n.value)]
+
+    def block_lines(self, node: int, bx: int, by: int, bz: int = 0):
+        n = ctypes.c_int64()
+        _check(lib().ktiler_graph_block_lines(self._h, node, bx, by, bz, None, 0, ctypes.byref(n)))
+        arr = (ctypes.c_int64 * max(1, n.value))()
+        _check(lib().ktiler_graph_block_lines(self._h, node, bx, by, bz, arr, n.value, ctypes.byref(n)))
+        return list(arr[:n.value])
+
+    def plan(self, cache_bytes: int = 0, kind: str | int = "budget", l2_fraction: float = 1.0, rows: int = 1,
+             exec_mode: str | int = "graph", discard: bool = False, pdl: bool = False, force_minimal: bool = False,
+             persistent_ctas: int = 0, skew: int = 0) -> "Plan":
+        k = FRAG_KINDS[kind] if isinstance(kind, str) else kind
+        m = EXEC_MODES[exec_mode] if isinstance(exec_mode, str) else exec_mode
+        flags = (PF_DISCARD_DEAD if discard else 0) | (PF_PDL if pdl else 0) | (PF_FORCE_MINIMAL if force_minimal else 0)
+        pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew)
+        h = ctypes.c_void_p()
+        _check(lib().ktiler_plan(self._h, cache_bytes, ctypes.byref(pol), ctypes.byref(h)))
+        return Plan(h, self)
+
+
+class Plan:
+    """Owning wrapper of a ktiler_plan_t.  Keeps its graph's Python objects alive (custom
+    launch callbacks)."""
+
+    def __init__(self, h, graph: Graph):
+        self._h = h
+        self._graph_keep = graph._keep
+
+    def close(self):
+        if self._h:
+            lib().ktiler_plan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def num_subkernels(self) -> int:
+        n = ctypes.c_int64()
+        _check(lib().ktiler_plan_num_subkernels(self._h, ctypes.byref(n)))
+        return n.value
+
+    def num_fragments(self) -> int:
+        n = ctypes.c_int64()
+        _check(lib().ktiler_plan_num_fragments(self._h, ctypes.byref(n)))
+        return n.value
+
+    def subkernels(self):
+        """List of dicts: node, fragment, n_blocks, footprint_bytes, rects [(x0,y0,z0,x1,y1,z1)]."""
+        out = []
+        for i in range(self.num_subkernels()):
+            info = SubKernelInfo()
+            _check(lib().ktiler_plan_get_subkernel(self._h, i, ctypes.byref(info), None, 0))
+            arr = (ctypes.c_int32 * (6 * max(1, info.n_rects)))()
+            _check(lib().ktiler_plan_get_subkernel(self._h, i, ctypes.byref(info), arr, info.n_rects))
+            out.append({"node": info.node, "fragment": info.fragment, "n_blocks": info.n_blocks,
+                        "footprint_bytes": info.footprint_bytes,
+                        "rects": [tuple(arr[6 * k:6 * k + 6]) for k in range(info.n_rects)]})
+        return out
+
+    def stats(self) -> dict:
+        s = PlanStats()
+        _check(lib().ktiler_plan_get_stats(self._h, ctypes.byref(s)))
+        return {f: getattr(s, f) for f, _ in PlanStats._fields_ if f != "pad"}
+
+    def execute(self, stream: int = 0) -> None:
+        _check(lib().ktiler_execute(self._h, ctypes.c_void_p(stream)))
+
+    def execute_host(self, inputs, outputs, stream: int = 0) -> None:
+        """inputs/outputs: lists of (buf_id, host_ptr, frame0, frames)."""
+        ci = (HostCopy * max(1, len(inputs)))(*[HostCopy(b, 0, p, f0, nf) for b, p, f0, nf in inputs])
+        co = (HostCopy * max(1, len(outputs)))(*[HostCopy(b, 0, p, f0, nf) for b, p, f0, nf in outputs])
+        _check(lib().ktiler_execute_host(self._h, ci, len(inputs), co, len(outputs), ctypes.c_void_p(stream)))

@@ -1,0 +1,223 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle,
+element by element, on the same seeded inputs.  Integer/uint8 outputs and the Sobel f32
+magnitude are compared bit for bit (every float in the canonical chain is
+exact by construction).
+
+Two tile geometries: the B200 geometry bench.py uses (pipeline.B200_GEOMETRY: 512x64 /
+256x32 tiles) and a SMALL geometry whose tiles are small enough that images of a few
+hundred pixels split into tens of fragments, so tiling, fragment edges, ragged Alg. 2
+fragments and discards are exercised at sizes the oracle finishes in seconds."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from inputs import synth  # noqa: E402
+from oracle import oracle as O  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+KEYS = ("gray", "blur", "down", "sob", "mask")
+SMALL = {"gray": (64, 16, 64), "blur": (64, 16, 64), "down": (32, 8, 64), "sobel": (32, 8, 64), "thresh": (32, 8, 64)}
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import __graft_entry__ as ge
+    ge.build()
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler
+    ktiler.lib()
+
+
+def _run(W, H, F, rgb, T=200.0, cache_bytes=0, internal=False, geometry=SMALL, **pol):
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    p = Pipeline(W, H, F, T=T, internal=internal, geometry=geometry)
+    # poison intermediates and output so a skipped block cannot pass
+    for k in KEYS:
+        p.b.store.tensors[k].fill_(0xA5)
+    p.view("rgb").copy_(torch.from_numpy(rgb))
+    plan = p.plan(cache_bytes, **pol)
+    p.run()
+    torch.cuda.synchronize()
+    out = {k: p.view(k).cpu().numpy() for k in KEYS}
+    return out, plan
+
+
+def _eq(a, b):
+    return np.array_equal(a.view(np.uint8), b.view(np.uint8))
+
+
+SIZES = [(512, 64, 1), (520, 102, 1), (1040, 256, 2), (2, 2, 1), (16, 4, 1), (34, 18, 3), (7680 // 8, 4320 // 8, 2),
+         (1552, 136, 1)]
+
+
+@pytest.mark.parametrize("W,H,F", SIZES)
+@pytest.mark.parametrize("kind", ["uniform", "scene"])
+@pytest.mark.parametrize("geo", ["b200", "small"])
+def test_each_kernel_untiled(W, H, F, kind, geo):
+    """Every kernel bit-exact: several tiles, ragged right/bottom tails, tiny images."""
+    rgb = synth.make(kind, W + H, W, H, F)
+    ref = O.pipeline(rgb, T=40.0)
+    out, _ = _run(W, H, F, rgb, T=40.0, kind="none", exec_mode="stream", geometry=None if geo == "b200" else SMALL)
+    for k in KEYS:
+        assert _eq(out[k], ref[k]), k
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+@pytest.mark.parametrize("kind", ["uniform", "scene"])
+def test_parity_seeds_tiled(seed, kind):
+    W, H, F = 1536, 320, 2
+    rgb = synth.make(kind, seed, W, H, F)
+    ref = O.pipeline(rgb, T=60.0)
+    out, plan = _run(W, H, F, rgb, T=60.0, cache_bytes=120 * 1024, kind="budget", exec_mode="graph")
+    assert plan.num_fragments() > 20
+    for k in KEYS:
+        assert _eq(out[k], ref[k]), k
+
+
+def test_closed_form_images():
+    W, H = 768, 256
+    for rgb in (synth.constant((17, 200, 3), W, H), synth.ramp(0, 1, W, H), synth.checkerboard(5, W, H),
+                synth.half_black_white(W, H)):
+        ref = O.pipeline(rgb, T=100.0)
+        out, _ = _run(W, H, 1, rgb, T=100.0, cache_bytes=100 * 1024, kind="budget", exec_mode="stream")
+        for k in KEYS:
+            assert _eq(out[k], ref[k]), k
+
+
+MODES = [
+    dict(exec_mode="stream"),
+    dict(exec_mode="graph"),
+    dict(exec_mode="graph", pdl=True),
+    dict(exec_mode="persist_l2"),
+    dict(exec_mode="persistent"),
+    dict(exec_mode="persistent", skew=-1),
+    dict(exec_mode="persistent", skew=3, persistent_ctas=7),
+]
+POLICIES = [
+    dict(kind="none"),
+    dict(kind="budget", cache_bytes=60 * 1024),
+    dict(kind="budget", cache_bytes=300 * 1024, l2_fraction=0.5),
+    dict(kind="rows", rows=1),
+    dict(kind="rows", rows=3),
+    dict(kind="balanced", cache_bytes=200 * 1024),
+]
+
+
+@pytest.mark.parametrize("mode", MODES, ids=lambda m: "-".join(f"{k}={v}" for k, v in m.items()))
+@pytest.mark.parametrize("pol", POLICIES, ids=lambda m: "-".join(f"{k}={v}" for k, v in m.items()))
+@pytest.mark.parametrize("discard", [False, True])
+def test_modes_policies(mode, pol, discard):
+    """Whole graph in every exec mode x fragment policy x discard: mask bit-exact (and all
+    intermediates when they are not discarded)."""
+    W, H, F = 1040, 230, 2
+    rgb = synth.scene(5, W, H, F)
+    ref = O.pipeline(rgb, T=50.0)
+    pol = dict(pol)
+    cb = pol.pop("cache_bytes", 1 << 20)
+    out, plan = _run(W, H, F, rgb, T=50.0, cache_bytes=cb, internal=discard, discard=discard, **mode, **pol)
+    keys = ("mask",) if discard else KEYS
+    for k in keys:
+        assert _eq(out[k], ref[k]), k
+
+
+@pytest.mark.parametrize("mode", ["graph", "persistent"])
+def test_b200_geometry_tiled(mode):
+    """The bench geometry itself, tiled into several fragments (budget just above one closure)."""
+    W, H, F = 2048, 1024, 2
+    rgb = synth.scene(17, W, H, F)
+    ref = O.pipeline(rgb, T=45.0)
+    out, plan = _run(W, H, F, rgb, T=45.0, cache_bytes=3 << 20, geometry=None, internal=True, discard=True,
+                     kind="budget", exec_mode=mode)
+    assert plan.num_fragments() >= 3
+    assert _eq(out["mask"], ref["mask"])
+
+
+def test_replay_is_idempotent():
+    """A plan executes many times (GRAPH replays, persistent epochs) with identical output."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 1024, 128, 1
+    for mode in ("graph", "persistent"):
+        p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
+        a = synth.uniform(1, W, H, F)
+        b = synth.scene(2, W, H, F)
+        p.plan(100 * 1024, kind="budget", exec_mode=mode, discard=True)
+        for it in range(6):
+            x = a if it % 2 == 0 else b
+            p.view("rgb").copy_(torch.from_numpy(x))
+            p.run()
+            torch.cuda.synchronize()
+            assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(x, T=40.0)["mask"]), (mode, it)
+
+
+@pytest.mark.parametrize("geometry", ["paper", "b200"])
+@pytest.mark.parametrize("lines", [36, 68, 2176, 0])
+@pytest.mark.parametrize("mode", ["graph", "persistent"])
+def test_motivational_graph(geometry, lines, mode):
+    """configs[0]: 256x256 RGB -> A -> B, paper geometry and B200 geometry, budgets from
+    the worked example (36 lines = 64 fragments, 2176 = untiled) and the device L2."""
+    from paper_conf_date_maghazeh0ep19_b200 import Motivational
+    rgb = synth.scene(1234, 256, 256)
+    ref = O.motivational(rgb)
+    m = Motivational(device="cuda", geometry=geometry, internal=False)
+    m.b.store.tensors["intm"].fill_(0xA5)
+    m.b.store.tensors["out"].fill_(0xA5)
+    m.view("in").copy_(torch.from_numpy(rgb))
+    try:
+        plan = m.plan(lines * 128, kind="budget", exec_mode=mode)
+    except Exception as e:  # b200 tiles are larger than 36 / 68 lines
+        assert geometry == "b200" and "UNTILEABLE" in str(e)
+        return
+    if geometry == "paper" and lines == 36:
+        assert plan.num_fragments() == 64
+    m.run()
+    torch.cuda.synchronize()
+    assert np.array_equal(m.view("intm").cpu().numpy(), ref["gray"])
+    assert np.array_equal(m.view("out").cpu().numpy(), ref["down"])
+
+
+def test_schedule_invariance_rows():
+    """P10 on the GPU: differently interleaved valid schedules (ROWS plans with different
+    fragment heights, persistent skews) all give the untiled result."""
+    W, H, F = 768, 192, 1
+    rgb = synth.uniform(3, W, H, F)
+    ref = O.pipeline(rgb, T=30.0)
+    for rows in (1, 2, 5, 12):
+        out, _ = _run(W, H, F, rgb, T=30.0, kind="rows", rows=rows, exec_mode="stream")
+        for k in KEYS:
+            assert _eq(out[k], ref[k]), (rows, k)
+        for skew in (-1, 1, 4):
+            out, _ = _run(W, H, F, rgb, T=30.0, kind="rows", rows=rows, exec_mode="persistent", skew=skew)
+            for k in KEYS:
+                assert _eq(out[k], ref[k]), (rows, skew, k)
+
+
+def test_host_io_end_to_end():
+    """ktiler_execute_host: pinned host rgb in, host mask out, through the C ABI."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 1024, 200, 3
+    rgb = synth.scene(9, W, H, F)
+    ref = O.pipeline(rgb, T=70.0)
+    p = Pipeline(W, H, F, T=70.0, internal=True, geometry=SMALL)
+    plan = p.plan(100 * 1024, kind="budget", exec_mode="graph", discard=True)
+    hin = torch.from_numpy(rgb).pin_memory()
+    hout = torch.empty((F, H // 2, W // 2), dtype=torch.uint8).pin_memory()
+    s = torch.cuda.current_stream().cuda_stream
+    plan.execute_host([(p.buf_id("rgb"), hin.data_ptr(), 0, 0)], [(p.buf_id("mask"), hout.data_ptr(), 0, 0)], s)
+    torch.cuda.synchronize()
+    assert np.array_equal(hout.numpy(), ref["mask"])
+
+
+def test_gpu_generator_matches_numpy():
+    from inputs import gpu as G
+    for kind in ("uniform", "scene"):
+        W, H, F = 200, 60, 2
+        t = torch.empty((F, H, W, 3), dtype=torch.uint8, device="cuda")
+        G.fill(kind, 11, t.data_ptr(), W * 3, W * H * 3, W, H, F=F)
+        torch.cuda.synchronize()
+        assert np.array_equal(t.cpu().numpy(), synth.make(kind, 11, W, H, F))
+        # a strip of rows
+        s = torch.empty((1, 20, W, 3), dtype=torch.uint8, device="cuda")
+        G.fill(kind, 11, s.data_ptr(), W * 3, 20 * W * 3, W, H, y0=17, rows=20, f0=1, F=1)
+        torch.cuda.synchronize()
+        assert np.array_equal(s.cpu().numpy()[0], synth.make(kind, 11, W, H, F)[1, 17:37])

@@ -1,0 +1,70 @@
+"""Plan/exec-mode sweep on one pipeline instance (BASELINE configs[2]/[3] fragment-size
+sweep).  Prints one JSON line per configuration: ms per execute (CUDA events, median of
+reps), Mpix/s, fragments, launches.  Not the headline bench (bench.py is)."""
+from __future__ import annotations
+
+import argparse
+import itertools
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--W", type=int, default=7680)
+    ap.add_argument("--H", type=int, default=4320)
+    ap.add_argument("--F", type=int, default=64)
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--configs", default="default", help="default | json list of plan kwargs")
+    args = ap.parse_args()
+    import torch
+
+    import __graft_entry__ as ge
+    from inputs import gpu as G
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    ge.build()
+    p = Pipeline(args.W, args.H, args.F, internal=True)
+    s = torch.cuda.current_stream()
+    G.fill("scene", 1234, p.view("rgb").data_ptr(), args.W * 3, args.W * 3 * args.H, args.W, args.H, F=args.F,
+           stream=s.cuda_stream)
+    torch.cuda.synchronize()
+    if args.configs == "default":
+        cfgs = [dict(kind="none", exec_mode="graph")]
+        for rows, skew in itertools.product((1, 2, 4, 8), (0, 2, 6)):
+            cfgs.append(dict(kind="rows", rows=rows, exec_mode="persistent", discard=True, skew=skew))
+        cfgs.append(dict(kind="none", exec_mode="persistent"))
+        cfgs.append(dict(kind="budget", l2_fraction=0.5, exec_mode="persistent", discard=True))
+        cfgs.append(dict(kind="budget", l2_fraction=1.0, exec_mode="graph", discard=True))
+    else:
+        cfgs = json.loads(args.configs)
+    pix = args.W * args.H * args.F
+    for c in cfgs:
+        try:
+            pl = p.b.g.plan(0, **c)
+            for _ in range(2):
+                pl.execute(s.cuda_stream)
+            ts = []
+            for _ in range(args.reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                pl.execute(s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ms = statistics.median(ts)
+            st = pl.stats()
+            print(json.dumps({"cfg": c, "minb": os.environ.get("KTILER_PERSIST_MINB", "default"), "ms": round(ms, 4),
+                              "Mpix/s": round(pix / ms / 1e3, 1), "fragments": st["n_fragments"],
+                              "launches": st["n_launches"]}), flush=True)
+            del pl
+        except Exception as e:
+            print(json.dumps({"cfg": c, "error": str(e)}), flush=True)
+
+
+if __name__ == "__main__":
+    main()
