@@ -32,9 +32,11 @@ namespace {
 
 using ktd::DBuf;
 constexpr int MAXR = 4, MAXD = 4;
-constexpr int PERSIST_THREADS = 256;
+constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+1 control warp)
+constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
+constexpr int PERSIST_THREADS = PCOMP_THREADS + 32;
 constexpr int MAXDEAD = 64;
-constexpr int PERSIST_MINB_DEFAULT = 3;
+constexpr int PERSIST_MINB_DEFAULT = 4;
 
 struct LRect {
   int32_t x0, y0, z0, x1, y1, z1;
@@ -45,10 +47,14 @@ struct DRect {  // whole 128-B lines: row r -> base + z*fs + y*pitch + lb0 + k*1
   int32_t y0, y1, z0, z1;
 };
 struct KParams {
+  CUtensorMap tmap;     // input tile map (tensor TMA), valid if use_tmap
+  uint32_t box_bytes;   // bytes one tensor-TMA box delivers
+  int32_t use_tmap;
   DBuf in, out;
   int32_t tw, th;
   float T;
   int32_t nrect, ndisc, pdl;
+  int64_t stage_bytes;  // one of the two staging buffers
   LRect r[MAXR];
   int64_t rpre[MAXR + 1];
   DRect d[MAXD];
@@ -73,29 +79,90 @@ __device__ __forceinline__ void do_discards(const KParams& p) {
   }
 }
 
-template <int OP, bool SCALAR>
-__global__ void __launch_bounds__(256) op_kernel(const __grid_constant__ KParams p) {
-  if (p.pdl) pdl_wait();
-  if (p.ndisc) do_discards(p);
-  if (p.pdl) pdl_launch();
-  int64_t lin = blockIdx.x;
-  if (lin >= p.rpre[p.nrect]) return;  // discard-only CTAs
+// Tile i of a launch: its rect list maps the launch's linear tile index to a block.
+__device__ __forceinline__ ktd::Tile launch_tile(const KParams& p, int64_t lin64) {
   int k = 0;
-  while (k + 1 < p.nrect && lin >= p.rpre[k + 1]) ++k;
+  while (k + 1 < p.nrect && lin64 >= p.rpre[k + 1]) ++k;
   const LRect& r = p.r[k];
-  lin -= p.rpre[k];
-  const int64_t w = r.x1 - r.x0, h = r.y1 - r.y0;
-  const int64_t bx = r.x0 + lin % w, by = r.y0 + (lin / w) % h, bz = r.z0 + lin / (w * h);
+  // 32-bit index math (a launch has < 2^31 blocks): 64-bit division is ~100 instructions
+  const unsigned lin = (unsigned)(lin64 - p.rpre[k]);
+  const unsigned w = (unsigned)(r.x1 - r.x0), h = (unsigned)(r.y1 - r.y0);
+  const unsigned q = lin / w, q2 = q / h;
+  const int64_t bx = r.x0 + (int)(lin - q * w), by = r.y0 + (int)(q - q2 * h), bz = r.z0 + (int)q2;
   ktd::Tile t;
   t.z = bz;
   t.x0 = p.tw * bx;
   t.y0 = p.th * by;
   t.x1 = min(t.x0 + p.tw, p.out.W);
   t.y1 = min(t.y0 + p.th, p.out.H);
+  t.fw = p.tw;
+  t.pad = 0;
+  return t;
+}
+
+template <int OP, bool SCALAR>
+__global__ void __launch_bounds__(256, (OP == 1 || OP == 3) ? 3 : 4) op_kernel(const __grid_constant__ KParams p) {
+  if (p.pdl) pdl_wait();
+  if (p.ndisc) do_discards(p);
+  if (p.pdl) pdl_launch();
+  const int64_t ntiles = p.rpre[p.nrect];
   const int nt = blockDim.x * blockDim.y * blockDim.z;
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  extern __shared__ __align__(16) uint8_t ktsm[];
-  ktd::run_tile(OP, SCALAR, p.in, p.out, t, p.T, nt, tid, ktsm);
+  if (SCALAR) {
+    for (int64_t i = blockIdx.x; i < ntiles; i += gridDim.x) ktd::scalar_tile(OP, p.in, p.out, launch_tile(p, i), p.T, nt, tid);
+    return;
+  }
+  // Grid-stride over the launch's tiles with two shared buffers: the TMA bulk copies of
+  // tile i+2 stream in while tile i+1 computes.
+  extern __shared__ __align__(128) uint8_t ktsm[];
+  __shared__ __align__(8) uint64_t mbar[2];
+  __shared__ ktd::Tile s_tile[2];  // decoded once by warp 0, read by all after the mbarrier
+  if (tid == 0) {
+    ktd::mbar_init(&mbar[0], 1);
+    ktd::mbar_init(&mbar[1], 1);
+    ktd::fence_proxy_async();
+  }
+  __syncthreads();
+  const int64_t i0 = blockIdx.x;
+  if (i0 >= ntiles) return;  // discard-only CTAs
+  auto issue = [&](int64_t i, int slot) {  // warp 0
+    const ktd::Tile t = launch_tile(p, i);
+    uint8_t* dst = ktsm + (slot ? p.stage_bytes : 0);
+    if (p.use_tmap) {
+      if (tid == 0) {
+        s_tile[slot] = t;
+        ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot]);
+      }
+    } else {
+      if (tid == 0) s_tile[slot] = t;
+      ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
+    }
+  };
+  if (tid < 32) {
+    issue(i0, 0);
+    if (i0 + gridDim.x < ntiles) issue(i0 + gridDim.x, 1);
+  }
+  unsigned ph = 0;
+  int b = 0;
+  for (int64_t i = i0; i < ntiles; i += gridDim.x, b ^= 1) {
+    uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+    ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
+    ph ^= 1u << b;
+    const ktd::Tile t = s_tile[b];
+    if ((OP == 1 || OP == 3) && ktd::needs_fix(OP, p.in, t)) {
+      ktd::stage_fix(OP, p.in, t, buf, nt, tid);
+      __syncthreads();
+    }
+    ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid);
+    const int64_t nx = i + 2 * (int64_t)gridDim.x;
+    if (nx < ntiles) {
+      __syncthreads();  // buffer b consumed
+      if (tid < 32) {
+        ktd::fence_proxy_async();
+        issue(nx, b);
+      }
+    }
+  }
 }
 
 __global__ void discard_kernel(const __grid_constant__ KParams p) {
@@ -108,6 +175,9 @@ __global__ void discard_kernel(const __grid_constant__ KParams p) {
 // persistent executor
 // ------------------------------------------------------------------------------------
 struct PNode {
+  CUtensorMap tmap;  // input tile map (tensor TMA), valid if use_tmap
+  uint32_t box_bytes;
+  int32_t use_tmap;
   DBuf in, out;
   int32_t op, scalar, tw, th;
   float T;
@@ -150,41 +220,44 @@ __device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-__device__ __forceinline__ void hit(int64_t a, int64_t o, int64_t hl, int64_t hr, int64_t lo, int64_t hi, int64_t n,
-                                    int64_t& i0, int64_t& i1) {
-  auto fd = [](int64_t x, int64_t b) { int64_t q = x / b; return (x % b != 0 && x < 0) ? q - 1 : q; };
-  i0 = max((int64_t)0, fd(lo - o - hr, a));
-  i1 = min(n, fd(hi - o + hl - 1, a) + 1);
+// Producer blocks i in [0, n) with [a*i, a*(i+1)) meeting [lo, hi) (write footprints have no
+// offsets or halos for built-ins).  32-bit: pixel coordinates are < 2^31.
+__device__ __forceinline__ void hit(int a, int lo, int hi, int n, int& i0, int& i1) {
+  i0 = lo > 0 ? lo / a : 0;
+  i1 = min(n, (hi + a - 1) / a);
   if (i1 < i0) i1 = i0;
 }
 
-
 // Decoded ticket: node, block, its output rect, and the producer-block range of its read
-// footprint (the closed-form dependency of the affine maps).
+// footprint (the closed-form dependency of the affine maps).  Computed
+// once per tile by the control warp and handed to the compute warps in shared memory.
 struct TInfo {
   const PNode* nd;
   ktd::Tile t;
-  int64_t bx, by, px0, py0, pw, ndep;
+  int bx, by, px0, py0, pw, ndep;
 };
 
 __device__ __forceinline__ TInfo decode(const PParams& p, uint64_t dsc) {
   TInfo r;
   r.nd = p.nodes + (dsc >> 60);
   const PNode& nd = *r.nd;
-  const int64_t bz = (dsc >> 48) & 0xFFF;
-  r.by = (dsc >> 24) & 0xFFFFFF;
-  r.bx = dsc & 0xFFFFFF;
-  r.t.z = bz;
-  r.t.x0 = nd.tw * r.bx;
-  r.t.y0 = nd.th * r.by;
-  r.t.x1 = min(r.t.x0 + nd.tw, nd.out.W);
-  r.t.y1 = min(r.t.y0 + nd.th, nd.out.H);
-  int64_t px0 = 0, px1 = 0, py0 = 0, py1 = 0;
+  r.by = (int)((dsc >> 24) & 0xFFFFFF);
+  r.bx = (int)(dsc & 0xFFFFFF);
+  const int tw = nd.tw, th = nd.th, W = (int)nd.out.W, H = (int)nd.out.H;
+  r.t.z = (int64_t)((dsc >> 48) & 0xFFF);
+  r.t.x0 = tw * r.bx;
+  r.t.y0 = th * r.by;
+  r.t.x1 = min(tw * r.bx + tw, W);
+  r.t.y1 = min(th * r.by + th, H);
+  r.t.fw = tw;
+  r.t.pad = 0;
+  int px0 = 0, px1 = 0, py0 = 0, py1 = 0;
   if (nd.pu >= 0) {
-    int64_t rx0 = max((int64_t)0, nd.rax * r.bx + nd.rox - nd.rhl), rx1 = min(nd.in.W, nd.rax * (r.bx + 1) + nd.rox + nd.rhr);
-    int64_t ry0 = max((int64_t)0, nd.ray * r.by + nd.roy - nd.rht), ry1 = min(nd.in.H, nd.ray * (r.by + 1) + nd.roy + nd.rhb);
-    hit(nd.wax, 0, 0, 0, rx0, rx1, nd.pgx, px0, px1);
-    hit(nd.way, 0, 0, 0, ry0, ry1, nd.pgy, py0, py1);
+    const int rax = (int)nd.rax, ray = (int)nd.ray, rox = (int)nd.rox, roy = (int)nd.roy;
+    const int rx0 = max(0, rax * r.bx + rox - nd.rhl), rx1 = min((int)nd.in.W, rax * (r.bx + 1) + rox + nd.rhr);
+    const int ry0 = max(0, ray * r.by + roy - nd.rht), ry1 = min((int)nd.in.H, ray * (r.by + 1) + roy + nd.rhb);
+    hit((int)nd.wax, rx0, rx1, nd.pgx, px0, px1);
+    hit((int)nd.way, ry0, ry1, nd.pgy, py0, py1);
   }
   r.px0 = px0;
   r.py0 = py0;
@@ -193,160 +266,198 @@ __device__ __forceinline__ TInfo decode(const PParams& p, uint64_t dsc) {
   return r;
 }
 
-__device__ __forceinline__ const unsigned int* dep_flag(const PParams& p, const TInfo& a, int64_t i) {
+__device__ __forceinline__ const unsigned int* dep_flag(const PParams& p, const TInfo& a, int i) {
   const PNode& nd = *a.nd;
-  return p.flags + nd.pflag0 + (a.t.z * nd.pgy + a.py0 + i / a.pw) * nd.pgx + a.px0 + i % a.pw;
+  const int dy = i / a.pw;
+  return p.flags + nd.pflag0 + ((int64_t)a.t.z * nd.pgy + a.py0 + dy) * nd.pgx + a.px0 + (i - dy * a.pw);
 }
 
-// Blocking wait for all producer blocks of a (every thread polls its share), then barrier.
-__device__ __forceinline__ void wait_deps(const PParams& p, const TInfo& a, unsigned epoch, int nt, int tid) {
-  for (int64_t i = tid; i < a.ndep; i += nt) {
+// ---- persistent executor: warp-specialized (PCOMP_WARPS compute warps + 1 control warp) ----
+__device__ __forceinline__ void nbar_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void nbar_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+__device__ __forceinline__ void mbar_arrive(uint64_t* m) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ktd::smem_u32(m)) : "memory");
+}
+constexpr uint64_t DESC_STOP = ~0ull;
+constexpr unsigned FULL = 0xFFFFFFFFu;
+
+// Control warp: are all producer blocks of a complete?  (one poll per flag, warp-uniform)
+__device__ __forceinline__ bool ctl_probe(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
+  bool ok = true;
+  for (int i = lane; i < a.ndep; i += 32) ok &= (ld_acquire(dep_flag(p, a, i)) == epoch);
+  return __all_sync(FULL, ok);
+}
+__device__ __forceinline__ void ctl_wait(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
+  for (int i = lane; i < a.ndep; i += 32) {
     const unsigned int* f = dep_flag(p, a, i);
     while (ld_acquire(f) != epoch) __nanosleep(32);
   }
-  __syncthreads();
+  __syncwarp();
 }
 
-// One non-blocking poll of a's producer flags; CTA-uniform result.
-__device__ __forceinline__ bool probe_deps(const PParams& p, const TInfo& a, unsigned epoch, int nt, int tid) {
-  int ok = 1;
-  for (int64_t i = tid; i < a.ndep; i += nt) ok &= (ld_acquire(dep_flag(p, a, i)) == epoch);
-  return __syncthreads_and(ok) != 0;
-}
-
-__device__ __forceinline__ void stage_any(const TInfo& a, uint8_t* sm, int nt, int tid) {
-  if (!a.nd->scalar) ktd::stage_tile(a.nd->op, a.nd->in, a.t, sm, nt, tid);
-}
-
-// Software-pipelined persistent executor.  Per CTA: while tile A is computed from shared
-// buffer `cur`, the input of the next tile B is already streaming into the other buffer
-// (cp.async), provided B's producers are complete (non-blocking probe); otherwise B is
-// staged after A is released, so a CTA never waits on a tile it has not released itself.
-// The ticket queue (A, B, C) lives in shared memory and thread 0 refills it one tile
-// ahead, so no atomic or descriptor load is ever waited on and nothing but the buffer
-// index stays live across a tile's arithmetic.  Deadlock freedom: tickets are taken in
-// schedule order, each CTA processes its tickets in increasing order and producers
-// precede consumers, so the smallest unfinished ticket is always runnable.
-struct PQueue {
-  int64_t tk[3];    // A, B, C
-  uint64_t dsc[3];
-  int64_t fut;      // thread 0's next grab (its descriptor is loaded one tile later)
-  int ndead;
-  int readyB;
-};
-
-__device__ __forceinline__ void release_and_discard(const PParams& p, const TInfo& a, unsigned epoch, PQueue& q,
-                                                    int64_t* dead, int nt, int tid) {
+// Control warp, after the compute warps finished tile a (named barrier): publish its
+// completion flag (gpu-scope release), then count it as a reader of its producer blocks;
+// the last reader of a block drops that block's lines from L2 without write-back.
+__device__ __forceinline__ void ctl_release(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
   const PNode& nd = *a.nd;
-  if (tid == 0) {
+  if (lane == 0) {
     __threadfence();
     st_release(p.flags + nd.flag0 + (a.t.z * nd.gy + a.by) * nd.gx + a.bx, epoch);
   }
   if (!(p.discard && nd.disc_in)) return;
-  // last reader of a producer block drops its lines from L2 (no write-back)
-  for (int64_t i = tid; i < a.ndep; i += nt) {
-    const int64_t pl = (a.t.z * nd.pgy + a.py0 + i / a.pw) * nd.pgx + a.px0 + i % a.pw;
-    unsigned int old = atomicAdd(p.rc + nd.pflag0 + pl, 1u);
-    if (old + 1 == nd.expect[pl]) {
-      p.rc[nd.pflag0 + pl] = 0;
-      int k = atomicAdd(&q.ndead, 1);
-      if (k < MAXDEAD) dead[k] = pl;
+  for (int base = 0; base < a.ndep; base += 32) {
+    const int i = base + lane;
+    int64_t pl = 0;
+    bool dead = false;
+    if (i < a.ndep) {
+      const int dy = i / a.pw;
+      pl = ((int64_t)a.t.z * nd.pgy + a.py0 + dy) * nd.pgx + a.px0 + (i - dy * a.pw);
+      const unsigned int old = atomicAdd(p.rc + nd.pflag0 + pl, 1u);
+      dead = old + 1 == nd.expect[pl];
+      if (dead) p.rc[nd.pflag0 + pl] = 0;
     }
-  }
-  __syncthreads();
-  const int nd_dead = min(q.ndead, MAXDEAD);
-  const int64_t eb = nd.op == 4 ? 4 : 1;  // element bytes of the producer output (= our input)
-  for (int k = 0; k < nd_dead; ++k) {
-    const int64_t pl = dead[k];
-    const int64_t qx = pl % nd.pgx, qy = (pl / nd.pgx) % nd.pgy;
-    const int64_t ax0 = nd.ptw * qx, ax1 = min(ax0 + nd.ptw, nd.in.W);
-    const int64_t ay0 = nd.pth * qy, ay1 = min(ay0 + nd.pth, nd.in.H);
-    const uint64_t fb = (uint64_t)(nd.in.p + a.t.z * nd.in.fstride);
-    // lines fully inside [ax0*eb, ax1*eb) of each row (the buffer pitch is a multiple of 128)
-    const int64_t l0 = (ax0 * eb + 127) >> 7, l1 = (ax1 * eb) >> 7, lpr = l1 > l0 ? l1 - l0 : 0;
-    const int64_t n = lpr * (ay1 - ay0);
-    for (int64_t j = tid; j < n; j += nt) {
-      const int64_t yy = ay0 + j / lpr, l = l0 + j % lpr;
-      ktd::discard_line((const void*)(fb + yy * nd.in.pitch + 128 * l));
+    unsigned mask = __ballot_sync(FULL, dead);
+    const int eb = nd.op == 4 ? 4 : 1;  // element bytes of the producer output (= our input)
+    while (mask) {
+      const int j = __ffs(mask) - 1;
+      mask &= mask - 1;
+      const int q = (int)(__shfl_sync(FULL, pl, j) - (int64_t)a.t.z * nd.pgy * nd.pgx);  // within the frame
+      const int qy = q / nd.pgx, qx = q - qy * nd.pgx;
+      const int ax0 = (int)nd.ptw * qx, ax1 = min(ax0 + (int)nd.ptw, (int)nd.in.W);
+      const int ay0 = (int)nd.pth * qy, ay1 = min(ay0 + (int)nd.pth, (int)nd.in.H);
+      const uint8_t* fb = nd.in.p + a.t.z * nd.in.fstride;
+      // lines fully inside [ax0*eb, ax1*eb) of each row (the buffer pitch is a multiple of 128)
+      const int l0 = (ax0 * eb + 127) >> 7, l1 = (ax1 * eb) >> 7, lpr = l1 > l0 ? l1 - l0 : 0;
+      const int n = lpr * (ay1 - ay0);
+      for (int k = lane; k < n; k += 32) {
+        const int dy = k / lpr;
+        ktd::discard_line(fb + (int64_t)(ay0 + dy) * nd.in.pitch + 128 * (l0 + k - dy * lpr));
+      }
     }
   }
 }
 
+// Persistent executor.  One launch runs the whole schedule: tiles are taken in schedule
+// order from an atomic ticket (deadlock-free: producers precede consumers and each CTA
+// handles its tickets in order, so the smallest unfinished ticket is always runnable).
+// Warp specialization inside a CTA:
+//   control warp  takes tickets, waits for a tile's producer flags (acquire), streams its
+//                 input tile into one of two shared buffers with TMA bulk copies (one per
+//                 row, completing on that buffer's mbarrier), and — once the compute
+//                 warps signal on a named barrier that a buffer's tile is done — publishes
+//                 the tile's flag (release) and retires dead producer lines (discard);
+//   compute warps wait on the buffer's mbarrier, compute the tile from shared memory and
+//                 arrive (non-blocking) on the buffer's named barrier.
+// So the input of tile i+1 streams while tile i computes, and no compute warp ever waits
+// on a fence, a flag or an atomic.  The control warp never waits on a producer flag while
+// it holds an unreleased tile of its own.
 template <int MINB>
 __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const __grid_constant__ PParams p) {
-  __shared__ PQueue q;
+  __shared__ __align__(8) uint64_t s_full[2];
+  __shared__ uint64_t s_desc[2];
+  __shared__ TInfo s_ti[2];  // decoded tile of each buffer (control warp -> compute warps)
   __shared__ unsigned int s_epoch;
-  __shared__ int64_t s_dead[MAXDEAD];
-  extern __shared__ __align__(16) uint8_t ktsm[];
-  const int nt = blockDim.x, tid = threadIdx.x;
+  extern __shared__ __align__(128) uint8_t ktsm[];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     s_epoch = *(volatile unsigned int*)&p.ctrl->epoch;
-    for (int k = 0; k < 3; ++k) {
-      const int64_t t = atomicAdd(&p.ctrl->ticket, 1u);
-      q.tk[k] = t;
-      q.dsc[k] = t < p.total ? p.desc[t] : 0;
-    }
-    q.fut = q.tk[2] < p.total ? (int64_t)atomicAdd(&p.ctrl->ticket, 1u) : p.total;
+    ktd::mbar_init(&s_full[0], 1);
+    ktd::mbar_init(&s_full[1], 1);
+    ktd::fence_proxy_async();
   }
   __syncthreads();
   const unsigned int epoch = s_epoch;
-  int cur = 0;
-  if (q.tk[0] < p.total) {
-    const TInfo a = decode(p, q.dsc[0]);
-    wait_deps(p, a, epoch, nt, tid);
-    stage_any(a, ktsm, nt, tid);
-  }
-  ktd::cp_async_commit();
-  while (q.tk[0] < p.total) {
-    uint8_t* const bufA = ktsm + (cur ? p.stage_bytes : 0);
-    uint8_t* const bufB = ktsm + (cur ? 0 : p.stage_bytes);
-    // ---- start B's staging if its producers are done ----
-    bool readyB = false;
-    if (q.tk[1] < p.total) {
-      const TInfo b = decode(p, q.dsc[1]);
-      readyB = probe_deps(p, b, epoch, nt, tid);
-      if (readyB) stage_any(b, bufB, nt, tid);
+  if (warp == PCOMP_WARPS) {
+    // ------------------------------ control warp ------------------------------
+    int64_t tq = 0;        // lane 0: next ticket (grabbed one tile ahead)
+    uint64_t dq = 0;       // lane 0: its descriptor
+    if (lane == 0) {
+      tq = atomicAdd(&p.ctrl->ticket, 1u);
+      dq = tq < p.total ? p.desc[tq] : 0;
     }
-    ktd::cp_async_commit();
-    // ---- thread 0: grab the ticket behind C (lands in q.fut while A computes) ----
-    int64_t fut = p.total;
-    uint64_t fdsc = 0;
-    if (tid == 0 && q.fut < p.total) {
-      fut = atomicAdd(&p.ctrl->ticket, 1u);
-      fdsc = p.desc[q.fut];
+    // the tile in flight in "this" buffer (b) and in the "other" one (b ^ 1); swapped
+    // every iteration, so no runtime-indexed arrays (they would live in local memory)
+    uint64_t d_this = 0, d_other = 0;
+    bool u_this = false, u_other = false;
+    int b = 0;
+    for (;; b ^= 1) {
+      const int64_t t = __shfl_sync(FULL, tq, 0);
+      const uint64_t d = __shfl_sync(FULL, dq, 0);
+      if (lane == 0 && t < p.total) {  // next grab; consumed next iteration
+        tq = atomicAdd(&p.ctrl->ticket, 1u);
+        dq = tq < p.total ? p.desc[tq] : 0;
+      }
+      // buffer b is free once the compute warps are done with the tile two back
+      if (u_this) {
+        nbar_sync(1 + b, PERSIST_THREADS);
+        ctl_release(p, decode(p, d_this), epoch, lane);
+        u_this = false;
+      }
+      if (t >= p.total) {
+        if (lane == 0) {
+          s_desc[b] = DESC_STOP;
+          mbar_arrive(&s_full[b]);
+        }
+        break;
+      }
+      const TInfo a = decode(p, d);
+      if (!ctl_probe(p, a, epoch, lane)) {
+        if (u_other) {  // never wait while holding an unreleased tile
+          nbar_sync(1 + (b ^ 1), PERSIST_THREADS);
+          ctl_release(p, decode(p, d_other), epoch, lane);
+          u_other = false;
+        }
+        ctl_wait(p, a, epoch, lane);
+      }
+      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+      if (lane == 0) {
+        s_desc[b] = d;
+        s_ti[b] = a;
+      }
+      if (a.nd->scalar) {
+        if (lane == 0) mbar_arrive(&s_full[b]);
+      } else {
+        ktd::fence_proxy_async();
+        if (a.nd->use_tmap) {
+          if (lane == 0) ktd::stage_issue_tmap(a.nd->op, &a.nd->tmap, a.nd->box_bytes, a.nd->in, a.t, buf, &s_full[b]);
+        } else {
+          ktd::stage_issue(a.nd->op, a.nd->in, a.t, buf, &s_full[b], lane);
+        }
+      }
+      // swap roles for the next iteration (which stages into b ^ 1)
+      d_this = d_other;
+      u_this = u_other;
+      d_other = d;
+      u_other = true;
     }
-    // ---- compute A ----
-    ktd::cp_async_wait<1>();
-    __syncthreads();
-    {
-      const TInfo a = decode(p, q.dsc[0]);
+    // drain: the tile in the other buffer (if any) is the last one in flight
+    if (u_other) {
+      nbar_sync(1 + (b ^ 1), PERSIST_THREADS);
+      ctl_release(p, decode(p, d_other), epoch, lane);
+    }
+  } else {
+    // ------------------------------ compute warps ------------------------------
+    unsigned ph = 0;  // bit b = phase parity of buffer b's mbarrier
+    for (int b = 0;; b ^= 1) {
+      ktd::mbar_wait(&s_full[b], (ph >> b) & 1u);
+      ph ^= 1u << b;
+      if (s_desc[b] == DESC_STOP) break;
+      const TInfo a = s_ti[b];
       const PNode& nd = *a.nd;
-      if (nd.scalar) ktd::scalar_tile(nd.op, nd.in, nd.out, a.t, nd.T, nt, tid);
-      else ktd::compute_tile(nd.op, nd.out, a.t, bufA, nd.T, nt, tid);
+      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+      if (nd.scalar) {
+        ktd::scalar_tile(nd.op, nd.in, nd.out, a.t, nd.T, PCOMP_THREADS, tid);
+      } else {
+        if ((nd.op == 1 || nd.op == 3) && ktd::needs_fix(nd.op, nd.in, a.t)) {
+          ktd::stage_fix(nd.op, nd.in, a.t, buf, PCOMP_THREADS, tid);
+          nbar_sync(3, PCOMP_THREADS);
+        }
+        ktd::compute_tile(nd.op, nd.out, a.t, buf, nd.T, PCOMP_THREADS, tid);
+      }
+      nbar_arrive(1 + b, PERSIST_THREADS);
     }
-    if (tid == 0) q.ndead = 0;
-    __syncthreads();
-    release_and_discard(p, decode(p, q.dsc[0]), epoch, q, s_dead, nt, tid);
-    __syncthreads();
-    // ---- shift the queue: B -> A, C -> B, fut -> C ----
-    if (tid == 0) {
-      const int64_t c = q.fut;
-      q.tk[0] = q.tk[1]; q.dsc[0] = q.dsc[1];
-      q.tk[1] = q.tk[2]; q.dsc[1] = q.dsc[2];
-      q.tk[2] = c;       q.dsc[2] = fdsc;
-      q.fut = fut;
-      q.readyB = readyB;
-    }
-    __syncthreads();
-    if (q.tk[0] < p.total && !q.readyB) {
-      const TInfo b = decode(p, q.dsc[0]);
-      wait_deps(p, b, epoch, nt, tid);
-      stage_any(b, bufB, nt, tid);
-      ktd::cp_async_commit();
-    }
-    cur ^= 1;
   }
-  ktd::cp_async_wait<0>();
+  __syncthreads();
   if (tid == 0) {
     __threadfence();
     unsigned int old = atomicAdd(&p.ctrl->done, 1u);
@@ -392,6 +503,7 @@ struct Launch {
   int64_t blocks = 0;
   dim3 block;
   int smem = 0;
+  int64_t resident = 0;  // CTAs of this kernel that fit the device at once
   std::vector<int32_t> crects;  // OP_CUSTOM rect list
 };
 
@@ -516,7 +628,8 @@ void build_launches(ktiler_plan_s* P) {
           pending.erase(pending.begin(), pending.begin() + nd);
         }
         L.block = dim3(n.block[0], n.block[1], n.block[2]);
-        L.smem = n.scalar ? 0 : ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay);
+        L.kp.stage_bytes = n.scalar ? 0 : (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127;
+        L.smem = (int)(2 * L.kp.stage_bytes);
         P->launches.push_back(L);
       }
     }
@@ -530,6 +643,55 @@ void build_launches(ktiler_plan_s* P) {
   flush_disc_only(0);
 }
 
+// ---- tensor maps for TMA staging (driver entry point, resolved at first execute) ----
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn get_encode() {
+  static EncodeTiledFn fn = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (EncodeTiledFn)f;
+  }
+  return fn;
+}
+
+// Input-tile map of built-in node n: the input buffer as 4-byte elements
+// [frames][height][ceil(row bytes / 4)], box = the staged window of one full tile
+// (ktd::stage_geo / stage_bytes).  False -> the kernels use per-row bulk copies instead.
+bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* box_bytes) {
+  if (getenv("KTILER_NO_TMAP")) return false;
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return false;
+  const kt::Access& w = n.acc[n.wacc];
+  const kt::Buffer& B = g.bufs[n.acc[n.racc].buf];
+  const int tw = (int)w.ax, th = (int)w.ay, nseg = (tw + 15) / 16;
+  int bw = 0, bh = 0;  // box bytes per row, box rows
+  switch (n.op) {
+    case KTILER_OP_GRAY: bw = 48 * nseg; bh = th; break;
+    case KTILER_OP_BLUR5: bw = 16 * (nseg + 2); bh = th + 4; break;
+    case KTILER_OP_DOWN2: bw = 32 * nseg; bh = 2 * th; break;
+    case KTILER_OP_SOBEL3: bw = 16 * (nseg + 2); bh = th + 2; break;
+    default: bw = 64 * nseg; bh = th; break;
+  }
+  if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != ktd::stage_bytes(n.op, tw, th)) return false;
+  if (B.d.pitch_bytes % 16 || B.d.frame_stride_bytes % 16) return false;
+  const int64_t rowbytes = B.d.width * B.d.elem_bytes;
+  cuuint64_t dims[3] = {(cuuint64_t)((rowbytes + 3) / 4), (cuuint64_t)B.d.height, (cuuint64_t)B.d.frames};
+  cuuint64_t strides[2] = {(cuuint64_t)B.d.pitch_bytes, (cuuint64_t)B.d.frame_stride_bytes};
+  cuuint32_t box[3] = {(cuuint32_t)(bw / 4), (cuuint32_t)bh, 1}, es[3] = {1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, B.d.base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return false;
+  *box_bytes = (uint32_t)(bw * bh);
+  return true;
+}
+
 ktiler_status cuda_fail(cudaError_t e, const char* what) {
   return fail(KTILER_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
@@ -541,16 +703,23 @@ ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
       continue;
     }
     kfn_t fn = L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
+    if (L.resident == 0 && L.smem > 32 * 1024) {  // static + dynamic may pass the 48 KB default
+      cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
+      if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
+    }
+    if (L.resident == 0) {  // CTAs that fit at once: the vector kernels grid-stride over tiles
+      int nsm = 0, occ = 0;
+      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)(L.block.x * L.block.y * L.block.z), L.smem);
+      L.resident = (int64_t)std::max(1, nsm) * std::max(1, occ);
+    }
     int64_t grid = std::max<int64_t>(L.blocks, 1);
+    if (L.node >= 0 && !L.n->scalar) grid = std::min<int64_t>(grid, L.resident);
     if (L.kp.ndisc) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = L.block;
     cfg.dynamicSmemBytes = (size_t)L.smem;
-    if (L.smem > 48 * 1024) {
-      cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
-      if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
-    }
     cfg.stream = st;
     cudaLaunchAttribute attr[2];
     int na = 0;
@@ -641,6 +810,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
       const kt::Buffer& ib = g.bufs[c.buf];
       q.disc_in = (ib.d.flags & KTILER_BUF_INTERNAL) && discardable(ib);
     }
+    q.use_tmap = !n.scalar && make_tmap(g, n, &q.tmap, &q.box_bytes);
   }
   int nsm = 0, occ = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
@@ -648,7 +818,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     // registers vs CTAs per SM (KTILER_PERSIST_MINB = 2, 3 or 4 minimum resident CTAs)
     const char* ev = getenv("KTILER_PERSIST_MINB");
     int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
-    P->pfn = mb >= 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>);
+    P->pfn = mb >= 5 ? persistent_kernel<5> : (mb == 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>));
   }
   P->psmem = 0;
   for (auto& n : g.nodes) {
@@ -657,7 +827,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   }
   P->pp.stage_bytes = P->psmem;
   P->psmem *= 2;
-  if (P->psmem > 48 * 1024) {
+  if (P->psmem > 32 * 1024) {
     cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
   }
@@ -844,6 +1014,10 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     if (p->pol.exec_mode == KTILER_EXEC_PERSISTENT) {
       ktiler_status s = setup_persistent(p);
       if (s) return s;
+    } else {
+      for (auto& L : p->launches)
+        if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar)
+          L.kp.use_tmap = make_tmap(p->g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
     }
   }
   switch (p->pol.exec_mode) {

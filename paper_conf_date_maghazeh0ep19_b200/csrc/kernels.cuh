@@ -22,6 +22,8 @@
 // Border: replicate (clamp-to-edge) at image edges only.
 #pragma once
 
+#include <cuda.h>  // CUtensorMap
+
 #include <cstdint>
 
 namespace ktd {
@@ -49,17 +51,6 @@ __device__ __forceinline__ void st16_stream(void* p, uint4 v, uint64_t pol) {
 __device__ __forceinline__ void discard_line(const void* p) {
   asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
 }
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async16_hint(void* smem, const void* gmem, uint64_t pol) {
-  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 __device__ __forceinline__ int64_t clampi(int64_t v, int64_t lo, int64_t hi) { return v < lo ? lo : (v > hi ? hi : v); }
 __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t s) { return __byte_perm(a, b, s); }
@@ -71,7 +62,10 @@ __device__ __forceinline__ uint32_t lds4(const uint8_t* p) { return *reinterpret
 
 struct Tile {
   int64_t z, x0, y0, x1, y1;  // output rect [x0,x1) x [y0,y1) of frame z
+  int fw;                     // full tile width (px): fixes the staging row stride, so
+  int pad;                    // ragged edge tiles use the same layout as the TMA box
   __device__ int nseg() const { return (int)((x1 - x0 + 15) >> 4); }
+  __device__ int fseg() const { return (fw + 15) >> 4; }
   __device__ int rows() const { return (int)(y1 - y0); }
 };
 
@@ -131,6 +125,50 @@ __device__ void scalar_tile(int op, const DBuf& in, const DBuf& out, const Tile&
 constexpr int BLUR_R = 8;
 constexpr int SOBEL_R = 2;
 
+// ---- TMA bulk copies completing on an mbarrier (the Blackwell async proxy) ----
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* m, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(count) : "memory");
+}
+// make mbarrier inits / generic smem accesses visible to the async proxy
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void mbar_arrive_expect(uint64_t* m, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* m) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(m))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* m, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred P;\n KT_WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n @!P bra KT_WAIT_%=;\n}" ::"r"(
+          smem_u32(m)),
+      "r"(parity)
+      : "memory");
+}
+
+// Staged window of op's input for tile t: rows [ry0, ry0+nr) (clamped to the image for the
+// stencils), byte columns [xb0, xb0 + stride) (negative / beyond-width columns of the
+// stencils are filled by stage_fix with the replicate rule).
+struct StageGeo {
+  int64_t ry0, xb0, limit;  // limit = roundup16(row bytes) <= pitch
+  int nr, stride;
+  bool halo;
+};
+__device__ __forceinline__ int64_t up16(int64_t v) { return (v + 15) & ~(int64_t)15; }
+__device__ __forceinline__ StageGeo stage_geo(int op, const DBuf& in, const Tile& t) {
+  const int nseg = t.fseg(), rows = t.rows();
+  switch (op) {
+    case 0: return {t.y0, 3 * t.x0, up16(3 * in.W), rows, 48 * nseg, false};
+    case 1: return {t.y0 - 2, t.x0 - 16, up16(in.W), rows + 4, 16 * (nseg + 2), true};
+    case 2: return {2 * t.y0, 2 * t.x0, up16(in.W), 2 * rows, 32 * nseg, false};
+    case 3: return {t.y0 - 1, t.x0 - 16, up16(in.W), rows + 2, 16 * (nseg + 2), true};
+    default: return {t.y0, 4 * t.x0, up16(4 * in.W), rows, 64 * nseg, false};
+  }
+}
+
 // Shared memory one staged input tile of op needs for an output tile tw x th.
 __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
   const int nseg = (tw + 15) / 16;
@@ -144,64 +182,76 @@ __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
   return 0;
 }
 
-// Row-contiguous staging: nr rows starting at image row ry0 (step 1), byte span
-// [xb, xb + cpr*16) per row, only chunks that start inside the row's data (< limit); the
-// chunk end never passes the pitch (pitch >= roundup16(width*elem)).
-__device__ __forceinline__ void stage_rows(const DBuf& in, int64_t z, int64_t ry0, int nr, int64_t xb, int cpr,
-                                           int64_t limit, uint8_t* sm, int nt, int tid, bool stream, uint64_t pol) {
-  const int total = nr * cpr;
-  for (int i = tid; i < total; i += nt) {
-    const int r = i / cpr, c = i - r * cpr;
-    const int64_t off = xb + 16 * c;
-    if (off < limit) {
-      const uint8_t* src = row_ptr(in, z, ry0 + r) + off;
-      uint8_t* dst = sm + r * (16 * cpr) + 16 * c;
-      // (cp.async with an L2::cache_hint operand mis-encodes its descriptor register in
-      // this toolchain -> illegal instruction on sm_100a; the read-once input goes plain)
-      (void)stream;
-      (void)pol;
-      cp_async16(dst, src);
+// Issue the staging of op's input for tile t with one bulk copy per row (TMA), completing
+// on mbarrier m.  Called by ONE warp (lane = its lane id); no wait.
+__device__ __forceinline__ void stage_issue(int op, const DBuf& in, const Tile& t, uint8_t* sm, uint64_t* m, int lane) {
+  const StageGeo g = stage_geo(op, in, t);
+  const int64_t lo = g.xb0 > 0 ? g.xb0 : 0;
+  const int64_t hi = g.xb0 + g.stride < g.limit ? g.xb0 + g.stride : g.limit;
+  const unsigned bytes = (unsigned)(hi - lo);
+  if (lane == 0) mbar_arrive_expect(m, bytes * (unsigned)g.nr);
+  __syncwarp();
+  for (int r = lane; r < g.nr; r += 32) {
+    const int64_t y = g.halo ? clampi(g.ry0 + r, 0, in.H - 1) : g.ry0 + r;
+    bulk_g2s(sm + r * g.stride + (lo - g.xb0), row_ptr(in, t.z, y) + lo, bytes, m);
+  }
+}
+
+// Tensor-map TMA (the fast path): ONE cp.async.bulk.tensor.3d per tile, issued by one
+// thread.  The map views the input buffer as 4-byte elements [frames][rows][row/4]; the box
+// is the whole staged window (stage_geo at full tile size), so out-of-image rows/columns
+// of a halo come back zero-filled and are fixed by stage_fix (replicate).  box_bytes is the
+// full box (also for ragged edge tiles, whose extra bytes are ignored).
+__device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map, unsigned box_bytes, const DBuf& in,
+                                                 const Tile& t, uint8_t* sm, uint64_t* m) {
+  const StageGeo g = stage_geo(op, in, t);
+  mbar_arrive_expect(m, box_bytes);
+  const int x = (int)(g.xb0 >> 2), y = (int)g.ry0, z = (int)t.z;
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
+          smem_u32(sm)),
+      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(m))
+      : "memory");
+}
+
+// After the copies landed (stencils only): replicate-fill the halo outside the image —
+// columns < 0 / >= W from pixel 0 / W-1 of the same row, then rows < 0 / >= H as copies of
+// the nearest image row — so the staged window holds in[clamp(y)][clamp(x)].  All threads;
+// the caller synchronizes afterwards.  Returns quickly for interior tiles.
+__device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid) {
+  if (op != 1 && op != 3) return;
+  const StageGeo g = stage_geo(op, in, t);
+  const int left = g.xb0 < 0 ? (int)(-g.xb0) : 0;                                       // columns < 0
+  const int rfrom = (int)(in.W - g.xb0) < g.stride ? (int)(in.W - g.xb0) : g.stride;      // columns >= W
+  const int right = g.stride - rfrom;
+  const int top = g.ry0 < 0 ? (int)(-g.ry0) : 0;                                         // rows < 0
+  const int bfrom = (int)(in.H - g.ry0) < g.nr ? (int)(in.H - g.ry0) : g.nr;              // rows >= H
+  const int per = left + right;
+  if (per) {
+    for (int i = tid; i < (bfrom - top) * per; i += nt) {
+      const int r = top + i / per, k = i % per;
+      uint8_t* row = sm + r * g.stride;
+      if (k < left) row[k] = row[left];                 // pixel 0
+      else row[rfrom + (k - left)] = row[rfrom - 1];    // pixel W-1
+    }
+  }
+  if (top || bfrom < g.nr) {
+    if (per) asm volatile("bar.sync 4, %0;" ::"r"(nt) : "memory");  // the nt staging threads only
+    const int n16 = g.stride >> 4, nfix = top + (g.nr - bfrom);
+    for (int i = tid; i < nfix * n16; i += nt) {
+      const int j = i / n16, c = i % n16;
+      const int r = j < top ? j : bfrom + (j - top);
+      const int src = j < top ? top : bfrom - 1;
+      reinterpret_cast<uint4*>(sm + r * g.stride)[c] = reinterpret_cast<const uint4*>(sm + src * g.stride)[c];
     }
   }
 }
 
-// Halo staging of a u8 tile: rows [ya, ya+nr) (clamped to [0,H)) and byte columns
-// [xs, xs + 16*nc) (clamped, replicate), row stride 16*nc.  Interior chunks move with
-// cp.async.cg; chunks crossing an image edge are gathered byte by byte.
-__device__ __forceinline__ void stage_halo(const DBuf& in, int64_t z, int64_t ya, int nr, int64_t xs, int nc,
-                                           uint8_t* sm, int nt, int tid) {
-  const int total = nr * nc;
-  for (int i = tid; i < total; i += nt) {
-    const int r = i / nc, c = i - r * nc;
-    const uint8_t* row = row_ptr(in, z, clampi(ya + r, 0, in.H - 1));
-    const int64_t x = xs + 16 * c;
-    uint8_t* d = sm + r * (16 * nc) + 16 * c;
-    if (x >= 0 && x + 16 <= in.W) {
-      cp_async16(d, row + x);
-    } else {
-      uint32_t w[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        uint32_t v = 0;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) v |= (uint32_t)ld1(row + clampi(x + 4 * q + j, 0, in.W - 1)) << (8 * j);
-        w[q] = v;
-      }
-      *reinterpret_cast<uint4*>(d) = make_uint4(w[0], w[1], w[2], w[3]);
-    }
-  }
-}
-
-// Issue the staging of op's input for tile t (no wait; the caller commits / waits).
-__device__ __forceinline__ void stage_tile(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid) {
-  const int nseg = t.nseg(), rows = t.rows();
-  switch (op) {
-    case 0: stage_rows(in, t.z, t.y0, rows, 3 * t.x0, 3 * nseg, 3 * in.W, sm, nt, tid, true, policy_evict_first()); break;
-    case 1: stage_halo(in, t.z, t.y0 - 2, rows + 4, t.x0 - 16, nseg + 2, sm, nt, tid); break;
-    case 2: stage_rows(in, t.z, 2 * t.y0, 2 * rows, 2 * t.x0, 2 * nseg, in.W, sm, nt, tid, false, 0); break;
-    case 3: stage_halo(in, t.z, t.y0 - 1, rows + 2, t.x0 - 16, nseg + 2, sm, nt, tid); break;
-    case 4: stage_rows(in, t.z, t.y0, rows, 4 * t.x0, 4 * nseg, 4 * in.W, sm, nt, tid, false, 0); break;
-  }
+// Does tile t of a stencil op need stage_fix?  (CTA-uniform)
+__device__ __forceinline__ bool needs_fix(int op, const DBuf& in, const Tile& t) {
+  if (op != 1 && op != 3) return false;
+  const StageGeo g = stage_geo(op, in, t);
+  return g.xb0 < 0 || g.xb0 + g.stride > in.W || g.ry0 < 0 || g.ry0 + g.nr > in.H;
 }
 
 __device__ __forceinline__ void store_u8_16(uint8_t* d, int64_t x, int64_t W, uint4 o) {
@@ -246,16 +296,43 @@ __device__ __forceinline__ uint4 gray16(const uint32_t w[12]) {
   return o;
 }
 
+// Items of a tile = (row group g, 16-px column segment s).  When nt is a multiple of
+// nseg every thread keeps a fixed segment and strides over row groups: one division per
+// tile, no per-item index arithmetic.
+template <class F>
+__device__ __forceinline__ void for_items(int nseg, int ngrp, int nt, int tid, F&& f) {
+  if (nseg == 16) {  // the B200 geometry: 256-pixel-wide tiles
+    const int s = tid & 15, gstep = nt >> 4;
+    for (int g = tid >> 4; g < ngrp; g += gstep) f(g, s);
+  } else if (nt % nseg == 0) {
+    const int s = tid % nseg, gstep = nt / nseg;
+    for (int g = tid / nseg; g < ngrp; g += gstep) f(g, s);
+  } else {
+    for (int it = tid; it < nseg * ngrp; it += nt) {
+      const int g = it / nseg;
+      f(g, it - g * nseg);
+    }
+  }
+}
+
+// Output base of a tile (pixel (x0, y0) of frame z) and its "all segments full" flag.
+__device__ __forceinline__ uint8_t* tile_out(const DBuf& out, const Tile& t, int elem) {
+  return out.p + t.z * out.fstride + t.y0 * out.pitch + t.x0 * elem;
+}
+
 __device__ void gray_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
-  const int nseg = t.nseg(), items = nseg * t.rows(), stride = 48 * nseg;
-  for (int it = tid; it < items; it += nt) {
-    const int r = it / nseg, s = it - r * nseg;
+  const int nseg = t.nseg(), stride = 48 * t.fseg();
+  const bool full = (t.x1 - t.x0) == 16 * nseg;
+  uint8_t* const ob = tile_out(out, t, 1);
+  const int pitch = (int)out.pitch;
+  for_items(nseg, t.rows(), nt, tid, [&](int r, int s) {
     const uint8_t* p = sm + r * stride + 48 * s;
     uint4 a = lds16(p), b = lds16(p + 16), c = lds16(p + 32);
     const uint32_t w[12] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w, c.x, c.y, c.z, c.w};
-    const int64_t x = t.x0 + 16 * s;
-    store_u8_16(const_cast<uint8_t*>(row_ptr(out, t.z, t.y0 + r)) + x, x, out.W, gray16(w));
-  }
+    uint8_t* d = ob + r * pitch + 16 * s;
+    const uint4 o = gray16(w);
+    if (full) st16(d, o); else store_u8_16(d, t.x0 + 16 * s, out.W, o);
+  });
 }
 
 // ---------------------------------------------------------------------------------
@@ -308,29 +385,30 @@ __device__ __forceinline__ uint4 vblur_pack(const uint32_t* h0, const uint32_t* 
 
 template <int R>
 __device__ void blur_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
-  const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (nseg + 2);
-  const int ngrp = (rows + R - 1) / R, items = nseg * ngrp;
-  for (int it = tid; it < items; it += nt) {
-    const int g = it / nseg, s = it - g * nseg;
+  const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (t.fseg() + 2);
+  const bool full = (t.x1 - t.x0) == 16 * nseg;
+  uint8_t* const ob = tile_out(out, t, 1);
+  const int pitch = (int)out.pitch;
+  for_items(nseg, (rows + R - 1) / R, nt, tid, [&](int g, int s) {
     const int ra = g * R, rb = min(ra + R, rows);
-    const uint8_t* col = sm + 16 * (s + 1);  // staged row r holds image row y0 - 2 + r
-    const int64_t x = t.x0 + 16 * s;
+    const uint8_t* col = sm + 16 * (s + 1) + ra * stride;  // staged row r holds image row y0 - 2 + r
+    uint8_t* d = ob + ra * pitch + 16 * s;
     uint32_t h[5][8];
     uint32_t w[6];
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
-      smem_window(col + (ra + i) * stride, w);
+      smem_window(col + i * stride, w);
       hblur16(w, h[i]);
     }
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (ra + r >= rb) break;
-      smem_window(col + (ra + r + 4) * stride, w);
+      smem_window(col + (r + 4) * stride, w);
       hblur16(w, h[(r + 4) % 5]);
-      uint4 o = vblur_pack(h[r % 5], h[(r + 1) % 5], h[(r + 2) % 5], h[(r + 3) % 5], h[(r + 4) % 5]);
-      store_u8_16(const_cast<uint8_t*>(row_ptr(out, t.z, t.y0 + ra + r)) + x, x, out.W, o);
+      const uint4 o = vblur_pack(h[r % 5], h[(r + 1) % 5], h[(r + 2) % 5], h[(r + 3) % 5], h[(r + 4) % 5]);
+      if (full) st16(d + r * pitch, o); else store_u8_16(d + r * pitch, t.x0 + 16 * s, out.W, o);
     }
-  }
+  });
 }
 
 // ---------------------------------------------------------------------------------
@@ -346,17 +424,19 @@ __device__ __forceinline__ uint32_t down4(uint32_t a0, uint32_t a1, uint32_t b0,
 }
 
 __device__ void down_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
-  const int nseg = t.nseg(), items = nseg * t.rows(), stride = 32 * nseg;
-  for (int it = tid; it < items; it += nt) {
-    const int r = it / nseg, s = it - r * nseg;
+  const int nseg = t.nseg(), stride = 32 * t.fseg();
+  const bool full = (t.x1 - t.x0) == 16 * nseg;
+  uint8_t* const ob = tile_out(out, t, 1);
+  const int pitch = (int)out.pitch;
+  for_items(nseg, t.rows(), nt, tid, [&](int r, int s) {
     const uint8_t* p0 = sm + (2 * r) * stride + 32 * s;
     const uint8_t* p1 = p0 + stride;
     uint4 a = lds16(p0), b = lds16(p0 + 16), c = lds16(p1), e = lds16(p1 + 16);
     const uint4 o = make_uint4(down4(a.x, a.y, c.x, c.y), down4(a.z, a.w, c.z, c.w), down4(b.x, b.y, e.x, e.y),
                                down4(b.z, b.w, e.z, e.w));
-    const int64_t x = t.x0 + 16 * s;
-    store_u8_16(const_cast<uint8_t*>(row_ptr(out, t.z, t.y0 + r)) + x, x, out.W, o);
-  }
+    uint8_t* d = ob + r * pitch + 16 * s;
+    if (full) st16(d, o); else store_u8_16(d, t.x0 + 16 * s, out.W, o);
+  });
 }
 
 // ---------------------------------------------------------------------------------
@@ -384,27 +464,34 @@ __device__ __forceinline__ float lane_f(uint32_t w, bool hi) {
   const float f = __uint_as_float(prmt(w, 0x4B000000u, hi ? 0x7632 : 0x7610));
   return f - 8389628.0f;  // 2^23 + 1020
 }
-__device__ __forceinline__ float mag(float gx, float gy) { return __fsqrt_rn(__fmaf_rn(gx, gx, __fmul_rn(gy, gy))); }
+// sqrt_rn of the exact sum; s = 0 (flat regions) would take __fsqrt_rn's special-case
+// subroutine, so it is evaluated on max(s, 1) and selected away.
+__device__ __forceinline__ float mag(float gx, float gy) {
+  const float s = __fmaf_rn(gx, gx, __fmul_rn(gy, gy));
+  const float r = __fsqrt_rn(fmaxf(s, 1.0f));
+  return s > 0.0f ? r : 0.0f;
+}
 
 template <int R>
 __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
-  const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (nseg + 2);
-  const int ngrp = (rows + R - 1) / R, items = nseg * ngrp;
-  for (int it = tid; it < items; it += nt) {
-    const int g = it / nseg, s = it - g * nseg;
+  const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (t.fseg() + 2);
+  const bool full = (t.x1 - t.x0) == 16 * nseg;
+  uint8_t* const ob = tile_out(out, t, 4);
+  const int pitch = (int)out.pitch;
+  for_items(nseg, (rows + R - 1) / R, nt, tid, [&](int g, int s) {
     const int ra = g * R, rb = min(ra + R, rows);
-    const uint8_t* col = sm + 16 * (s + 1);  // staged row r holds image row y0 - 1 + r
-    const int64_t x = t.x0 + 16 * s;
+    const uint8_t* col = sm + 16 * (s + 1) + ra * stride;  // staged row r holds image row y0 - 1 + r
+    uint8_t* drow = ob + ra * pitch + 64 * s;
     SobelRow w[3];
     uint32_t tw[6];
-    smem_window(col + ra * stride, tw);
+    smem_window(col, tw);
     sobel_split(tw, w[0]);
-    smem_window(col + (ra + 1) * stride, tw);
+    smem_window(col + stride, tw);
     sobel_split(tw, w[1]);
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (ra + r >= rb) break;
-      smem_window(col + (ra + r + 2) * stride, tw);
+      smem_window(col + (r + 2) * stride, tw);
       sobel_split(tw, w[(r + 2) % 3]);
       const SobelRow& T = w[r % 3];
       const SobelRow& M = w[(r + 1) % 3];
@@ -417,7 +504,7 @@ __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm,
         DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
         DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
       }
-      float* dst = reinterpret_cast<float*>(const_cast<uint8_t*>(row_ptr(out, t.z, t.y0 + ra + r))) + x;
+      float* dst = reinterpret_cast<float*>(drow + r * pitch);
       float m[16];
 #pragma unroll
       for (int q = 1; q <= 4; ++q) {
@@ -431,18 +518,19 @@ __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm,
         m[b + 2] = mag(lane_f(gxe, true), lane_f(gye, true));
         m[b + 3] = mag(lane_f(gxo, true), lane_f(gyo, true));
       }
-      if (x + 16 <= out.W) {
+      if (full || t.x0 + 16 * s + 16 <= out.W) {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
           st16(dst + 4 * q, make_uint4(__float_as_uint(m[4 * q]), __float_as_uint(m[4 * q + 1]),
                                        __float_as_uint(m[4 * q + 2]), __float_as_uint(m[4 * q + 3])));
       } else {
+        const int64_t x = t.x0 + 16 * s;
 #pragma unroll
         for (int k = 0; k < 16; ++k)
           if (x + k < out.W) dst[k] = m[k];
       }
     }
-  }
+  });
 }
 
 // ---------------------------------------------------------------------------------
@@ -456,15 +544,16 @@ __device__ __forceinline__ uint32_t gt4(uint4 v, float T) {
 
 __device__ void thresh_compute(const DBuf& out, const Tile& t, const uint8_t* sm, float T, int nt, int tid) {
   const uint64_t pol = policy_evict_first();
-  const int nseg = t.nseg(), items = nseg * t.rows(), stride = 64 * nseg;
-  for (int it = tid; it < items; it += nt) {
-    const int r = it / nseg, s = it - r * nseg;
+  const int nseg = t.nseg(), stride = 64 * t.fseg();
+  const bool full = (t.x1 - t.x0) == 16 * nseg;
+  uint8_t* const ob = tile_out(out, t, 1);
+  const int pitch = (int)out.pitch;
+  for_items(nseg, t.rows(), nt, tid, [&](int r, int s) {
     const uint8_t* p = sm + r * stride + 64 * s;
     const uint4 o = make_uint4(gt4(lds16(p), T), gt4(lds16(p + 16), T), gt4(lds16(p + 32), T), gt4(lds16(p + 48), T));
-    const int64_t x = t.x0 + 16 * s;
-    uint8_t* d = const_cast<uint8_t*>(row_ptr(out, t.z, t.y0 + r)) + x;
-    if (x + 16 <= out.W) st16_stream(d, o, pol); else store_u8_16(d, x, out.W, o);
-  }
+    uint8_t* d = ob + r * pitch + 16 * s;
+    if (full) st16_stream(d, o, pol); else store_u8_16(d, t.x0 + 16 * s, out.W, o);
+  });
 }
 
 // Compute op's output tile from its staged input (after the staging is complete).
@@ -479,16 +568,17 @@ __device__ __forceinline__ void compute_tile(int op, const DBuf& out, const Tile
   }
 }
 
-// One whole block (stream / graph modes): stage, wait, compute.
+// One whole block (stream / graph modes): stage (TMA), wait, fix edges, compute.
+// m: an mbarrier in shared memory initialised with count 1 (phase 0 unused before).
 __device__ __forceinline__ void run_tile(int op, bool scalar, const DBuf& in, const DBuf& out, const Tile& t, float T,
-                                         int nt, int tid, uint8_t* sm) {
+                                         int nt, int tid, uint8_t* sm, uint64_t* m) {
   if (scalar) {
     scalar_tile(op, in, out, t, T, nt, tid);
     return;
   }
-  stage_tile(op, in, t, sm, nt, tid);
-  cp_async_commit();
-  cp_async_wait<0>();
+  if (tid < 32) stage_issue(op, in, t, sm, m, tid);
+  mbar_wait(m, 0);
+  stage_fix(op, in, t, sm, nt, tid);
   __syncthreads();
   compute_tile(op, out, t, sm, T, nt, tid);
 }
