@@ -379,13 +379,28 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
     // every iteration, so no runtime-indexed arrays (they would live in local memory)
     uint64_t d_this = 0, d_other = 0;
     bool u_this = false, u_other = false;
+    // Reorder window: up to 4 taken-but-unstaged tickets, oldest first.  The control warp
+    // stages the oldest one whose producers are complete, so a not-yet-ready consumer does
+    // not idle the CTA; if none is ready it waits for the oldest (always runnable once
+    // every smaller ticket is done, so the executor stays deadlock-free).
+    uint64_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
+    int nw = 0;
+    bool more = true;
     int b = 0;
     for (;; b ^= 1) {
-      const int64_t t = __shfl_sync(FULL, tq, 0);
-      const uint64_t d = __shfl_sync(FULL, dq, 0);
-      if (lane == 0 && t < p.total) {  // next grab; consumed next iteration
-        tq = atomicAdd(&p.ctrl->ticket, 1u);
-        dq = tq < p.total ? p.desc[tq] : 0;
+      while (nw < 4 && more) {  // refill the window (one grab in steady state)
+        const int64_t t = __shfl_sync(FULL, tq, 0);
+        const uint64_t d = __shfl_sync(FULL, dq, 0);
+        if (t >= p.total) {
+          more = false;
+          break;
+        }
+        if (lane == 0) {
+          tq = atomicAdd(&p.ctrl->ticket, 1u);
+          dq = tq < p.total ? p.desc[tq] : 0;
+        }
+        if (nw == 0) w0 = d; else if (nw == 1) w1 = d; else if (nw == 2) w2 = d; else w3 = d;
+        ++nw;
       }
       // buffer b is free once the compute warps are done with the tile two back
       if (u_this) {
@@ -393,22 +408,33 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
         ctl_release(p, decode(p, d_this), epoch, lane);
         u_this = false;
       }
-      if (t >= p.total) {
+      if (nw == 0) {
         if (lane == 0) {
           s_desc[b] = DESC_STOP;
           mbar_arrive(&s_full[b]);
         }
         break;
       }
-      const TInfo a = decode(p, d);
-      if (!ctl_probe(p, a, epoch, lane)) {
+      int ch = -1;
+      if (ctl_probe(p, decode(p, w0), epoch, lane)) ch = 0;
+      else if (nw > 1 && ctl_probe(p, decode(p, w1), epoch, lane)) ch = 1;
+      else if (nw > 2 && ctl_probe(p, decode(p, w2), epoch, lane)) ch = 2;
+      else if (nw > 3 && ctl_probe(p, decode(p, w3), epoch, lane)) ch = 3;
+      if (ch < 0) {
         if (u_other) {  // never wait while holding an unreleased tile
           nbar_sync(1 + (b ^ 1), PERSIST_THREADS);
           ctl_release(p, decode(p, d_other), epoch, lane);
           u_other = false;
         }
-        ctl_wait(p, a, epoch, lane);
+        ctl_wait(p, decode(p, w0), epoch, lane);
+        ch = 0;
       }
+      const uint64_t d = ch == 0 ? w0 : (ch == 1 ? w1 : (ch == 2 ? w2 : w3));
+      if (ch <= 0) w0 = w1;
+      if (ch <= 1) w1 = w2;
+      if (ch <= 2) w2 = w3;
+      --nw;
+      const TInfo a = decode(p, d);
       uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
       if (lane == 0) {
         s_desc[b] = d;
@@ -504,6 +530,7 @@ struct Launch {
   dim3 block;
   int smem = 0;
   int64_t resident = 0;  // CTAs of this kernel that fit the device at once
+  int sub = -1;          // schedule sub-kernel (kernel launches) / discard list (DAG discards)
   std::vector<int32_t> crects;  // OP_CUSTOM rect list
 };
 
@@ -515,6 +542,7 @@ struct ktiler_plan_s {
   ktiler_fragment_policy pol{};
   double plan_ms = 0;
   std::vector<Launch> launches;
+  std::vector<Launch> dag_disc;  // GRAPH_DAG: discard launches (sub = the discard list)
   int device = -1;
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
@@ -560,6 +588,7 @@ void build_launches(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
   const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
+  const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG;
   std::vector<DRect> pending;
   auto flush_disc_only = [&](size_t keep) {
     while (pending.size() > keep) {
@@ -617,7 +646,8 @@ void build_launches(ktiler_plan_s* P) {
           L.kp.rpre[i + 1] = L.kp.rpre[i] + q.count();
         }
         L.blocks = L.kp.rpre[m];
-        if (c == 0 && !pending.empty()) {
+        L.sub = (int)si;
+        if (!dag && c == 0 && !pending.empty()) {
           size_t nd = std::min<size_t>(MAXD, pending.size());
           L.kp.ndisc = (int32_t)nd;
           L.kp.dpre[0] = 0;
@@ -639,6 +669,15 @@ void build_launches(ktiler_plan_s* P) {
         DRect dr = drect(g, d);
         if (dr.lpr > 0) pending.push_back(dr);
       }
+    if (dag && !pending.empty()) {  // one discard node per list (chunks of MAXD rects)
+      const size_t base = P->launches.size();
+      flush_disc_only(0);
+      for (size_t k = base; k < P->launches.size(); ++k) {
+        P->launches[k].sub = (int)si;
+        P->dag_disc.push_back(P->launches[k]);
+      }
+      P->launches.resize(base);
+    }
   }
   flush_disc_only(0);
 }
@@ -696,26 +735,120 @@ ktiler_status cuda_fail(cudaError_t e, const char* what) {
   return fail(KTILER_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
+kfn_t launch_fn(const Launch& L) {
+  return L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
+}
+
+// Dynamic-smem attribute + grid of one launch: the vector kernels grid-stride over their
+// tiles with as many CTAs as fit the device at once.
+ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_out) {
+  if (L.resident == 0 && L.smem > 32 * 1024) {  // static + dynamic may pass the 48 KB default
+    cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
+    if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
+  }
+  if (L.resident == 0) {
+    int nsm = 0, occ = 0;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)(L.block.x * L.block.y * L.block.z), L.smem);
+    L.resident = (int64_t)std::max(1, nsm) * std::max(1, occ);
+  }
+  int64_t grid = std::max<int64_t>(L.blocks, 1);
+  // grid-stride CTAs (x tiles_per_cta) in stream/graph modes; in GRAPH_DAG one CTA per
+  // tile by default, so concurrent sub-kernels interleave at tile granularity
+  static const int tpc_env = getenv("KTILER_TILES_PER_CTA") ? atoi(getenv("KTILER_TILES_PER_CTA")) : -1;
+  const int tpc = tpc_env >= 0 ? tpc_env : (P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG ? 1 : 0);
+  if (L.node >= 0 && !L.n->scalar) {
+    if (tpc > 0) grid = (grid + tpc - 1) / tpc;
+    else grid = std::min<int64_t>(grid, L.resident);
+  }
+  if (L.kp.ndisc) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+  *grid_out = grid;
+  return KTILER_OK;
+}
+
+// GRAPH_DAG: the sub-kernels as graph nodes whose edges are their exact dependencies
+// (Schedule::sub_deps), the previous sub-kernel of the same kernel (keeps each kernel's
+// order), and a run-ahead window — a source sub-kernel of fragment f waits for the leaf
+// sub-kernels of fragment f - window — so at most `window` fragments are in flight (the
+// L2 footprint stays bounded) while their launches overlap each other's gaps and tails.
+// A discard node waits for every sub-kernel that reads the blocks it retires.
+ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
+  const kt::Schedule& S = P->s;
+  const kt::Graph& g = P->g;
+  const int nsub = (int)S.subs.size();
+  const int window = P->pol.window > 0 ? P->pol.window : 2;
+  cudaGraph_t gr = nullptr;
+  cudaError_t e = cudaGraphCreate(&gr, 0);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGraphCreate");
+  std::vector<std::vector<cudaGraphNode_t>> nodes_of(nsub);
+  std::vector<std::vector<int>> leaf_subs(S.nfrag);
+  for (int i = 0; i < nsub; ++i)
+    if (g.out_ch[S.subs[i].node].empty()) leaf_subs[S.subs[i].frag].push_back(i);
+  std::vector<int> last_of_node(g.nodes.size(), -1);
+  auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, cudaGraphNode_t* node) -> ktiler_status {
+    kfn_t fn = launch_fn(L);
+    int64_t grid = 0;
+    ktiler_status ps = prep_launch(P, L, fn, &grid);
+    if (ps) return ps;
+    void* args[1] = {&L.kp};
+    cudaKernelNodeParams kp = {};
+    kp.func = (void*)fn;
+    kp.gridDim = dim3((unsigned)grid);
+    kp.blockDim = L.block;
+    kp.sharedMemBytes = (unsigned)L.smem;
+    kp.kernelParams = args;
+    cudaError_t ee = cudaGraphAddKernelNode(node, gr, deps.data(), deps.size(), &kp);
+    if (ee != cudaSuccess) return cuda_fail(ee, "cudaGraphAddKernelNode");
+    return KTILER_OK;
+  };
+  size_t li = 0;
+  for (int i = 0; i < nsub; ++i) {
+    std::vector<cudaGraphNode_t> deps;
+    for (int d : S.sub_deps[i]) deps.insert(deps.end(), nodes_of[d].begin(), nodes_of[d].end());
+    const int prev = last_of_node[S.subs[i].node];
+    if (prev >= 0) deps.insert(deps.end(), nodes_of[prev].begin(), nodes_of[prev].end());
+    const int f = S.subs[i].frag;
+    if (S.sub_deps[i].empty() && f >= window)
+      for (int j : leaf_subs[f - window]) deps.insert(deps.end(), nodes_of[j].begin(), nodes_of[j].end());
+    std::sort(deps.begin(), deps.end());
+    deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
+    for (; li < P->launches.size() && P->launches[li].sub == i; ++li) {
+      cudaGraphNode_t nd;
+      ktiler_status st = add_node(P->launches[li], deps, &nd);
+      if (st) {
+        cudaGraphDestroy(gr);
+        return st;
+      }
+      nodes_of[i].push_back(nd);
+    }
+    last_of_node[S.subs[i].node] = i;
+  }
+  for (auto& D : P->dag_disc) {
+    std::vector<cudaGraphNode_t> deps;
+    for (int r : S.discard_readers[D.sub]) deps.insert(deps.end(), nodes_of[r].begin(), nodes_of[r].end());
+    std::sort(deps.begin(), deps.end());
+    deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
+    cudaGraphNode_t nd;
+    ktiler_status st = add_node(D, deps, &nd);
+    if (st) {
+      cudaGraphDestroy(gr);
+      return st;
+    }
+  }
+  *out = gr;
+  return KTILER_OK;
+}
+
 ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
   for (auto& L : P->launches) {
     if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
       L.n->launch(L.n->user, L.crects.data(), (int32_t)(L.crects.size() / 6), (void*)st);
       continue;
     }
-    kfn_t fn = L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
-    if (L.resident == 0 && L.smem > 32 * 1024) {  // static + dynamic may pass the 48 KB default
-      cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
-      if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
-    }
-    if (L.resident == 0) {  // CTAs that fit at once: the vector kernels grid-stride over tiles
-      int nsm = 0, occ = 0;
-      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, (int)(L.block.x * L.block.y * L.block.z), L.smem);
-      L.resident = (int64_t)std::max(1, nsm) * std::max(1, occ);
-    }
-    int64_t grid = std::max<int64_t>(L.blocks, 1);
-    if (L.node >= 0 && !L.n->scalar) grid = std::min<int64_t>(grid, L.resident);
-    if (L.kp.ndisc) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+    kfn_t fn = launch_fn(L);
+    int64_t grid = 0;
+    ktiler_status ps = prep_launch(P, L, fn, &grid);
+    if (ps) return ps;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = L.block;
@@ -920,7 +1053,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
   kt::Graph* G = kt::graph_of(gh);
   ktiler_status s = G->finalize();
   if (s) return s;
-  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_PERSISTENT)
+  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_DAG)
     return fail(KTILER_E_INVALID, "unknown exec_mode");
   if (cache_bytes == 0) {
     int dev = 0, l2 = 0;
@@ -991,7 +1124,7 @@ ktiler_status ktiler_plan_get_stats(ktiler_plan_t p, ktiler_plan_stats* out) {
   std::memset(out, 0, sizeof(*out));
   out->n_subkernels = (int64_t)p->s.subs.size();
   out->n_fragments = p->s.nfrag;
-  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT ? 1 : (int64_t)p->launches.size();
+  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT ? 1 : (int64_t)(p->launches.size() + p->dag_disc.size());
   out->n_discard_lines = (p->pol.flags & KTILER_PF_DISCARD_DEAD) ? p->s.discard_lines : 0;
   out->budget_bytes = p->s.budget;
   out->max_footprint_bytes = p->s.max_footprint;
@@ -1024,6 +1157,18 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     case KTILER_EXEC_STREAM: {
       ktiler_status s = enqueue(p, st);
       if (s) return s;
+      break;
+    }
+    case KTILER_EXEC_GRAPH_DAG: {
+      if (!p->exec) {
+        if (p->has_custom) return fail(KTILER_E_UNSUPPORTED, "GRAPH_DAG runs built-in ops only");
+        cudaGraph_t gr = nullptr;
+        ktiler_status s = build_dag(p, &gr);
+        if (s) return s;
+        p->graph = gr;
+        if ((e = cudaGraphInstantiate(&p->exec, gr, 0)) != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+      }
+      if ((e = cudaGraphLaunch(p->exec, st)) != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
       break;
     }
     case KTILER_EXEC_GRAPH:

@@ -145,6 +145,11 @@ struct Schedule {
   // discards[i] = ranges that become dead once subs[i] has completed
   std::vector<std::vector<Discard>> discards;
   int64_t discard_lines = 0;
+  // sub-kernel dependency sets (a sub-kernel depends on another iff one
+  // of its blocks depends on one of the other's) and, per discard list, every sub-kernel
+  // that reads the dying blocks (a discard may only run after all of them) — GRAPH_DAG
+  std::vector<std::vector<int32_t>> sub_deps;
+  std::vector<std::vector<int32_t>> discard_readers;
 };
 
 ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out);

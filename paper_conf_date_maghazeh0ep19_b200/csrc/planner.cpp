@@ -396,7 +396,30 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
           for (int64_t x = r.x0; x < r.x1; ++x) sub_of[n.gid0 + (z * n.gy() + y) * n.gx() + x] = (int32_t)i;
   }
   s.discards.assign(s.subs.size(), {});
+  s.discard_readers.assign(s.subs.size(), {});
   s.discard_lines = 0;
+  // sub-kernel dependencies: the producer sub-kernels of every block of each sub-kernel
+  s.sub_deps.assign(s.subs.size(), {});
+  for (size_t i = 0; i < s.subs.size(); ++i) {
+    const SubKernel& sk = s.subs[i];
+    std::vector<int32_t>& dep = s.sub_deps[i];
+    for (const Chan& c : g.in_ch[sk.node]) {
+      const Node& u = g.nodes[c.u];
+      for (auto& r : sk.rects)
+        for (int64_t z = r.z0; z < r.z1; ++z)
+          for (int64_t y = r.y0; y < r.y1; ++y)
+            for (int64_t x = r.x0; x < r.x1; ++x) {
+              BRange pr = g.producers(c, x, y);
+              for (int64_t py = pr.y0; py < pr.y1; ++py)
+                for (int64_t px = pr.x0; px < pr.x1; ++px) {
+                  const int32_t so = sub_of[u.gid0 + (z * u.gy() + py) * u.gx() + px];
+                  if (dep.empty() || dep.back() != so) dep.push_back(so);
+                }
+            }
+    }
+    std::sort(dep.begin(), dep.end());
+    dep.erase(std::unique(dep.begin(), dep.end()), dep.end());
+  }
   for (int u = 0; u < (int)g.nodes.size(); ++u) {
     const Node& n = g.nodes[u];
     const Access& w = n.acc[n.wacc];
@@ -407,15 +430,23 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
     for (int64_t l = 0; l < n.nblocks; ++l) {
       int64_t px = l % n.gx(), py = (l / n.gx()) % n.gy(), pz = l / (n.gx() * n.gy());
       int32_t last = sub_of[n.gid0 + l];
+      std::vector<int32_t> rd{last};
       for (const Chan& c : g.out_ch[u]) {
         if (c.buf != w.buf) continue;
         const Node& v = g.nodes[c.v];
         BRange r = g.consumers(c, px, py);
         for (int64_t y = r.y0; y < r.y1; ++y)
-          for (int64_t x = r.x0; x < r.x1; ++x)
-            last = std::max(last, sub_of[v.gid0 + (pz * v.gy() + y) * v.gx() + x]);
+          for (int64_t x = r.x0; x < r.x1; ++x) {
+            const int32_t sc = sub_of[v.gid0 + (pz * v.gy() + y) * v.gx() + x];
+            last = std::max(last, sc);
+            rd.push_back(sc);
+          }
       }
-      if (last >= 0) dead[last].push_back(l);
+      if (last >= 0) {
+        dead[last].push_back(l);
+        auto& R = s.discard_readers[last];
+        R.insert(R.end(), rd.begin(), rd.end());
+      }
     }
     const int64_t e = B.d.elem_bytes;
     for (size_t si = 0; si < dead.size(); ++si) {
@@ -461,6 +492,10 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
         s.discards[si].push_back(d);
       }
     }
+  }
+  for (auto& R : s.discard_readers) {
+    std::sort(R.begin(), R.end());
+    R.erase(std::unique(R.begin(), R.end()), R.end());
   }
   for (auto& v : s.discards)
     for (auto& d : v) {

@@ -19,11 +19,11 @@ BUF_INTERNAL = 1
 READ, WRITE = 1, 2
 OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM = range(6)
 FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE = range(4)
-EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT = range(4)
+EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG = range(5)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL = 1, 2, 4
 
 EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
-              "persistent": EXEC_PERSISTENT}
+              "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG}
 FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE}
 
 
@@ -57,7 +57,7 @@ class KernelDesc(ctypes.Structure):
 class Policy(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("l2_fraction", ctypes.c_double), ("rows", ctypes.c_int64),
                 ("exec_mode", ctypes.c_int32), ("flags", ctypes.c_uint32), ("persistent_ctas", ctypes.c_int32),
-                ("pipeline_skew", ctypes.c_int32)]
+                ("pipeline_skew", ctypes.c_int32), ("window", ctypes.c_int32)]
 
 
 class SubKernelInfo(ctypes.Structure):
@@ -201,11 +201,11 @@ class Graph:
 
     def plan(self, cache_bytes: int = 0, kind: str | int = "budget", l2_fraction: float = 1.0, rows: int = 1,
              exec_mode: str | int = "graph", discard: bool = False, pdl: bool = False, force_minimal: bool = False,
-             persistent_ctas: int = 0, skew: int = 0) -> "Plan":
+             persistent_ctas: int = 0, skew: int = 0, window: int = 0) -> "Plan":
         k = FRAG_KINDS[kind] if isinstance(kind, str) else kind
         m = EXEC_MODES[exec_mode] if isinstance(exec_mode, str) else exec_mode
         flags = (PF_DISCARD_DEAD if discard else 0) | (PF_PDL if pdl else 0) | (PF_FORCE_MINIMAL if force_minimal else 0)
-        pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew)
+        pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew, window)
         h = ctypes.c_void_p()
         _check(lib().ktiler_plan(self._h, cache_bytes, ctypes.byref(pol), ctypes.byref(h)))
         return Plan(h, self)

@@ -1,0 +1,211 @@
+"""CPU tests of the C ABI (no GPU): the library loads and exports every symbol declared in
+include/ktiler.h; the C++ planner equals the literal Alg. 2 oracle;
+analytic dependencies and memory lines equal the traced ones (P11); error paths."""
+import os
+import re
+
+import pytest
+
+from oracle import oracle as O
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def K():
+    import __graft_entry__ as ge
+    ge.build()
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler
+    ktiler.lib()
+    return ktiler
+
+
+def test_exports_every_header_symbol(K):
+    hdr = open(os.path.join(ROOT, "include", "ktiler.h")).read()
+    names = sorted(set(re.findall(r"^[a-z0-9_ ]+\**\s*(ktiler_[a-z_]+)\(", hdr, re.M)))
+    assert len(names) >= 18
+    lib = K.lib()
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(K.EXPORTS) <= set(names)
+    assert lib.ktiler_abi_version() == 1
+    assert lib.ktiler_status_str(3).decode() == "KTILER_E_UNTILEABLE"
+
+
+def _paper_pipe(bases):
+    from paper_conf_date_maghazeh0ep19_b200 import Motivational
+    return Motivational(device=None, bases=bases)
+
+
+@pytest.fixture(scope="module")
+def fig1():
+    g = O.motivational_graph()
+    return g, O.trace(g)
+
+
+def _blocks_by_sub(plan):
+    out = []
+    for sk in plan.subkernels():
+        blocks = []
+        for (x0, y0, z0, x1, y1, z1) in sk["rects"]:
+            blocks += [(x, y, z) for z in range(z0, z1) for y in range(y0, y1) for x in range(x0, x1)]
+        out.append((sk["node"], sorted(blocks), sk["fragment"]))
+    return out
+
+
+@pytest.mark.parametrize("lines", [36, 50, 68, 104, 136, 2175, 2176])
+def test_planner_equals_oracle_alg2_fig1(K, fig1, lines):
+    """P8/P9: the C++ planner reproduces the literal Alg. 2 schedule on the paper's example,
+    sub-kernel by sub-kernel (same blocks, same order, same fragments)."""
+    g, tr = fig1
+    m = _paper_pipe(g.bases())
+    plan = m.plan(lines * 128, kind="budget", exec_mode="stream")
+    ours = _blocks_by_sub(plan)
+    ref = O.cluster_tile(g, tr, lines * 128)
+    assert [(n, b, f) for n, b, f in ours] == [(n, sorted(b), f) for (n, b), f in zip(ref.seq, ref.frag)]
+
+
+def test_planner_untileable(K, fig1):
+    g, _ = fig1
+    m = _paper_pipe(g.bases())
+    with pytest.raises(K.KtilerError) as e:
+        m.plan(35 * 128, kind="budget", exec_mode="stream")
+    assert e.value.status == K.E_UNTILEABLE
+    # FORCE_MINIMAL commits the over-budget closures instead
+    p = m.plan(35 * 128, kind="budget", exec_mode="stream", force_minimal=True)
+    assert p.num_fragments() == 64
+
+
+def _pipe_pair(W, H, F, geo):
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    og = O.pipeline_graph(W, H, F, full_tile=geo["gray"][:2], half_tile=geo["down"][:2])
+    bases = og.bases()
+    p = Pipeline(W, H, F, device=None, geometry=geo, pitch_align=1, bases=bases)
+    return og, p
+
+
+SMALL = {"gray": (16, 8, 32), "blur": (16, 8, 32), "down": (8, 4, 32), "sobel": (8, 4, 32), "thresh": (8, 4, 32)}
+# tiles that leave ragged right and bottom tails (pitches must stay multiples of 16 B)
+RAGGED = {"gray": (64, 8, 32), "blur": (64, 8, 32), "down": (32, 4, 32), "sobel": (32, 4, 32), "thresh": (32, 4, 32)}
+GEOS = [(64, 96, 2, SMALL), (96, 38, 1, RAGGED), (32, 24, 3, SMALL), (160, 70, 1, RAGGED)]
+
+
+@pytest.mark.parametrize("W,H,F,geo", GEOS, ids=lambda v: str(v) if not isinstance(v, dict) else "")
+@pytest.mark.parametrize("budget", [6000, 9000, 20000, 1 << 30])
+def test_planner_equals_oracle_alg2_pipeline(K, W, H, F, geo, budget):
+    """P9: C++ planner == literal Alg. 2 on the 5-kernel chain (odd remainders included)."""
+    og, p = _pipe_pair(W, H, F, geo)
+    tr = O.trace(og)
+    ref = O.cluster_tile(og, tr, budget)
+    if ref.cost == O.INF:
+        with pytest.raises(K.KtilerError):
+            p.plan(budget, kind="budget", exec_mode="stream")
+        return
+    plan = p.plan(budget, kind="budget", exec_mode="stream")
+    ours = _blocks_by_sub(plan)
+    assert [(n, b, f) for n, b, f in ours] == [(n, sorted(b), f) for (n, b), f in zip(ref.seq, ref.frag)]
+    assert not O.validate_schedule(og, tr, [(n, b) for n, b, _ in ours], budget, [f for _, _, f in ours])
+
+
+@pytest.mark.parametrize("W,H,F,geo", GEOS[:2], ids=lambda v: str(v) if not isinstance(v, dict) else "")
+def test_analytic_deps_equal_traced(K, W, H, F, geo):
+    """P11: analytic (affine-footprint) dependencies == traced RAW dependencies (equality)
+    and analytic memory lines == traced lines, for every block of every kernel."""
+    og, p = _pipe_pair(W, H, F, geo)
+    tr = O.trace(og)
+    G = p.graph
+    for i in range(len(og.nodes)):
+        for b in og.blocks(i):
+            gid = og.gid(i, b)
+            want = sorted(og.block_of(q) for q in tr.deps[gid])
+            got = sorted((n, (bx, by, bz)) for n, bx, by, bz in G.block_deps(i, *b))
+            assert got == want, (i, b)
+            assert sorted(G.block_lines(i, *b)) == sorted(tr.lines[gid]), (i, b)
+
+
+def test_analytic_deps_paper_geometry(K, fig1):
+    g, tr = fig1
+    m = _paper_pipe(g.bases())
+    for i in range(2):
+        for b in g.blocks(i)[::7]:
+            gid = g.gid(i, b)
+            want = sorted(g.block_of(q) for q in tr.deps[gid])
+            got = sorted((n, (bx, by, bz)) for n, bx, by, bz in m.graph.block_deps(i, *b))
+            assert got == want
+            assert sorted(m.graph.block_lines(i, *b)) == sorted(tr.lines[gid])
+
+
+@pytest.mark.parametrize("kind,extra", [("rows", dict(rows=1)), ("rows", dict(rows=5)),
+                                        ("balanced", dict(l2_fraction=1.0)), ("none", {})])
+def test_policies_valid(K, kind, extra):
+    """Every policy yields a valid partition in dependency order (O-11)."""
+    og, p = _pipe_pair(64, 96, 2, SMALL)
+    tr = O.trace(og)
+    plan = p.plan(9000, kind=kind, exec_mode="stream", **extra)
+    ours = _blocks_by_sub(plan)
+    assert not O.validate_schedule(og, tr, [(n, b) for n, b, _ in ours])
+
+
+def test_plan_is_deterministic_and_content_free(K):
+    """T-R6: a plan depends on shapes only — planning twice gives the same
+    schedule (the planner never dereferences buffers)."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    a = Pipeline(7680, 4320, 4, device=None).plan(126 << 20, kind="budget", l2_fraction=0.5, exec_mode="graph")
+    b = Pipeline(7680, 4320, 4, device=None).plan(126 << 20, kind="budget", l2_fraction=0.5, exec_mode="graph")
+    sa, sb = a.subkernels(), b.subkernels()
+    assert [(s["node"], s["rects"]) for s in sa] == [(s["node"], s["rects"]) for s in sb]
+    st = a.stats()
+    assert st["n_fragments"] > 4 and st["max_footprint_bytes"] <= st["budget_bytes"]
+
+
+def test_error_paths(K):
+    g = K.Graph()
+    with pytest.raises(K.KtilerError) as e:
+        g.add_buffer(0x1000 + 4, 16, 16, 1)  # misaligned
+    assert e.value.status == K.E_INVALID
+    a = g.add_buffer(0x100000, 64, 64, 3)
+    with pytest.raises(K.KtilerError):
+        g.add_buffer(0x100000 + 128, 64, 64, 1)  # aliasing
+    b = g.add_buffer(0x200000, 64, 64, 1)
+    c = g.add_buffer(0x300000, 32, 32, 1)
+    acc = lambda buf, mode, ax, ay, h=0: dict(buf=buf, mode=mode, ax=ax, ay=ay, hl=h, hr=h, ht=h, hb=h)
+    # wrong declared footprint for a built-in -> rejected
+    with pytest.raises(K.KtilerError):
+        g.add_kernel(K.OP_BLUR5, (4, 4, 1), (64, 1, 1), [acc(b, K.READ, 16, 16, 1), acc(c, K.WRITE, 16, 16)])
+    n0 = g.add_kernel(K.OP_GRAY, (4, 8, 1), (64, 1, 1), [acc(a, K.READ, 16, 8), acc(b, K.WRITE, 16, 8)])
+    with pytest.raises(K.KtilerError):
+        g.add_edge(n0, n0, b)
+    with pytest.raises(K.KtilerError):  # grid does not cover the output
+        g.add_kernel(K.OP_DOWN2, (1, 1, 1), (64, 1, 1), [acc(b, K.READ, 32, 16), acc(c, K.WRITE, 16, 8)])
+    # odd-size down2 input
+    g2 = K.Graph()
+    x = g2.add_buffer(0x100000, 63, 64, 1, pitch_bytes=64)
+    y = g2.add_buffer(0x200000, 31, 32, 1, pitch_bytes=32)
+    with pytest.raises(K.KtilerError):
+        g2.add_kernel(K.OP_DOWN2, (2, 4, 1), (64, 1, 1), [acc(x, K.READ, 32, 16), acc(y, K.WRITE, 16, 8)])
+
+
+def test_cycle_detected(K):
+    """A graph that is not a DAG is rejected at plan time (KTILER_E_CYCLE)."""
+    g = K.Graph()
+    x = g.add_buffer(0x100000, 64, 64, 1)
+    y = g.add_buffer(0x200000, 64, 64, 1)
+    acc = lambda buf, mode: dict(buf=buf, mode=mode, ax=16, ay=16)
+    for src, dst in ((x, y), (y, x)):
+        g.add_kernel(K.OP_CUSTOM, (4, 4, 1), (64, 1, 1), [acc(src, K.READ), acc(dst, K.WRITE)],
+                     launch=lambda *a: None)
+    with pytest.raises(K.KtilerError) as e:
+        g.plan(1 << 20, kind="budget", exec_mode="stream")
+    assert e.value.status == K.E_CYCLE
+
+
+def test_plan_without_device_requires_cache_bytes(K):
+    """cache_bytes = 0 queries the device L2; with no device that must fail loudly."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("has a device")
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    p = Pipeline(256, 256, 1, device=None)
+    with pytest.raises(K.KtilerError) as e:
+        p.plan(0, kind="budget", exec_mode="graph")
+    assert e.value.status == K.E_CUDA

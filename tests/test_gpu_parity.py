@@ -93,6 +93,9 @@ MODES = [
     dict(exec_mode="persistent"),
     dict(exec_mode="persistent", skew=-1),
     dict(exec_mode="persistent", skew=3, persistent_ctas=7),
+    dict(exec_mode="dag"),
+    dict(exec_mode="dag", window=1),
+    dict(exec_mode="dag", window=4),
 ]
 POLICIES = [
     dict(kind="none"),
