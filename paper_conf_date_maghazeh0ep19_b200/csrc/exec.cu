@@ -46,8 +46,30 @@ struct DRect {  // whole 128-B lines: row r -> base + z*fs + y*pitch + lb0 + k*1
   int64_t pitch, fstride, lb0, lpr;
   int32_t y0, y1, z0, z1;
 };
+// Device-side trace ring (ktiler_trace_enable): NULL rec = tracing off.
+struct TraceBuf {
+  ktiler_trace_record* rec;
+  unsigned long long* n;
+  int64_t cap;
+};
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void trace_put(const TraceBuf& tb, uint64_t id, uint32_t kind, uint64_t t0, uint64_t t1) {
+  const unsigned long long k = atomicAdd(tb.n, 1ull);
+  if ((int64_t)k < tb.cap) {
+    uint32_t sm;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    tb.rec[k] = ktiler_trace_record{id, sm, kind, t0, t1};
+  }
+}
+
 struct KParams {
   CUtensorMap tmap;     // input tile map (tensor TMA), valid if use_tmap
+  TraceBuf tb;
+  int64_t lid;          // launch index (trace id)
   uint32_t box_bytes;   // bytes one tensor-TMA box delivers
   int32_t use_tmap;
   DBuf in, out;
@@ -59,7 +81,46 @@ struct KParams {
   int64_t rpre[MAXR + 1];
   DRect d[MAXD];
   int64_t dpre[MAXD + 1];
+  // GRAPH_CHAIN: per-block epoch flags and launch completion (see chain_* below)
+  int32_t chain;           // 1: flag-synchronised PDL chain
+  int32_t gx, gy;          // this node's grid (block linear index -> flag)
+  int32_t pgx, pgy;        // producer node's grid (0: graph input, nothing to wait on)
+  int32_t rax, ray, rox, roy, rhl, rhr, rht, rhb;  // read footprint (affine map)
+  int32_t wax, way;        // producer write footprint
+  unsigned int* flags;     // this node's block flags
+  const unsigned int* pflags;  // producer node's block flags
+  const unsigned int* epoch;   // current execute's epoch
+  unsigned int* dcount;    // this launch's finished-CTA counter
+  unsigned int* prefix;    // prefix[l] == epoch <=> launches 0..l all finished (this one at [0])
+  const unsigned int* disc_prefix;  // discards may run once *disc_prefix == epoch
 };
+
+__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// GRAPH_CHAIN, one warp: wait until every producer block of output block (bx, by, bz)
+// has published this epoch.  Producer range = closed form of the affine footprints
+// (SURVEY §8(a) a3), the same one the planner uses.
+__device__ __forceinline__ void chain_wait(const KParams& p, int bx, int by, int bz, unsigned epoch, int lane) {
+  if (p.pgx == 0) return;
+  const int rx0 = max(0, p.rax * bx + p.rox - p.rhl), rx1 = min((int)p.in.W, p.rax * (bx + 1) + p.rox + p.rhr);
+  const int ry0 = max(0, p.ray * by + p.roy - p.rht), ry1 = min((int)p.in.H, p.ray * (by + 1) + p.roy + p.rhb);
+  const int px0 = rx0 / p.wax, px1 = min(p.pgx, (rx1 + p.wax - 1) / p.wax);
+  const int py0 = ry0 / p.way, py1 = min(p.pgy, (ry1 + p.way - 1) / p.way);
+  const int pw = px1 - px0, n = pw * (py1 - py0);
+  for (int i = lane; i < n; i += 32) {
+    const int dy = i / pw;
+    const unsigned int* f = p.pflags + ((int64_t)bz * p.pgy + py0 + dy) * p.pgx + px0 + (i - dy * pw);
+    while (ld_acquire(f) != epoch) __nanosleep(64);
+  }
+  __syncwarp();
+}
 
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
@@ -96,79 +157,177 @@ __device__ __forceinline__ ktd::Tile launch_tile(const KParams& p, int64_t lin64
   t.x1 = min(t.x0 + p.tw, p.out.W);
   t.y1 = min(t.y0 + p.th, p.out.H);
   t.fw = p.tw;
-  t.pad = 0;
+  t.pad = (int)(((unsigned)bz * (unsigned)p.gy + (unsigned)by) * (unsigned)p.gx + (unsigned)bx);  // block index
   return t;
+}
+
+// GRAPH_CHAIN: publish output block t.pad of this node, after a CTA barrier.  bar.sync
+// orders every thread's tile writes before this thread's gpu-scope release (PTX memory
+// model: release is cumulative over writes that precede it in causality order), so the
+// consumer's acquire of the flag sees the whole tile — no separate fence.
+__device__ __forceinline__ void chain_publish(const KParams& p, const ktd::Tile& t, unsigned epoch) {
+  st_release(p.flags + t.pad, epoch);
+}
+
+// GRAPH_CHAIN end of CTA (thread 0): count it; the last CTA of the launch waits for the
+// previous launches (prefix[-1]) and publishes prefix[0] — "launches 0..this all done".
+__device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, bool first_launch) {
+  // relaxed: the count only says "this CTA's reads are consumed" (they were, before the
+  // barrier); data visibility travels through the block flags
+  const unsigned old = atomicAdd(p.dcount, 1u);
+  if (old == gridDim.x - 1) {
+    *p.dcount = 0;  // ready for the next execute (every CTA of this launch has counted)
+    if (!first_launch)
+      while (ld_acquire(p.prefix - 1) != epoch) __nanosleep(128);
+    __threadfence();
+    st_release(p.prefix, epoch);
+  }
 }
 
 template <int OP, bool SCALAR>
 __global__ void __launch_bounds__(256, (OP == 1 || OP == 3) ? 3 : 4) op_kernel(const __grid_constant__ KParams p) {
-  if (p.pdl) pdl_wait();
-  if (p.ndisc) do_discards(p);
-  if (p.pdl) pdl_launch();
-  const int64_t ntiles = p.rpre[p.nrect];
+  __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
+  __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
-  if (SCALAR) {
-    for (int64_t i = blockIdx.x; i < ntiles; i += gridDim.x) ktd::scalar_tile(OP, p.in, p.out, launch_tile(p, i), p.T, nt, tid);
-    return;
-  }
-  // Grid-stride over the launch's tiles with two shared buffers: the TMA bulk copies of
-  // tile i+2 stream in while tile i+1 computes.
-  extern __shared__ __align__(128) uint8_t ktsm[];
-  __shared__ __align__(8) uint64_t mbar[2];
-  __shared__ ktd::Tile s_tile[2];  // decoded once by warp 0, read by all after the mbarrier
   if (tid == 0) {
-    ktd::mbar_init(&mbar[0], 1);
-    ktd::mbar_init(&mbar[1], 1);
-    ktd::fence_proxy_async();
+    if (p.tb.rec) s_t0 = gtimer();
+    if (p.chain) s_epoch = *(volatile const unsigned int*)p.epoch;
   }
-  __syncthreads();
-  const int64_t i0 = blockIdx.x;
-  if (i0 >= ntiles) return;  // discard-only CTAs
-  auto issue = [&](int64_t i, int slot) {  // warp 0
-    const ktd::Tile t = launch_tile(p, i);
-    uint8_t* dst = ktsm + (slot ? p.stage_bytes : 0);
-    if (p.use_tmap) {
-      if (tid == 0) {
-        s_tile[slot] = t;
-        ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot]);
+  if (p.chain) {
+    pdl_launch();  // the next sub-kernel may become resident now: it waits on tile flags
+  } else {
+    if (p.pdl) pdl_wait();
+    if (p.ndisc) do_discards(p);
+    if (p.pdl) pdl_launch();
+  }
+  const int64_t ntiles = p.rpre[p.nrect];
+  if (SCALAR) {
+    __syncthreads();
+    const unsigned epoch = s_epoch;
+    for (int64_t i = blockIdx.x; i < ntiles; i += gridDim.x) {
+      const ktd::Tile t = launch_tile(p, i);
+      if (p.chain) {
+        if (tid < 32) chain_wait(p, (int)(t.x0 / p.tw), (int)(t.y0 / p.th), (int)t.z, epoch, tid);
+        __syncthreads();
       }
-    } else {
-      if (tid == 0) s_tile[slot] = t;
-      ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
+      ktd::scalar_tile(OP, p.in, p.out, t, p.T, nt, tid);
+      if (p.chain) {
+        __syncthreads();
+        if (tid == 0) chain_publish(p, t, epoch);
+      }
     }
-  };
-  if (tid < 32) {
-    issue(i0, 0);
-    if (i0 + gridDim.x < ntiles) issue(i0 + gridDim.x, 1);
-  }
-  unsigned ph = 0;
-  int b = 0;
-  for (int64_t i = i0; i < ntiles; i += gridDim.x, b ^= 1) {
-    uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
-    ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
-    ph ^= 1u << b;
-    const ktd::Tile t = s_tile[b];
-    if ((OP == 1 || OP == 3) && ktd::needs_fix(OP, p.in, t)) {
-      ktd::stage_fix(OP, p.in, t, buf, nt, tid);
-      __syncthreads();
+  } else {
+    // Grid-stride over the launch's tiles with two shared buffers: the TMA bulk copies of
+    // tile i+2 stream in while tile i+1 computes.
+    extern __shared__ __align__(128) uint8_t ktsm[];
+    __shared__ __align__(8) uint64_t mbar[2];
+    __shared__ ktd::Tile s_tile[2];  // decoded once by warp 0, read by all after the mbarrier
+    __shared__ uint64_t s_tw[2];     // trace (chain): producers ready
+    if (tid == 0) {
+      ktd::mbar_init(&mbar[0], 1);
+      ktd::mbar_init(&mbar[1], 1);
+      ktd::fence_proxy_async();
     }
-    ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid);
-    const int64_t nx = i + 2 * (int64_t)gridDim.x;
-    if (nx < ntiles) {
-      __syncthreads();  // buffer b consumed
-      if (tid < 32) {
+    __syncthreads();
+    const unsigned epoch = s_epoch;
+    const int64_t i0 = blockIdx.x;
+    auto issue = [&](int64_t i, int slot) {  // warp 0
+      const ktd::Tile t = launch_tile(p, i);
+      if (p.chain) {  // producers' tiles complete (acquire), then hand them to the async proxy
+        chain_wait(p, (int)(t.x0 / p.tw), (int)(t.y0 / p.th), (int)t.z, epoch, tid);
+        ktd::fence_proxy_async();
+        if (p.tb.rec && tid == 0) s_tw[slot] = gtimer();
+      }
+      uint8_t* dst = ktsm + (slot ? p.stage_bytes : 0);
+      if (p.use_tmap) {
+        if (tid == 0) {
+          s_tile[slot] = t;
+          ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot]);
+        }
+      } else {
+        if (tid == 0) s_tile[slot] = t;
+        ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
+      }
+    };
+    if (i0 < ntiles && tid < 32) {
+      issue(i0, 0);
+      if (i0 + gridDim.x < ntiles) issue(i0 + gridDim.x, 1);
+    }
+    unsigned ph = 0;
+    int b = 0;
+    for (int64_t i = i0; i < ntiles; i += gridDim.x, b ^= 1) {
+      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+      ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
+      ph ^= 1u << b;
+      const ktd::Tile t = s_tile[b];
+      if ((OP == 1 || OP == 3) && ktd::needs_fix(OP, p.in, t)) {
+        ktd::stage_fix(OP, p.in, t, buf, nt, tid);
+        __syncthreads();
+      }
+      ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid);
+      const int64_t nx = i + 2 * (int64_t)gridDim.x;
+      if (p.chain) {
+        __syncthreads();  // tile written (and buffer b consumed)
+        if (tid == 0) {
+          const uint64_t tc = p.tb.rec ? gtimer() : 0;
+          chain_publish(p, t, epoch);
+          if (p.tb.rec) {
+            trace_put(p.tb, p.lid, 3, s_tw[b], tc);  // producers ready -> tile computed
+            trace_put(p.tb, p.lid, 4, tc, gtimer());  // publish (fence + release)
+          }
+        }
+      } else if (nx < ntiles) {
+        __syncthreads();  // buffer b consumed
+      }
+      if (nx < ntiles && tid < 32) {
         ktd::fence_proxy_async();
         issue(nx, b);
       }
     }
   }
+  if (p.chain) {
+    __syncthreads();
+    if (tid == 0) chain_finish(p, s_epoch, p.chain == 2);
+    if (p.ndisc) {  // lines dead after an earlier launch: wait until it and all before it finished
+      if (tid == 0)
+        while (ld_acquire(p.disc_prefix) != s_epoch) __nanosleep(128);
+      __syncthreads();
+      do_discards(p);
+    }
+  }
+  if (p.tb.rec) {
+    __syncthreads();
+    if (tid == 0) trace_put(p.tb, p.lid, 0, s_t0, gtimer());
+  }
 }
 
+// GRAPH_CHAIN tail (launched without PDL): wait until every launch of the chain finished
+// (prefix of the last one), then retire the remaining dead lines.  The epoch is advanced by
+// chain_epoch_kernel, stream-ordered after this one (a CTA of this kernel may start late
+// and must still read the current epoch).
+__global__ void chain_tail_kernel(const __grid_constant__ KParams p) {
+  __shared__ unsigned int s_ep;
+  if (threadIdx.x == 0) {
+    s_ep = *(volatile const unsigned int*)p.epoch;
+    while (ld_acquire(p.disc_prefix) != s_ep) __nanosleep(256);
+  }
+  __syncthreads();
+  if (p.ndisc) do_discards(p);
+}
+
+// GRAPH_CHAIN: advance the epoch (one thread), stream-ordered after the tail kernel.
+__global__ void chain_epoch_kernel(unsigned int* epoch) { *epoch += 1u; }
+
 __global__ void discard_kernel(const __grid_constant__ KParams p) {
+  const uint64_t tt0 = p.tb.rec ? gtimer() : 0;
   if (p.pdl) pdl_wait();
   do_discards(p);
   if (p.pdl) pdl_launch();
+  if (p.tb.rec) {
+    __syncthreads();
+    if (threadIdx.x == 0) trace_put(p.tb, p.lid, 0, tt0, gtimer());
+  }
 }
 
 // ------------------------------------------------------------------------------------
@@ -209,16 +368,9 @@ struct PParams {
   unsigned int* rc;
   PCtrl* ctrl;
   int64_t stage_bytes;  // one staging buffer (the kernel double-buffers)
+  TraceBuf tb;
 };
 
-__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
-  unsigned int v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
 
 // Producer blocks i in [0, n) with [a*i, a*(i+1)) meeting [lo, hi) (write footprints have no
 // offsets or halos for built-ins).  32-bit: pixel coordinates are < 2^31.
@@ -357,6 +509,7 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
   __shared__ uint64_t s_desc[2];
   __shared__ TInfo s_ti[2];  // decoded tile of each buffer (control warp -> compute warps)
   __shared__ unsigned int s_epoch;
+  __shared__ uint64_t s_tc0, s_tq0;  // trace timestamps (kept out of registers)
   extern __shared__ __align__(128) uint8_t ktsm[];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
@@ -415,6 +568,7 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
         }
         break;
       }
+      if (p.tb.rec && lane == 0) s_tq0 = gtimer();
       int ch = -1;
       if (ctl_probe(p, decode(p, w0), epoch, lane)) ch = 0;
       else if (nw > 1 && ctl_probe(p, decode(p, w1), epoch, lane)) ch = 1;
@@ -450,6 +604,7 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
           ktd::stage_issue(a.nd->op, a.nd->in, a.t, buf, &s_full[b], lane);
         }
       }
+      if (p.tb.rec && lane == 0) trace_put(p.tb, d, 1, s_tq0, gtimer());
       // swap roles for the next iteration (which stages into b ^ 1)
       d_this = d_other;
       u_this = u_other;
@@ -468,6 +623,7 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
       ktd::mbar_wait(&s_full[b], (ph >> b) & 1u);
       ph ^= 1u << b;
       if (s_desc[b] == DESC_STOP) break;
+      if (p.tb.rec && tid == 0) s_tc0 = gtimer();
       const TInfo a = s_ti[b];
       const PNode& nd = *a.nd;
       uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
@@ -480,6 +636,7 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
         }
         ktd::compute_tile(nd.op, nd.out, a.t, buf, nd.T, PCOMP_THREADS, tid);
       }
+      if (p.tb.rec && tid == 0) trace_put(p.tb, s_desc[b], 2, s_tc0, gtimer());
       nbar_arrive(1 + b, PERSIST_THREADS);
     }
   }
@@ -554,10 +711,18 @@ struct ktiler_plan_s {
   void (*pfn)(PParams) = nullptr;
   int64_t skew = 0;
   bool has_custom = false;
+  TraceBuf tb{nullptr, nullptr, 0};
+  bool executed = false;
+  // GRAPH_CHAIN state: one device block (epoch | flags | dcount | prefix) and the tail
+  void* cmem = nullptr;
+  unsigned int* epoch = nullptr;
+  std::vector<Launch> chain_tail;
   ~ktiler_plan_s() {
     if (exec) cudaGraphExecDestroy(exec);
     if (graph) cudaGraphDestroy(graph);
     if (dmem) cudaFree(dmem);
+    if (tb.rec) cudaFree(tb.rec);
+    if (cmem) cudaFree(cmem);
   }
 };
 
@@ -588,7 +753,9 @@ void build_launches(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
   const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
-  const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG;
+  // GRAPH_DAG and GRAPH_CHAIN keep each sub-kernel's discard list apart (dag_disc, sub =
+  // the list's sub-kernel): DAG makes them graph nodes, CHAIN attaches them to later launches
+  const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN;
   std::vector<DRect> pending;
   auto flush_disc_only = [&](size_t keep) {
     while (pending.size() > keep) {
@@ -742,8 +909,11 @@ kfn_t launch_fn(const Launch& L) {
 // Dynamic-smem attribute + grid of one launch: the vector kernels grid-stride over their
 // tiles with as many CTAs as fit the device at once.
 ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_out) {
-  if (L.resident == 0 && L.smem > 32 * 1024) {  // static + dynamic may pass the 48 KB default
-    cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, L.smem);
+  // static + dynamic may pass the 48 KB default; the attribute is per function, so it is
+  // always set to the two-buffer maximum (a one-buffer launch of the same kernel uses less)
+  const int smem_max = std::max(L.smem, (int)(2 * L.kp.stage_bytes));
+  if (L.resident == 0 && smem_max > 32 * 1024) {
+    cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
   }
   if (L.resident == 0) {
@@ -756,12 +926,20 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
   // grid-stride CTAs (x tiles_per_cta) in stream/graph modes; in GRAPH_DAG one CTA per
   // tile by default, so concurrent sub-kernels interleave at tile granularity
   static const int tpc_env = getenv("KTILER_TILES_PER_CTA") ? atoi(getenv("KTILER_TILES_PER_CTA")) : -1;
-  const int tpc = tpc_env >= 0 ? tpc_env : (P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG ? 1 : 0);
+  const bool chain = P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN;
+  const int tpc = tpc_env >= 0 ? tpc_env : ((P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || chain) ? 1 : 0);
   if (L.node >= 0 && !L.n->scalar) {
     if (tpc > 0) grid = (grid + tpc - 1) / tpc;
     else grid = std::min<int64_t>(grid, L.resident);
   }
-  if (L.kp.ndisc) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+  if (L.node >= 0 && !L.n->scalar && grid >= L.blocks && L.smem != (int)L.kp.stage_bytes) {
+    // one tile per CTA: the second staging buffer is never used -> more resident CTAs
+    L.smem = (int)L.kp.stage_bytes;
+    L.resident = 0;
+    return prep_launch(P, L, fn, grid_out);
+  }
+  // (GRAPH_CHAIN: the launch's own CTAs share its discards; extra CTAs would only spin)
+  if (L.kp.ndisc && !chain) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
   *grid_out = grid;
   return KTILER_OK;
 }
@@ -856,7 +1034,7 @@ ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
     cfg.stream = st;
     cudaLaunchAttribute attr[2];
     int na = 0;
-    if (L.kp.pdl) {
+    if (L.kp.pdl || L.kp.chain == 1) {
       attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
       attr[na].val.programmaticStreamSerializationAllowed = 1;
       ++na;
@@ -883,6 +1061,103 @@ ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
     cudaError_t e = cudaLaunchKernelEx(&cfg, fn, L.kp);
     if (e != cudaSuccess) return cuda_fail(e, "sub-kernel launch");
   }
+  if (P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN) {
+    for (auto& T : P->chain_tail) {
+      const int64_t lines = T.kp.ndisc ? T.kp.dpre[T.kp.ndisc] : 0;
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(1184, (lines + 255) / 256));
+      chain_tail_kernel<<<grid, 256, 0, st>>>(T.kp);
+    }
+    chain_epoch_kernel<<<1, 1, 0, st>>>(P->epoch);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "chain tail launch");
+  }
+  return KTILER_OK;
+}
+
+// GRAPH_CHAIN setup (first execute): device flags/counters, per-launch producer maps, and
+// placement of each discard list on a later launch that first waits for the prefix flag of
+// the list's last reader launch (lines are only dropped once nobody can still read them).
+ktiler_status setup_chain(ktiler_plan_s* P) {
+  const kt::Graph& g = P->g;
+  const int nn = (int)g.nodes.size();
+  if (P->has_custom) return fail(KTILER_E_UNSUPPORTED, "GRAPH_CHAIN runs built-in ops only");
+  std::vector<int64_t> flag0(nn);
+  int64_t nflags = 0;
+  for (int v = 0; v < nn; ++v) {
+    flag0[v] = nflags;
+    nflags += g.nodes[v].nblocks;
+  }
+  const int64_t nl = (int64_t)P->launches.size();
+  const size_t bytes = (size_t)(1 + nflags + 2 * nl + 64) * 4;
+  char* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, bytes);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (chain flags)");
+  P->cmem = d;
+  if ((e = cudaMemset(d, 0, bytes)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
+  unsigned int* u = (unsigned int*)d;
+  const unsigned int one = 1;
+  if ((e = cudaMemcpy(u, &one, 4, cudaMemcpyHostToDevice)) != cudaSuccess) return cuda_fail(e, "cudaMemcpy");
+  P->epoch = u;
+  unsigned int* flags = u + 1;
+  unsigned int* dcount = flags + nflags;
+  unsigned int* prefix = dcount + nl;
+  std::vector<int64_t> last_launch_of_sub(P->s.subs.size(), -1);
+  for (int64_t l = 0; l < nl; ++l) {
+    Launch& L = P->launches[l];
+    const kt::Node& n = g.nodes[L.node];
+    const kt::Access& r = n.acc[n.racc];
+    KParams& k = L.kp;
+    k.chain = l == 0 ? 2 : 1;
+    k.pdl = 0;
+    k.gx = (int32_t)n.gx();
+    k.gy = (int32_t)n.gy();
+    k.flags = flags + flag0[L.node];
+    k.epoch = P->epoch;
+    k.dcount = dcount + l;
+    k.prefix = prefix + l;
+    k.pgx = 0;
+    for (auto& c : g.in_ch[L.node]) {
+      const kt::Node& pu = g.nodes[c.u];
+      const kt::Access& uw = pu.acc[c.w];
+      k.pgx = (int32_t)pu.gx();
+      k.pgy = (int32_t)pu.gy();
+      k.pflags = flags + flag0[c.u];
+      k.rax = (int32_t)r.ax; k.ray = (int32_t)r.ay; k.rox = (int32_t)r.ox; k.roy = (int32_t)r.oy;
+      k.rhl = r.hl; k.rhr = r.hr; k.rht = r.ht; k.rhb = r.hb;
+      k.wax = (int32_t)uw.ax; k.way = (int32_t)uw.ay;
+    }
+    last_launch_of_sub[L.sub] = l;
+  }
+  // discard lists: list D (dead after sub-kernel D.sub) goes to the first launch of a
+  // sub-kernel >= D.sub + 2 without discards of its own, else to the tail
+  int64_t next = 0;
+  for (auto& D : P->dag_disc) {
+    const int64_t wait_l = last_launch_of_sub[D.sub];
+    while (next < nl && (P->launches[next].sub < D.sub + 2 || P->launches[next].kp.ndisc)) ++next;
+    KParams* k = nullptr;
+    if (next < nl) {
+      k = &P->launches[next].kp;
+    } else {
+      Launch T;
+      std::memset(&T.kp, 0, sizeof(T.kp));
+      P->chain_tail.push_back(T);
+      k = &P->chain_tail.back().kp;
+    }
+    k->ndisc = D.kp.ndisc;
+    std::memcpy(k->d, D.kp.d, sizeof(k->d));
+    std::memcpy(k->dpre, D.kp.dpre, sizeof(k->dpre));
+    k->disc_prefix = prefix + wait_l;
+  }
+  if (P->chain_tail.empty()) {
+    Launch T;
+    std::memset(&T.kp, 0, sizeof(T.kp));
+    P->chain_tail.push_back(T);
+  }
+  for (auto& T : P->chain_tail) {
+    T.kp.epoch = P->epoch;
+    T.kp.disc_prefix = prefix + (nl - 1);  // the tail waits for the whole chain
+  }
+  P->dag_disc.clear();
   return KTILER_OK;
 }
 
@@ -1053,7 +1328,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
   kt::Graph* G = kt::graph_of(gh);
   ktiler_status s = G->finalize();
   if (s) return s;
-  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_DAG)
+  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_CHAIN)
     return fail(KTILER_E_INVALID, "unknown exec_mode");
   if (cache_bytes == 0) {
     int dev = 0, l2 = 0;
@@ -1124,7 +1399,10 @@ ktiler_status ktiler_plan_get_stats(ktiler_plan_t p, ktiler_plan_stats* out) {
   std::memset(out, 0, sizeof(*out));
   out->n_subkernels = (int64_t)p->s.subs.size();
   out->n_fragments = p->s.nfrag;
-  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT ? 1 : (int64_t)(p->launches.size() + p->dag_disc.size());
+  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT
+                        ? 1
+                        : (int64_t)(p->launches.size() + p->dag_disc.size()) +
+                              (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN ? 2 : 0);
   out->n_discard_lines = (p->pol.flags & KTILER_PF_DISCARD_DEAD) ? p->s.discard_lines : 0;
   out->budget_bytes = p->s.budget;
   out->max_footprint_bytes = p->s.max_footprint;
@@ -1147,12 +1425,27 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     if (p->pol.exec_mode == KTILER_EXEC_PERSISTENT) {
       ktiler_status s = setup_persistent(p);
       if (s) return s;
+      p->pp.tb = p->tb;
     } else {
       for (auto& L : p->launches)
         if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar)
           L.kp.use_tmap = make_tmap(p->g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
+      if (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN) {
+        ktiler_status s = setup_chain(p);
+        if (s) return s;
+      }
+      int64_t lid = 0;
+      for (auto& L : p->launches) {
+        L.kp.tb = p->tb;
+        L.kp.lid = lid++;
+      }
+      for (auto& L : p->dag_disc) {
+        L.kp.tb = p->tb;
+        L.kp.lid = lid++;
+      }
     }
   }
+  p->executed = true;
   switch (p->pol.exec_mode) {
     case KTILER_EXEC_STREAM: {
       ktiler_status s = enqueue(p, st);
@@ -1172,6 +1465,7 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
       break;
     }
     case KTILER_EXEC_GRAPH:
+    case KTILER_EXEC_GRAPH_CHAIN:
     case KTILER_EXEC_GRAPH_PERSIST_L2: {
       if (!p->exec) {
         cudaStream_t cs;
@@ -1239,6 +1533,50 @@ ktiler_status ktiler_execute_host(ktiler_plan_t p, const ktiler_host_copy* in, i
     s = copy(outc[i], false);
     if (s) return s;
   }
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_trace_enable(ktiler_plan_t p, int64_t capacity) {
+  if (!p || capacity <= 0) return fail(KTILER_E_INVALID, "NULL plan or capacity <= 0");
+  if (p->executed || p->tb.rec) return fail(KTILER_E_STATE, "ktiler_trace_enable must precede the first execute");
+  void* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, (size_t)capacity * sizeof(ktiler_trace_record) + 256);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (trace)");
+  if ((e = cudaMemset(d, 0, (size_t)capacity * sizeof(ktiler_trace_record) + 256)) != cudaSuccess)
+    return cuda_fail(e, "cudaMemset (trace)");
+  p->tb.rec = (ktiler_trace_record*)d;
+  p->tb.n = (unsigned long long*)((char*)d + (size_t)capacity * sizeof(ktiler_trace_record));
+  p->tb.cap = capacity;
+  kt::clear_error();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_trace_read(ktiler_plan_t p, ktiler_trace_record* out, int64_t cap, int64_t* n) {
+  if (!p || !n) return fail(KTILER_E_INVALID, "NULL argument");
+  if (!p->tb.rec) return fail(KTILER_E_STATE, "tracing not enabled");
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceSynchronize");
+  unsigned long long cnt = 0;
+  if ((e = cudaMemcpy(&cnt, p->tb.n, sizeof(cnt), cudaMemcpyDeviceToHost)) != cudaSuccess) return cuda_fail(e, "cudaMemcpy");
+  *n = (int64_t)cnt;
+  if (out && cap > 0) {
+    int64_t k = std::min<int64_t>({cap, (int64_t)cnt, p->tb.cap});
+    if (k > 0 && (e = cudaMemcpy(out, p->tb.rec, (size_t)k * sizeof(ktiler_trace_record), cudaMemcpyDeviceToHost)) != cudaSuccess)
+      return cuda_fail(e, "cudaMemcpy");
+    if ((e = cudaMemset(p->tb.n, 0, sizeof(cnt))) != cudaSuccess) return cuda_fail(e, "cudaMemset");
+  }
+  kt::clear_error();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_get_launch(ktiler_plan_t p, int64_t i, int32_t* sub, int32_t* node, int64_t* tiles) {
+  if (!p) return fail(KTILER_E_INVALID, "NULL plan");
+  const int64_t nl = (int64_t)p->launches.size(), nd = (int64_t)p->dag_disc.size();
+  if (i < 0 || i >= nl + nd) return fail(KTILER_E_INVALID, "launch index out of range");
+  const Launch& L = i < nl ? p->launches[i] : p->dag_disc[i - nl];
+  if (sub) *sub = L.node >= 0 ? L.sub : -1;
+  if (node) *node = L.node;
+  if (tiles) *tiles = L.node >= 0 ? L.blocks : 0;
   return KTILER_OK;
 }
 

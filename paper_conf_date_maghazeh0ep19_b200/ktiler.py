@@ -19,11 +19,11 @@ BUF_INTERNAL = 1
 READ, WRITE = 1, 2
 OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM = range(6)
 FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE = range(4)
-EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG = range(5)
+EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN = range(6)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL = 1, 2, 4
 
 EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
-              "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG}
+              "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG, "chain": EXEC_GRAPH_CHAIN}
 FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE}
 
 
@@ -72,6 +72,11 @@ class PlanStats(ctypes.Structure):
                 ("pad", ctypes.c_int32)]
 
 
+class TraceRecord(ctypes.Structure):
+    _fields_ = [("id", ctypes.c_uint64), ("smid", ctypes.c_uint32), ("kind", ctypes.c_uint32),
+                ("t0_ns", ctypes.c_uint64), ("t1_ns", ctypes.c_uint64)]
+
+
 class HostCopy(ctypes.Structure):
     _fields_ = [("buf_id", ctypes.c_int32), ("pad", ctypes.c_int32), ("host", ctypes.c_void_p),
                 ("frame0", ctypes.c_int64), ("frames", ctypes.c_int64)]
@@ -81,7 +86,8 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_graph_destroy", "ktiler_add_buffer", "ktiler_add_kernel", "ktiler_add_edge",
            "ktiler_graph_block_deps", "ktiler_graph_block_lines", "ktiler_plan", "ktiler_plan_destroy",
            "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
-           "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host"]
+           "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
+           "ktiler_trace_read", "ktiler_plan_get_launch"]
 
 _LIB = None
 
@@ -115,6 +121,9 @@ def lib() -> ctypes.CDLL:
         "ktiler_plan_get_stats": ([vp, P(PlanStats)], st),
         "ktiler_execute": ([vp, vp], st),
         "ktiler_execute_host": ([vp, P(HostCopy), i32, P(HostCopy), i32, vp], st),
+        "ktiler_trace_enable": ([vp, i64], st),
+        "ktiler_trace_read": ([vp, vp, i64, P(i64)], st),
+        "ktiler_plan_get_launch": ([vp, i64, P(i32), P(i32), P(i64)], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -257,6 +266,34 @@ class Plan:
         s = PlanStats()
         _check(lib().ktiler_plan_get_stats(self._h, ctypes.byref(s)))
         return {f: getattr(s, f) for f, _ in PlanStats._fields_ if f != "pad"}
+
+    def trace_enable(self, capacity: int = 1 << 20) -> None:
+        """Device-side timeline records (include/ktiler.h, ktiler_trace_enable); call before
+        the first execute."""
+        _check(lib().ktiler_trace_enable(self._h, capacity))
+        self._trace_cap = capacity
+
+    def trace_read(self):
+        """numpy structured array of the records written since the last read (synchronizes)."""
+        import numpy as np
+        n = ctypes.c_int64()
+        cap = self._trace_cap
+        buf = (TraceRecord * cap)()
+        _check(lib().ktiler_trace_read(self._h, ctypes.cast(buf, ctypes.c_void_p), cap, ctypes.byref(n)))
+        dt = np.dtype([("id", "<u8"), ("smid", "<u4"), ("kind", "<u4"), ("t0", "<u8"), ("t1", "<u8")])
+        k = min(n.value, cap)
+        return np.frombuffer(bytes(buf)[:k * dt.itemsize], dtype=dt).copy(), n.value
+
+    def launches(self):
+        """[(sub, node, tiles)] of the plan's launch list (trace ids index it)."""
+        out, i = [], 0
+        while True:
+            sub, node, tiles = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int64()
+            if lib().ktiler_plan_get_launch(self._h, i, ctypes.byref(sub), ctypes.byref(node), ctypes.byref(tiles)):
+                break
+            out.append((sub.value, node.value, tiles.value))
+            i += 1
+        return out
 
     def execute(self, stream: int = 0) -> None:
         _check(lib().ktiler_execute(self._h, ctypes.c_void_p(stream)))

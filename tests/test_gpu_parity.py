@@ -96,6 +96,7 @@ MODES = [
     dict(exec_mode="dag"),
     dict(exec_mode="dag", window=1),
     dict(exec_mode="dag", window=4),
+    dict(exec_mode="chain"),
 ]
 POLICIES = [
     dict(kind="none"),
@@ -124,7 +125,7 @@ def test_modes_policies(mode, pol, discard):
         assert _eq(out[k], ref[k]), k
 
 
-@pytest.mark.parametrize("mode", ["graph", "persistent"])
+@pytest.mark.parametrize("mode", ["graph", "persistent", "chain"])
 def test_b200_geometry_tiled(mode):
     """The bench geometry itself, tiled into several fragments (budget just above one closure)."""
     W, H, F = 2048, 1024, 2
@@ -140,7 +141,7 @@ def test_replay_is_idempotent():
     """A plan executes many times (GRAPH replays, persistent epochs) with identical output."""
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
     W, H, F = 1024, 128, 1
-    for mode in ("graph", "persistent"):
+    for mode in ("graph", "persistent", "chain"):
         p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
         a = synth.uniform(1, W, H, F)
         b = synth.scene(2, W, H, F)
@@ -224,3 +225,29 @@ def test_gpu_generator_matches_numpy():
         G.fill(kind, 11, s.data_ptr(), W * 3, 20 * W * 3, W, H, y0=17, rows=20, f0=1, F=1)
         torch.cuda.synchronize()
         assert np.array_equal(s.cpu().numpy()[0], synth.make(kind, 11, W, H, F)[1, 17:37])
+
+
+@pytest.mark.parametrize("mode", ["graph", "chain", "persistent"])
+def test_trace_records(mode):
+    """ktiler_trace_*: one record per CTA (launch modes) or two per tile (persistent), with
+    ordered timestamps; tracing does not change the result."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 1024, 256, 2
+    rgb = synth.scene(21, W, H, F)
+    p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
+    p.view("rgb").copy_(torch.from_numpy(rgb))
+    plan = p.plan(100 * 1024, kind="budget", exec_mode=mode, discard=True)
+    plan.trace_enable(1 << 16)
+    p.run()
+    rec, n = plan.trace_read()
+    assert n == len(rec) > 0
+    assert (rec["t1"] >= rec["t0"]).all()
+    if mode == "persistent":
+        tiles = sum(s["n_blocks"] for s in plan.subkernels())
+        assert (rec["kind"] == 2).sum() == tiles and (rec["kind"] == 1).sum() == tiles
+    else:
+        assert set(rec["kind"].tolist()) == ({0, 3, 4} if mode == "chain" else {0})
+        assert set(rec["id"].tolist()) <= set(range(len(plan.launches())))
+    assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(rgb, T=40.0)["mask"])
+    with pytest.raises(Exception):
+        plan.trace_enable(16)  # after the first execute
