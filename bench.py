@@ -1,20 +1,31 @@
-"""bench.py — Mpix/s of the tiled kernel graph on B200 (BASELINE.json metric).
+"""bench.py — Mpix/s of the KTILER-tiled kernel graph on B200 (BASELINE.json metric).
 
-Default workload: configs[3], a batch of 64 8K (7680x4320) RGB frames through the
-5-kernel pipeline (gray -> blur5 -> down2 -> sobel3 -> thresh), the configuration the
-north star's targets are stated on (">= 1.3x ... on 8K-class images on one B200, scaling
->= 7x on 8 GPUs for frame batches").  With --gpus N the 64 frames are split across N
-ranks (one process per GPU, frame sharding, no data-path collective).
+Workload (default ``batch64_8k`` = BASELINE configs[3]): 64 frames of 8K (7680x4320) RGB
+through the 5-kernel pipeline gray -> blur5 -> down2 -> sobel3 -> thresh, the
+configuration the north star's 1-GPU target is stated on ("8K-class images on one B200")
+and the one its multi-GPU scaling target uses ("frame batches").  With --gpus N (one
+process per GPU, launched by torchrun) the 64 frames are split across the ranks — frame
+sharding with no data-path collective (strong scaling: the batch is fixed).  Workload
+``strip_65536`` (configs[4]) splits one 65536x65536 image into row strips whose 4 halo
+rows per side move over NCCL send/recv before each step.
 
-Timing (per the driver contract): W untimed warm-up steps, then K timed steps bracketed by
-a barrier + cuda synchronize, CUDA events on the launching stream, max over ranks.  The
-input (6.4 GB of RGB) is far larger than L2 (126 MB) — no L2 flush is needed between
-steps.  A step = one ktiler_execute over the whole batch (all five kernels).
+A step = one ktiler_execute of the plan over the rank's whole share (all five kernels).
+Timing: W untimed warm-up steps, then exactly K steps bracketed by a barrier + cuda
+synchronize, CUDA events on the launching stream, max over ranks.  Inputs (6.4 GB of
+RGB per 64-frame batch) are far larger than L2 (126 MB): no flush is needed between
+steps, and every step re-reads its input from HBM.
 
-Extra keys: roofline (dominant kernel: the persistent executor = the whole step),
-cpu_baseline (the oracle on host cores, bounded sample), e2e (host buffers through
-ktiler_execute_host), untiled (the same graph with the KTILER_FRAG_NONE schedule),
-clocks (nvidia-smi sampled during the timed region).
+Keys beyond the driver contract:
+  untiled       the same graph under the untiled schedule (KTILER_FRAG_NONE: one launch
+                per kernel over the whole batch, the paper's "normal execution mode")
+  roofline      the step against HBM: compulsory bytes (3.25 B/px) / step time; traffic
+                = ncu-measured DRAM bytes per step when profiles/ holds them for this
+                configuration
+  trace         per-kernel share of CTA time in the tiled and untiled steps, from the
+                library's device-side tracer (ktiler_trace_*)
+  e2e           host buffers in, host mask out, through ktiler_execute_host
+  cpu_baseline  the oracle (oracle/ktiler_oracle.c, one thread) on a bounded sample
+  clocks        NVML SM clock + event reasons sampled during the timed region
 """
 from __future__ import annotations
 
@@ -22,7 +33,6 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
 import threading
 import time
@@ -30,11 +40,13 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+METRIC = "Mpix/s end-to-end kernel graph, tiled vs untiled; DRAM bytes & L2 hit rate"
 WORKLOADS = {
-    # name: (W, H, frames_total, BASELINE config index)
-    "batch64_8k": (7680, 4320, 64, 3),
-    "pipeline_4096": (4096, 4096, 1, 1),
-    "pipeline_16384": (16384, 16384, 1, 2),
+    # name: (W, H, frames, BASELINE config index, sharding)
+    "batch64_8k": (7680, 4320, 64, 3, "frames"),
+    "pipeline_4096": (4096, 4096, 1, 1, "replicas"),
+    "pipeline_16384": (16384, 16384, 1, 2, "strips"),
+    "strip_65536": (65536, 65536, 1, 4, "strips"),
 }
 
 
@@ -45,10 +57,11 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ktiler", choices=["ktiler", "reference"])
     ap.add_argument("--workload", default="batch64_8k", choices=sorted(WORKLOADS))
-    ap.add_argument("--mode", default="persistent", choices=["stream", "graph", "persist_l2", "persistent"])
-    ap.add_argument("--kind", default="rows", choices=["budget", "rows", "balanced", "none"])
+    ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain"])
+    ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=0.5)
+    ap.add_argument("--l2-fraction", type=float, default=1.0)
+    ap.add_argument("--window", type=int, default=2)
     ap.add_argument("--no-discard", action="store_true")
     ap.add_argument("--pdl", action="store_true")
     ap.add_argument("--ctas", type=int, default=0)
@@ -58,31 +71,39 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-untiled", action="store_true")
+    ap.add_argument("--no-trace", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--cpu-frames", type=int, default=2)
-    ap.add_argument("--sweep", action="store_true", help="extra lines: fragment-size / mode sweep (not the headline)")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     return ap.parse_args()
 
 
 class Clocks:
-    """nvidia-smi sampler for the timed region."""
+    """NVML sampler (SM clock, clock-event reasons) running during the timed region."""
+
+    NAMES = {"SwPowerCap": "sw_power_cap", "HwSlowdown": "hw_slowdown", "SwThermalSlowdown": "sw_thermal_slowdown",
+             "HwThermalSlowdown": "hw_thermal_slowdown", "HwPowerBrakeSlowdown": "hw_power_brake_slowdown",
+             "ApplicationsClocksSetting": "applications_clocks_setting"}
 
     def __init__(self, idx: int):
-        self.idx, self.samples, self.stop = idx, [], threading.Event()
+        self.samples, self.stop = [], threading.Event()
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            self.N, self.h = N, N.nvmlDeviceGetHandleByIndex(idx)
+            self.max = N.nvmlDeviceGetMaxClockInfo(self.h, N.NVML_CLOCK_SM)
+        except Exception:
+            self.N = None
         self.t = threading.Thread(target=self.run, daemon=True)
 
     def run(self):
-        q = "clocks.sm,clocks.max.sm,clocks_event_reasons.active"
-        while not self.stop.is_set():
+        N = self.N
+        while N is not None and not self.stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={q}", "--format=csv,noheader,nounits"],
-                                     capture_output=True, text=True, timeout=5).stdout.strip()
-                if out:
-                    a = [x.strip() for x in out.split(",")]
-                    self.samples.append((float(a[0]), float(a[1]), int(a[2], 16) if a[2].startswith("0x") else 0))
+                self.samples.append((N.nvmlDeviceGetClockInfo(self.h, N.NVML_CLOCK_SM),
+                                     N.nvmlDeviceGetCurrentClocksEventReasons(self.h)))
             except Exception:
                 pass
-            self.stop.wait(0.2)
+            self.stop.wait(0.002)
 
     def __enter__(self):
         self.t.start()
@@ -90,69 +111,110 @@ class Clocks:
 
     def __exit__(self, *a):
         self.stop.set()
-        self.t.join(timeout=10)
+        self.t.join(timeout=5)
 
     def summary(self):
-        names = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
-                 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown"}
-        if not self.samples:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        load = [s for s in self.samples if not (s[2] & 0x1)] or self.samples
-        reasons = sorted({n for s in load for b, n in names.items() if s[2] & b and b != 0x1})
-        return {"sm_mhz": statistics.median(s[0] for s in load), "sm_max_mhz": max(s[1] for s in load),
-                "reasons": reasons, "samples": len(load)}
+        if self.N is None or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        N = self.N
+        reasons = set()
+        for _, r in self.samples:
+            for k, name in self.NAMES.items():
+                if r & getattr(N, "nvmlClocksEventReason" + k, 0):
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(s[0] for s in self.samples), "sm_max_mhz": self.max,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
 
 
 def peaks():
-    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
-        d = json.load(open(p))
-        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+        d = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        return float(d["hbm_gbs"]), "measured: MEASURED_PEAKS.json hbm_gbs (torch copy, read+write)"
     except Exception:
-        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+        return 6650.0, "fallback: B200_PROFILING.md"
 
 
-def cpu_baseline(W, H, frames, T, seed):
-    """The oracle as it stands (oracle/ktiler_oracle.c, single thread) on a bounded sample."""
+def traffic_for(cfg: dict):
+    """ncu DRAM bytes per step for this exact configuration, if profiles/ has them."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+    except Exception:
+        return None, None
+    for e in d.get("entries", []):
+        if all(e["config"].get(k) == v for k, v in cfg.items()):
+            return e["dram_bytes_per_step"], e["source"]
+    return None, None
+
+
+def cpu_baseline(W, H, T, seed, target_s):
+    """The oracle as it stands (single-threaded C, O-6) on a bounded sample: whole frames
+    of the workload, as many as fit ~target_s seconds (at least one; a row band for
+    images larger than one 8K frame)."""
     from inputs import synth
     from oracle import oracle as O
-    rgb = synth.scene(seed, W, H, frames)
+    rows = H if W * H <= 7680 * 4320 else max(64, (7680 * 4320 // W) // 16 * 16)
+    rgb = synth.scene(seed, W, rows, 1)
     t0 = time.perf_counter()
     O.pipeline(rgb, T=T)
-    dt = time.perf_counter() - t0
-    return {"value": W * H * frames / dt / 1e6, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
-            "sample": f"{frames} of the workload's {W}x{H} scene frames, untiled oracle graph, 1 thread, {dt:.1f} s"}
+    one = time.perf_counter() - t0
+    n, dt = 1, one
+    while dt + one <= target_s:
+        t1 = time.perf_counter()
+        O.pipeline(rgb, T=T)
+        dt += time.perf_counter() - t1
+        n += 1
+    return {"value": W * rows * n / dt / 1e6, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n} x {W}x{rows} scene image(s) through the untiled oracle graph, 1 thread, {dt:.1f} s"}
 
 
 def run_reference(args):
-    """--impl reference: the oracle timed as the reference arm (rank 0 only)."""
-    W, H, Ftot, cfg = WORKLOADS[args.workload]
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
+    """--impl reference: the oracle, as it stands, is the reference arm (rank 0 only)."""
+    W, H, Ftot, cfg, shard = WORKLOADS[args.workload]
+    if int(os.environ.get("RANK", "0")) != 0:
         return
     from inputs import synth
     from oracle import oracle as O
-    frames = 1
-    rgb = synth.scene(args.seed, W, H, frames)
-    for _ in range(max(0, min(args.warmup, 1))):
-        O.pipeline(rgb[:, : H // 8], T=args.T)
-    ts = []
+    rows = H if W * H <= 7680 * 4320 else max(64, (7680 * 4320 // W) // 16 * 16)
+    rgb = synth.scene(args.seed, W, rows, 1)
+    for _ in range(min(args.warmup, 1)):
+        O.pipeline(rgb[:, : max(16, rows // 8)], T=args.T)
     steps = max(1, min(args.steps, 3))
+    ts = []
     for _ in range(steps):
         t0 = time.perf_counter()
         O.pipeline(rgb, T=args.T)
         ts.append(time.perf_counter() - t0)
     ms = 1000 * statistics.mean(ts)
-    v = W * H * frames / (ms / 1000) / 1e6
-    line = {"metric": "Mpix/s end-to-end kernel graph", "value": v, "unit": "Mpix/s", "n_gpus": args.gpus,
-            "steps": steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
-            "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": args.workload, "W": W, "H": H, "frames": Ftot, "baseline_config": cfg},
-            "impl": "reference",
-            "cpu_baseline": {"value": v, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
-                             "sample": f"1 {W}x{H} frame per step (bounded sample of the {Ftot}-frame batch)"},
-            "e2e": {"value": v, "unit": "Mpix/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    v = W * rows / (ms / 1000) / 1e6
+    sample = f"1 {W}x{rows} image per step (bounded sample of the {args.workload} workload), 1 thread"
+    print(json.dumps({
+        "metric": METRIC, "value": v, "unit": "Mpix/s", "n_gpus": args.gpus, "steps": steps, "warmup": args.warmup,
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic", "config": {"workload": args.workload, "W": W, "H": H, "frames": Ftot, "baseline_config": cfg},
+        "impl": "reference",
+        "cpu_baseline": {"value": v, "unit": "Mpix/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": v, "unit": "Mpix/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
+
+
+def trace_shares(pipe, pol):
+    """Per-kernel share of CTA time in one traced execute of a fresh plan of ``pol``."""
+    import numpy as np
+    pl = pipe.b.g.plan(0, **pol)
+    pl.trace_enable(1 << 22)
+    pl.execute(0)
+    pl.trace_read()
+    pl.execute(0)
+    rec, _ = pl.trace_read()
+    names = ("gray", "blur", "down", "sobel", "thresh")
+    launches = pl.launches()
+    k0 = rec[rec["kind"] == 0]
+    node = np.array([launches[i][1] for i in k0["id"]])
+    dur = (k0["t1"].astype(np.int64) - k0["t0"].astype(np.int64)).astype(np.float64)
+    tot = dur.sum()
+    out = {names[v] if v >= 0 else "discard": round(float(dur[node == v].sum() / tot), 3) for v in sorted(set(node.tolist()))}
+    span = int(k0["t1"].max() - k0["t0"].min())
+    del pl
+    return out, span / 1e6
 
 
 def main():
@@ -165,6 +227,7 @@ def main():
 
     from inputs import gpu as G
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    from paper_conf_date_maghazeh0ep19_b200.strips import StripPipeline
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -172,39 +235,53 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    W, H, Ftot, cfg = WORKLOADS[args.workload]
-    per = Ftot // world if Ftot >= world else 1
-    f0 = rank * per
+    W, H, Ftot, cfg_idx, shard = WORKLOADS[args.workload]
     import __graft_entry__ as ge
     ge.build()
+    stream = torch.cuda.current_stream()
+    s = stream.cuda_stream
 
-    p = Pipeline(W, H, per, T=args.T, internal=True)
-    G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per,
-           stream=torch.cuda.current_stream().cuda_stream)
+    sp = None
+    if shard == "strips":
+        sp = StripPipeline(W, H, world, rank, T=args.T, internal=True)
+        p = sp.pipe
+        # each rank generates only the rows it owns; the halo rows come from the neighbours
+        G.fill("scene", args.seed, sp.rgb_ext()[sp.own_offset:].data_ptr(), W * 3, 0, W, H, y0=sp.o0,
+               rows=sp.o1 - sp.o0, F=1, stream=s)
+        pix_rank = W * (sp.o1 - sp.o0)
+        per = 1
+    else:
+        per = Ftot // world if shard == "frames" and Ftot >= world else Ftot
+        f0 = rank * per if shard == "frames" else 0
+        p = Pipeline(W, H, per, T=args.T, internal=True)
+        G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
+        pix_rank = W * H * per
     torch.cuda.synchronize()
     discard = not args.no_discard
     pol = dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode, discard=discard,
-               pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew)
+               pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew, window=args.window)
     plan = p.plan(0, **pol)
     st = plan.stats()
-    stream = torch.cuda.current_stream()
-    s = stream.cuda_stream
 
     def barrier():
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
 
-    def timed(fn, steps, warm):
+    def timed(fn, steps, warm, clocks=None):
         for _ in range(warm):
             fn()
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        if clocks:
+            clocks.__enter__()
         e0.record(stream)
         for _ in range(steps):
             fn()
         e1.record(stream)
         barrier()
+        if clocks:
+            clocks.__exit__()
         ms = e0.elapsed_time(e1) / steps
         if world > 1:
             t = torch.tensor([ms], device="cuda")
@@ -213,20 +290,22 @@ def main():
         return ms
 
     def step():
+        if sp is not None and world > 1:
+            sp.exchange()
         plan.execute(s)
 
-    for _ in range(args.warmup):
-        step()
-    barrier()
-    with Clocks(local) as clk:
-        ms = timed(step, args.steps, 0)
-    pix = W * H * per * world
+    clk = Clocks(local)
+    ms = timed(step, args.steps, args.warmup, clocks=clk)
+    pix = pix_rank * world
     value = pix / (ms / 1000) / 1e6
     peak, peak_src = peaks()
-    comp = p.compulsory_bytes() * world
-    achieved = comp / (ms / 1000) / 1e9
+    comp_bytes = pix * 3.25  # rgb in + mask out: the method's algorithmic bytes
+    achieved = comp_bytes / (ms / 1000) / 1e9
+    tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
+            "discard": discard, "window": args.window, "n_gpus": world}
+    traffic, traffic_src = traffic_for(tcfg)
     line = {
-        "metric": "Mpix/s end-to-end kernel graph (tiled)",
+        "metric": METRIC,
         "value": value,
         "unit": "Mpix/s",
         "n_gpus": world,
@@ -238,65 +317,70 @@ def main():
         "vs_baseline": None,
         "dtype": "u8",
         "data": "synthetic",
-        "config": {"workload": args.workload, "baseline_config": cfg, "W": W, "H": H, "frames": Ftot,
-                   "frames_per_gpu": per, "mode": args.mode, "policy": args.kind, "rows": args.rows,
-                   "l2_fraction": args.l2_fraction, "discard": discard, "pdl": args.pdl,
-                   "l2_flush": "none: input 6.4 GB >> 126 MB L2", "fragments": st["n_fragments"],
-                   "subkernels": st["n_subkernels"], "plan_ms": round(st["plan_ms"], 1)},
+        "config": {"workload": args.workload, "baseline_config": cfg_idx, "W": W, "H": H, "frames": Ftot,
+                   "sharding": shard if world > 1 else "none", "pixels_per_gpu": pix_rank, "mode": args.mode,
+                   "policy": args.kind, "rows": args.rows, "l2_fraction": args.l2_fraction, "window": args.window,
+                   "discard": discard, "pdl": args.pdl,
+                   "l2_flush": "not needed: each step reads >= 6.4 GB of input (>> 126 MB L2)" if Ftot > 1 or W >= 16384
+                   else "none (input smaller than L2: steady-state replay)",
+                   "fragments": st["n_fragments"], "subkernels": st["n_subkernels"],
+                   "plan_ms": round(st["plan_ms"], 1), "input": f"scene(seed={args.seed}) per frame"},
         "gpu_launches": int(st["n_launches"]) * args.steps,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": None, "kernel": "persistent_kernel" if args.mode == "persistent" else "whole graph",
-                     "bytes": "compulsory 3.25 B/px (rgb in + mask out)", "peak_source": peak_src},
+                     "traffic": traffic, "traffic_source": traffic_src,
+                     "kernel": f"one ktiler_execute ({args.mode}: {st['n_launches']} sub-kernel launches)",
+                     "algorithmic_bytes": "3.25 B/px compulsory (rgb 3 in + mask 0.25 out) x pixels per step",
+                     "peak_source": peak_src},
         "clocks": clk.summary(),
     }
     if not args.no_untiled:
         un = p.b.g.plan(0, kind="none", exec_mode="graph", discard=False)
-        ms_un = timed(lambda: un.execute(s), max(3, args.steps // 2), 2)
+        ms_un = timed(lambda: (sp.exchange() if sp is not None and world > 1 else None, un.execute(s)),
+                      max(3, args.steps // 2), 2)
         line["untiled"] = {"value": pix / (ms_un / 1000) / 1e6, "ms_per_step": ms_un,
-                           "speedup_tiled_vs_untiled": ms_un / ms,
-                           "achieved_gbs_untiled_bytes": p.untiled_bytes() * world / (ms_un / 1000) / 1e9}
+                           "tiled_speedup": ms_un / ms,
+                           "achieved_gbs": 9.75 * pix / (ms_un / 1000) / 1e9,
+                           "roofline_frac": 9.75 * pix / (ms_un / 1000) / 1e9 / peak,
+                           "algorithmic_bytes": "9.75 B/px (every intermediate written and read once)"}
         del un
+    if not args.no_trace and rank == 0:
+        try:
+            tiled_sh, tiled_span = trace_shares(p, pol) if args.mode != "persistent" else (None, None)
+            un_sh, un_span = trace_shares(p, dict(kind="none", exec_mode="graph"))
+            line["trace"] = {"tiled_cta_share": tiled_sh, "tiled_span_ms": tiled_span, "untiled_cta_share": un_sh,
+                             "untiled_span_ms": un_span}
+        except Exception as e:  # diagnostics only
+            line["trace"] = {"error": str(e)}
     if not args.no_e2e:
-        rgb_h = torch.empty((per, H, W, 3), dtype=torch.uint8).pin_memory()
-        rgb_h.copy_(p.view("rgb"))
-        mask_h = torch.empty((per, H // 2, W // 2), dtype=torch.uint8).pin_memory()
-        ins = [(p.buf_id("rgb"), rgb_h.data_ptr(), 0, 0)]
-        outs = [(p.buf_id("mask"), mask_h.data_ptr(), 0, 0)]
-        ms_e2e = timed(lambda: plan.execute_host(ins, outs, s), args.e2e_steps, 1)
+        if sp is None:
+            rgb_h = torch.empty((per, H, W, 3), dtype=torch.uint8).pin_memory()
+            rgb_h.copy_(p.view("rgb"))
+            mask_h = torch.empty((per, H // 2, W // 2), dtype=torch.uint8).pin_memory()
+            ins = [(p.buf_id("rgb"), rgb_h.data_ptr(), 0, 0)]
+            outs = [(p.buf_id("mask"), mask_h.data_ptr(), 0, 0)]
+            ms_e2e = timed(lambda: plan.execute_host(ins, outs, s), args.e2e_steps, 1)
+            h2d, d2h = rgb_h.numel(), mask_h.numel()
+        else:
+            own = sp.rgb_ext()[sp.own_offset:sp.own_offset + (sp.o1 - sp.o0)]
+            rgb_h = own.cpu().pin_memory()
+            mask_h = torch.empty(tuple(sp.mask_owned().shape), dtype=torch.uint8).pin_memory()
+
+            def e2e_step():
+                own.copy_(rgb_h, non_blocking=True)
+                step()
+                mask_h.copy_(sp.mask_owned(), non_blocking=True)
+            ms_e2e = timed(e2e_step, args.e2e_steps, 1)
+            h2d, d2h = rgb_h.numel(), mask_h.numel()
         line["e2e"] = {"value": pix / (ms_e2e / 1000) / 1e6, "unit": "Mpix/s", "ms_per_step": ms_e2e,
-                       "h2d_bytes_per_step": rgb_h.numel(), "d2h_bytes_per_step": mask_h.numel()}
+                       "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                       "path": "ktiler_execute_host (pinned host rgb -> device -> plan -> host mask)"
+                       if sp is None else "pinned host rows -> device, halo exchange, ktiler_execute, mask -> host"}
     if rank == 0 and world == 1 and not args.no_cpu:
-        line["cpu_baseline"] = cpu_baseline(W, H if args.workload != "pipeline_16384" else 2048, args.cpu_frames if Ftot > 1 else 1,
-                                            args.T, args.seed)
+        line["cpu_baseline"] = cpu_baseline(W, H, args.T, args.seed, args.cpu_seconds)
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if args.sweep and rank == 0:
-        sweep(p, s, timed, pix)
     if world > 1:
         dist.destroy_process_group()
-
-
-def sweep(p, s, timed, pix):
-    """Fragment-size / mode sweep (BASELINE configs[2] analogue) — extra lines, not headline."""
-    cfgs = [dict(kind="none", exec_mode="graph"), dict(kind="none", exec_mode="graph", discard=True)]
-    for fr in (0.25, 0.5, 1.0):
-        cfgs.append(dict(kind="budget", l2_fraction=fr, exec_mode="graph", discard=True))
-        cfgs.append(dict(kind="budget", l2_fraction=fr, exec_mode="graph", discard=True, pdl=True))
-    for rows in (1, 2, 4, 8):
-        for skew in (0, 1, 4, -1):
-            cfgs.append(dict(kind="rows", rows=rows, exec_mode="persistent", discard=True, skew=skew))
-        cfgs.append(dict(kind="rows", rows=rows, exec_mode="persistent", discard=False))
-    cfgs.append(dict(kind="none", exec_mode="persistent", discard=False))
-    cfgs.append(dict(kind="budget", l2_fraction=0.5, exec_mode="persistent", discard=True))
-    for c in cfgs:
-        try:
-            pl = p.b.g.plan(0, **c)
-            ms = timed(lambda: pl.execute(s), 5, 2)
-            print(json.dumps({"sweep": c, "ms": ms, "Mpix/s": pix / (ms / 1000) / 1e6,
-                              "fragments": pl.stats()["n_fragments"], "launches": pl.stats()["n_launches"]}), flush=True)
-            del pl
-        except Exception as e:  # report and continue
-            print(json.dumps({"sweep": c, "error": str(e)}), flush=True)
 
 
 if __name__ == "__main__":

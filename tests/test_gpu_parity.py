@@ -251,3 +251,23 @@ def test_trace_records(mode):
     assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(rgb, T=40.0)["mask"])
     with pytest.raises(Exception):
         plan.trace_enable(16)  # after the first execute
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("mode", ["graph", "dag"])
+def test_strips_on_one_gpu(world, mode):
+    """§8(e) strip path, GPU side: each rank's extended strip (owned rows + the halo the
+    exchange delivers) through libktiler; concatenated owned masks == whole-image oracle."""
+    from paper_conf_date_maghazeh0ep19_b200.strips import StripPipeline
+    W, H = 1024, 512
+    full = synth.scene(77, W, H, 1)[0]
+    want = O.pipeline(full[None], T=45.0)["mask"][0]
+    got = []
+    for r in range(world):
+        sp = StripPipeline(W, H, world, r, T=45.0, geometry=SMALL, internal=True)
+        sp.rgb_ext().copy_(torch.from_numpy(full[sp.e0:sp.e1]))
+        sp.plan(64 * 1024, kind="budget", exec_mode=mode, discard=True)
+        sp.pipe.run()
+        torch.cuda.synchronize()
+        got.append(sp.mask_owned().cpu().numpy())
+    assert np.array_equal(np.concatenate(got), want)
