@@ -31,7 +31,7 @@ Graph* graph_of(ktiler_graph_t g);
 namespace {
 
 using ktd::DBuf;
-constexpr int MAXR = 4, MAXD = 4;
+constexpr int MAXR = 4, MAXD = 8;
 constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+1 control warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
 constexpr int PERSIST_THREADS = PCOMP_THREADS + 32;
@@ -314,6 +314,18 @@ __global__ void chain_tail_kernel(const __grid_constant__ KParams p) {
   }
   __syncthreads();
   if (p.ndisc) do_discards(p);
+}
+
+// ktiler_selftest(KTILER_SELFTEST_SQRT): the production sqrt2_int vs __fsqrt_rn.
+__global__ void selftest_sqrt_kernel(unsigned n, unsigned long long* bad) {
+  unsigned long long local = 0;
+  for (unsigned i = 2 * (blockIdx.x * blockDim.x + threadIdx.x); i <= n; i += 2 * gridDim.x * blockDim.x) {
+    const float a = (float)i, b = (float)(i + 1);
+    const float2 r = ktd::sqrt2_int(make_float2(a, b));
+    local += (__float_as_uint(r.x) != __float_as_uint(__fsqrt_rn(a))) +
+             (i + 1 <= n && __float_as_uint(r.y) != __float_as_uint(__fsqrt_rn(b)));
+  }
+  if (local) atomicAdd(bad, local);
 }
 
 // GRAPH_CHAIN: advance the epoch (one thread), stream-ordered after the tail kernel.
@@ -849,6 +861,39 @@ void build_launches(ktiler_plan_s* P) {
   flush_disc_only(0);
 }
 
+// GRAPH_DAG: discard lists ride in the prologue of the first launch of a source sub-kernel
+// of fragment f + window or later (f = the list's fragment).  Through the window edge and
+// the per-node chains, that launch follows every sub-kernel of fragments <= f, hence every
+// reader of the list's lines.  Lists with no such launch stay in dag_disc as graph nodes.
+void fold_dag_discards(ktiler_plan_s* P) {
+  const kt::Schedule& S = P->s;
+  const kt::Graph& g = P->g;
+  const int window = P->pol.window > 0 ? P->pol.window : 2;
+  std::vector<int64_t> src_launch(S.nfrag, -1);
+  for (size_t k = 0; k < P->launches.size(); ++k) {
+    const Launch& L = P->launches[k];
+    if (L.node >= 0 && g.in_ch[L.node].empty() && src_launch[S.subs[L.sub].frag] < 0)
+      src_launch[S.subs[L.sub].frag] = (int64_t)k;
+  }
+  std::vector<Launch> rest;
+  for (auto& D : P->dag_disc) {
+    bool placed = false;
+    for (int f = S.subs[D.sub].frag + window; f < S.nfrag && !placed; ++f) {
+      if (src_launch[f] < 0) continue;
+      KParams& k = P->launches[src_launch[f]].kp;
+      if (k.ndisc + D.kp.ndisc > MAXD) continue;
+      for (int j = 0; j < D.kp.ndisc; ++j) {
+        k.d[k.ndisc] = D.kp.d[j];
+        k.dpre[k.ndisc + 1] = k.dpre[k.ndisc] + (D.kp.dpre[j + 1] - D.kp.dpre[j]);
+        ++k.ndisc;
+      }
+      placed = true;
+    }
+    if (!placed) rest.push_back(D);
+  }
+  P->dag_disc.swap(rest);
+}
+
 // ---- tensor maps for TMA staging (driver entry point, resolved at first execute) ----
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
@@ -1001,7 +1046,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     }
     last_of_node[S.subs[i].node] = i;
   }
-  for (auto& D : P->dag_disc) {
+  for (Launch& D : P->dag_disc) {
     std::vector<cudaGraphNode_t> deps;
     for (int r : S.discard_readers[D.sub]) deps.insert(deps.end(), nodes_of[r].begin(), nodes_of[r].end());
     std::sort(deps.begin(), deps.end());
@@ -1350,6 +1395,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
     }
     kt::compute_discards(P->g, P->s);
     build_launches(P);
+    if (pol->exec_mode == KTILER_EXEC_GRAPH_DAG) fold_dag_discards(P);
   } catch (const std::bad_alloc&) {
     delete P;
     return fail(KTILER_E_NOMEM, "host allocation failed while planning");
@@ -1533,6 +1579,23 @@ ktiler_status ktiler_execute_host(ktiler_plan_t p, const ktiler_host_copy* in, i
     s = copy(outc[i], false);
     if (s) return s;
   }
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_selftest(int32_t which, int64_t* failures) {
+  if (!failures) return fail(KTILER_E_INVALID, "NULL argument");
+  if (which != KTILER_SELFTEST_SQRT) return fail(KTILER_E_INVALID, "unknown self-test");
+  unsigned long long* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, sizeof(*d));
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (selftest)");
+  cudaMemset(d, 0, sizeof(*d));
+  selftest_sqrt_kernel<<<1184, 256>>>(2u * 1020u * 1020u, d);
+  unsigned long long h = 0;
+  e = cudaMemcpy(&h, d, sizeof(h), cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  if (e != cudaSuccess) return cuda_fail(e, "selftest");
+  *failures = (int64_t)h;
+  kt::clear_error();
   return KTILER_OK;
 }
 

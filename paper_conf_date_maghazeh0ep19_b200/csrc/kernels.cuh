@@ -123,7 +123,7 @@ __device__ void scalar_tile(int op, const DBuf& in, const DBuf& out, const Tile&
 // staging
 // ---------------------------------------------------------------------------------
 constexpr int BLUR_R = 8;
-constexpr int SOBEL_R = 2;
+constexpr int SOBEL_R = 4;
 
 // ---- TMA bulk copies completing on an mbarrier (the Blackwell async proxy) ----
 __device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
@@ -296,22 +296,17 @@ __device__ __forceinline__ uint4 gray16(const uint32_t w[12]) {
   return o;
 }
 
-// Items of a tile = (row group g, 16-px column segment s).  When nt is a multiple of
-// nseg every thread keeps a fixed segment and strides over row groups: one division per
-// tile, no per-item index arithmetic.
+// Items of a tile = (row group g, 16-px column segment s), item it = g * nseg + s, dealt
+// round-robin to the CTA's threads.  One loop, so each op's (fully unrolled) item body is
+// instantiated once — several copies overflow the instruction cache.  The B200 geometry
+// (256-px tiles, nseg = 16) takes the shift path for the index split.
 template <class F>
 __device__ __forceinline__ void for_items(int nseg, int ngrp, int nt, int tid, F&& f) {
-  if (nseg == 16) {  // the B200 geometry: 256-pixel-wide tiles
-    const int s = tid & 15, gstep = nt >> 4;
-    for (int g = tid >> 4; g < ngrp; g += gstep) f(g, s);
-  } else if (nt % nseg == 0) {
-    const int s = tid % nseg, gstep = nt / nseg;
-    for (int g = tid / nseg; g < ngrp; g += gstep) f(g, s);
-  } else {
-    for (int it = tid; it < nseg * ngrp; it += nt) {
-      const int g = it / nseg;
-      f(g, it - g * nseg);
-    }
+  const int total = nseg * ngrp;
+  const bool n16 = nseg == 16;
+  for (int it = tid; it < total; it += nt) {
+    const int g = n16 ? (it >> 4) : it / nseg;
+    f(g, it - g * nseg);
   }
 }
 
@@ -358,18 +353,31 @@ __device__ __forceinline__ uint32_t pair_at(const uint32_t t[6]) {
 }
 
 // h[k] = (h[2k], h[2k+1]), h[i] = s[i-2] + 4 s[i-1] + 6 s[i] + 4 s[i+1] + s[i+2] <= 4080.
+// Pairs P[i] = (byte x+i-2, byte x+i-1) of the window as u16x2: per window word q,
+// L_q = (b0, b1), M_q = (b1, b2), H_q = (b2, b3) are one PRMT each, and the pair that
+// straddles words q and q+1 is (H_q.hi, L_{q+1}.lo) — one more PRMT (19 in all).
 __device__ __forceinline__ void hblur16(const uint32_t t[6], uint32_t h[8]) {
+  uint32_t L[6], M[6], H[6], X[5];
+#pragma unroll
+  for (int q = 0; q < 6; ++q) {
+    if (q >= 1) L[q] = prmt(t[q], 0, 0x4140);
+    if (q >= 1 && q <= 4) M[q] = prmt(t[q], 0, 0x4241);
+    if (q <= 4) H[q] = prmt(t[q], 0, 0x4342);
+  }
+#pragma unroll
+  for (int q = 0; q < 5; ++q) X[q] = prmt(H[q], L[q + 1], 0x5432);
+  // P[i]: window offset o = i + 2 -> word q = o >> 2, byte o & 3 -> H / X / L / M
   uint32_t P[19];
-  P[0] = pair_at<-2>(t); P[1] = pair_at<-1>(t); P[2] = pair_at<0>(t); P[3] = pair_at<1>(t);
-  P[4] = pair_at<2>(t); P[5] = pair_at<3>(t); P[6] = pair_at<4>(t); P[7] = pair_at<5>(t);
-  P[8] = pair_at<6>(t); P[9] = pair_at<7>(t); P[10] = pair_at<8>(t); P[11] = pair_at<9>(t);
-  P[12] = pair_at<10>(t); P[13] = pair_at<11>(t); P[14] = pair_at<12>(t); P[15] = pair_at<13>(t);
-  P[16] = pair_at<14>(t); P[17] = pair_at<15>(t); P[18] = pair_at<16>(t);
+#pragma unroll
+  for (int i = 0; i < 19; ++i) {
+    const int o = i + 2, q = o >> 2, b = o & 3;
+    P[i] = b == 0 ? L[q] : (b == 1 ? M[q] : (b == 2 ? H[q] : X[q]));
+  }
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
     uint32_t a = P[2 * k] + P[2 * k + 4];
-    uint32_t b = P[2 * k + 1] + P[2 * k + 3];
-    h[k] = a + 4u * b + 6u * P[2 * k + 2];
+    uint32_t c = P[2 * k + 1] + P[2 * k + 3];
+    h[k] = a + 4u * c + 6u * P[2 * k + 2];
   }
 }
 
@@ -451,25 +459,43 @@ __device__ void down_compute(const DBuf& out, const Tile& t, const uint8_t* sm, 
 // (2^23 + 1020); gx^2 + gy^2 < 2^24 is exact in f32 and sqrt_rn is correctly rounded.
 // ---------------------------------------------------------------------------------
 struct SobelRow {
-  uint32_t e[6], o[6];
+  uint32_t e[6], o[6];  // e[1..5] and o[0..4] are used
 };
 __device__ __forceinline__ void sobel_split(const uint32_t t[6], SobelRow& r) {
 #pragma unroll
   for (int q = 0; q < 6; ++q) {
-    r.e[q] = prmt(t[q], 0, 0x4240);
-    r.o[q] = prmt(t[q], 0, 0x4341);
+    if (q >= 1) r.e[q] = prmt(t[q], 0, 0x4240);
+    if (q <= 4) r.o[q] = prmt(t[q], 0, 0x4341);
   }
 }
-__device__ __forceinline__ float lane_f(uint32_t w, bool hi) {
-  const float f = __uint_as_float(prmt(w, 0x4B000000u, hi ? 0x7632 : 0x7610));
-  return f - 8389628.0f;  // 2^23 + 1020
+__device__ __forceinline__ float rsqrt_approx(float x) {
+  float y;
+  asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
 }
-// sqrt_rn of the exact sum; s = 0 (flat regions) would take __fsqrt_rn's special-case
-// subroutine, so it is evaluated on max(s, 1) and selected away.
-__device__ __forceinline__ float mag(float gx, float gy) {
-  const float s = __fmaf_rn(gx, gx, __fmul_rn(gy, gy));
-  const float r = __fsqrt_rn(fmaxf(s, 1.0f));
-  return s > 0.0f ? r : 0.0f;
+// Both lanes of a biased u16x2 word as floats (lane - 1020): (0x4B000000 | lane) is
+// 2^23 + lane exactly, one packed f32x2 add removes 2^23 + 1020.
+__device__ __forceinline__ float2 lanes_f2(uint32_t w) {
+  const float lo = __uint_as_float(prmt(w, 0x4B000000u, 0x7610));
+  const float hi = __uint_as_float(prmt(w, 0x4B000000u, 0x7632));
+  return __fadd2_rn(make_float2(lo, hi), make_float2(-8389628.0f, -8389628.0f));
+}
+// Correctly rounded sqrt of two integer-valued floats s in [0, 2*1020^2]: rsqrt.approx,
+// then one Newton correction r = g + (s - g^2) * y/2 with g = s*y.  Equal to __fsqrt_rn
+// on every integer of that domain — checked exhaustively on the device by
+// ktiler_selftest(KTILER_SELFTEST_SQRT) (tests/test_gpu_parity.py).  s = 0 gives 0 (y is
+// taken at max(s, 1)).
+__device__ __forceinline__ float2 sqrt2_int(float2 s) {
+  const float2 y = make_float2(rsqrt_approx(fmaxf(s.x, 1.0f)), rsqrt_approx(fmaxf(s.y, 1.0f)));
+  const float2 g = __fmul2_rn(s, y);
+  const float2 h = __fmul2_rn(y, make_float2(0.5f, 0.5f));
+  const float2 e = __ffma2_rn(make_float2(-g.x, -g.y), g, s);
+  return __ffma2_rn(e, h, g);
+}
+// Magnitudes of the two lanes of biased (gx, gy) words: gx^2 + gy^2 < 2^21 is exact in f32.
+__device__ __forceinline__ float2 mag2(uint32_t gx, uint32_t gy) {
+  const float2 X = lanes_f2(gx), Y = lanes_f2(gy);
+  return sqrt2_int(__ffma2_rn(X, X, __fmul2_rn(Y, Y)));
 }
 
 template <int R>
@@ -482,6 +508,7 @@ __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm,
     const int ra = g * R, rb = min(ra + R, rows);
     const uint8_t* col = sm + 16 * (s + 1) + ra * stride;  // staged row r holds image row y0 - 1 + r
     uint8_t* drow = ob + ra * pitch + 64 * s;
+    const bool seg_full = full || t.x0 + 16 * s + 16 <= out.W;
     SobelRow w[3];
     uint32_t tw[6];
     smem_window(col, tw);
@@ -496,38 +523,39 @@ __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm,
       const SobelRow& T = w[r % 3];
       const SobelRow& M = w[(r + 1) % 3];
       const SobelRow& B = w[(r + 2) % 3];
+      // column smoothing S = top + 2 mid + bot, difference D = bot - top + 255 (per lane)
       uint32_t SE[6], SO[6], DE[6], DO[6];
 #pragma unroll
       for (int q = 0; q < 6; ++q) {
-        SE[q] = T.e[q] + 2u * M.e[q] + B.e[q];
-        SO[q] = T.o[q] + 2u * M.o[q] + B.o[q];
-        DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
-        DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
+        if (q >= 1) {
+          SE[q] = T.e[q] + B.e[q] + 2u * M.e[q];
+          DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
+        }
+        if (q <= 4) {
+          SO[q] = T.o[q] + B.o[q] + 2u * M.o[q];
+          DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
+        }
       }
       float* dst = reinterpret_cast<float*>(drow + r * pitch);
-      float m[16];
 #pragma unroll
       for (int q = 1; q <= 4; ++q) {
         const uint32_t gxe = SO[q] + 0x03FC03FCu - prmt(SO[q - 1], SO[q], 0x5432);
         const uint32_t gye = prmt(DO[q - 1], DO[q], 0x5432) + 2u * DE[q] + DO[q];
         const uint32_t gxo = prmt(SE[q], SE[q + 1], 0x5432) + 0x03FC03FCu - SE[q];
         const uint32_t gyo = DE[q] + 2u * DO[q] + prmt(DE[q], DE[q + 1], 0x5432);
-        const int b = 4 * (q - 1);
-        m[b + 0] = mag(lane_f(gxe, false), lane_f(gye, false));
-        m[b + 1] = mag(lane_f(gxo, false), lane_f(gyo, false));
-        m[b + 2] = mag(lane_f(gxe, true), lane_f(gye, true));
-        m[b + 3] = mag(lane_f(gxo, true), lane_f(gyo, true));
-      }
-      if (full || t.x0 + 16 * s + 16 <= out.W) {
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          st16(dst + 4 * q, make_uint4(__float_as_uint(m[4 * q]), __float_as_uint(m[4 * q + 1]),
-                                       __float_as_uint(m[4 * q + 2]), __float_as_uint(m[4 * q + 3])));
-      } else {
-        const int64_t x = t.x0 + 16 * s;
-#pragma unroll
-        for (int k = 0; k < 16; ++k)
-          if (x + k < out.W) dst[k] = m[k];
+        const float2 ev = mag2(gxe, gye);  // columns c, c+2 (c = x + 4q - 4)
+        const float2 od = mag2(gxo, gyo);  // columns c+1, c+3
+        if (seg_full) {
+          st16(dst + 4 * (q - 1), make_uint4(__float_as_uint(ev.x), __float_as_uint(od.x), __float_as_uint(ev.y),
+                                             __float_as_uint(od.y)));
+        } else {
+          const int64_t x = t.x0 + 16 * s + 4 * (q - 1);
+          float* d = dst + 4 * (q - 1);
+          if (x < out.W) d[0] = ev.x;
+          if (x + 1 < out.W) d[1] = od.x;
+          if (x + 2 < out.W) d[2] = ev.y;
+          if (x + 3 < out.W) d[3] = od.y;
+        }
       }
     }
   });

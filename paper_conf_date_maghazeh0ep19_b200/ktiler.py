@@ -27,6 +27,16 @@ EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRA
 FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE}
 
 
+SELFTEST_SQRT = 0
+
+
+def selftest(which: int = SELFTEST_SQRT) -> int:
+    """ktiler_selftest: number of failing inputs (0 = pass)."""
+    n = ctypes.c_int64()
+    _check(lib().ktiler_selftest(which, ctypes.byref(n)))
+    return n.value
+
+
 class KtilerError(RuntimeError):
     def __init__(self, status: int, msg: str):
         self.status = status
@@ -87,7 +97,7 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_graph_block_deps", "ktiler_graph_block_lines", "ktiler_plan", "ktiler_plan_destroy",
            "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
            "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
-           "ktiler_trace_read", "ktiler_plan_get_launch"]
+           "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest"]
 
 _LIB = None
 
@@ -124,6 +134,7 @@ def lib() -> ctypes.CDLL:
         "ktiler_trace_enable": ([vp, i64], st),
         "ktiler_trace_read": ([vp, vp, i64, P(i64)], st),
         "ktiler_plan_get_launch": ([vp, i64, P(i32), P(i32), P(i64)], st),
+        "ktiler_selftest": ([i32, P(i64)], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)

@@ -26,7 +26,7 @@ B200_GEOMETRY = {
     "gray": (256, 32, 256),    # 512 items of 16 px; 24.6 KB staged rgb
     "blur": (256, 64, 128),    # 128 column strips x 8 rows; 19.6 KB staged halo tile
     "down": (256, 32, 256),    # 512 items; 16 KB staged blur rows
-    "sobel": (256, 32, 256),   # 256 strips x 2 rows; 9.8 KB halo tile
+    "sobel": (256, 64, 256),   # 256 strips x 4 rows; 19 KB halo tile
     "thresh": (256, 16, 256),  # 256 items; 16 KB staged f32
 }
 

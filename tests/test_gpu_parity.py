@@ -271,3 +271,9 @@ def test_strips_on_one_gpu(world, mode):
         torch.cuda.synchronize()
         got.append(sp.mask_owned().cpu().numpy())
     assert np.array_equal(np.concatenate(got), want)
+
+
+def test_selftest_sqrt_exhaustive():
+    """The Sobel magnitude's fast sqrt equals __fsqrt_rn on every integer of its domain."""
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler
+    assert ktiler.selftest(ktiler.SELFTEST_SQRT) == 0
