@@ -861,30 +861,70 @@ void build_launches(ktiler_plan_s* P) {
   flush_disc_only(0);
 }
 
-// GRAPH_DAG: discard lists ride in the prologue of the first launch of a source sub-kernel
-// of fragment f + window or later (f = the list's fragment).  Through the window edge and
-// the per-node chains, that launch follows every sub-kernel of fragments <= f, hence every
-// reader of the list's lines.  Lists with no such launch stay in dag_disc as graph nodes.
-void fold_dag_discards(ktiler_plan_s* P) {
+// GRAPH_DAG edges at sub-kernel level: exact sub-kernel dependencies (Schedule::sub_deps),
+// the previous sub-kernel of the same node, and the run-ahead window (a sub-kernel with no
+// producers in fragment f waits for the leaf sub-kernels of fragment f - window).
+std::vector<std::vector<int>> dag_edges(const ktiler_plan_s* P) {
   const kt::Schedule& S = P->s;
   const kt::Graph& g = P->g;
+  const int nsub = (int)S.subs.size();
   const int window = P->pol.window > 0 ? P->pol.window : 2;
-  std::vector<int64_t> src_launch(S.nfrag, -1);
+  std::vector<std::vector<int>> leaf_subs(S.nfrag), e(nsub);
+  for (int i = 0; i < nsub; ++i)
+    if (g.out_ch[S.subs[i].node].empty()) leaf_subs[S.subs[i].frag].push_back(i);
+  std::vector<int> last_of_node(g.nodes.size(), -1);
+  for (int i = 0; i < nsub; ++i) {
+    e[i].assign(S.sub_deps[i].begin(), S.sub_deps[i].end());
+    const int prev = last_of_node[S.subs[i].node];
+    if (prev >= 0) e[i].push_back(prev);
+    const int f = S.subs[i].frag;
+    if (S.sub_deps[i].empty() && f >= window) e[i].insert(e[i].end(), leaf_subs[f - window].begin(), leaf_subs[f - window].end());
+    std::sort(e[i].begin(), e[i].end());
+    e[i].erase(std::unique(e[i].begin(), e[i].end()), e[i].end());
+    last_of_node[S.subs[i].node] = i;
+  }
+  return e;
+}
+
+// GRAPH_DAG: each discard list rides in the prologue of the earliest later launch that
+// (transitively) follows every reader of the list's lines — usually the very next
+// sub-kernel of the schedule — so dead lines leave L2 as early as in the linear graph,
+// without extra graph nodes.  Lists with no such launch stay in dag_disc as nodes.
+void fold_dag_discards(ktiler_plan_s* P) {
+  const kt::Schedule& S = P->s;
+  const int nsub = (int)S.subs.size();
+  const std::vector<std::vector<int>> e = dag_edges(P);
+  // ancestor bitsets in schedule order (every edge points to an earlier sub-kernel)
+  const int words = (nsub + 63) / 64;
+  std::vector<uint64_t> anc((size_t)nsub * words, 0);
+  for (int i = 0; i < nsub; ++i) {
+    uint64_t* a = &anc[(size_t)i * words];
+    for (int d : e[i]) {
+      const uint64_t* b = &anc[(size_t)d * words];
+      for (int w = 0; w < words; ++w) a[w] |= b[w];
+      a[d >> 6] |= 1ull << (d & 63);
+    }
+  }
+  std::vector<int64_t> first_launch(nsub, -1);
   for (size_t k = 0; k < P->launches.size(); ++k) {
     const Launch& L = P->launches[k];
-    if (L.node >= 0 && g.in_ch[L.node].empty() && src_launch[S.subs[L.sub].frag] < 0)
-      src_launch[S.subs[L.sub].frag] = (int64_t)k;
+    if (L.node >= 0 && L.sub >= 0 && first_launch[L.sub] < 0) first_launch[L.sub] = (int64_t)k;
   }
   std::vector<Launch> rest;
   for (auto& D : P->dag_disc) {
+    const std::vector<int32_t>& readers = S.discard_readers[D.sub];
     bool placed = false;
-    for (int f = S.subs[D.sub].frag + window; f < S.nfrag && !placed; ++f) {
-      if (src_launch[f] < 0) continue;
-      KParams& k = P->launches[src_launch[f]].kp;
+    for (int j = D.sub + 1; j < nsub && !placed; ++j) {
+      if (first_launch[j] < 0) continue;
+      const uint64_t* a = &anc[(size_t)j * words];
+      bool ok = true;
+      for (int r : readers) ok = ok && ((a[r >> 6] >> (r & 63)) & 1) != 0;
+      if (!ok) continue;
+      KParams& k = P->launches[first_launch[j]].kp;
       if (k.ndisc + D.kp.ndisc > MAXD) continue;
-      for (int j = 0; j < D.kp.ndisc; ++j) {
-        k.d[k.ndisc] = D.kp.d[j];
-        k.dpre[k.ndisc + 1] = k.dpre[k.ndisc] + (D.kp.dpre[j + 1] - D.kp.dpre[j]);
+      for (int q = 0; q < D.kp.ndisc; ++q) {
+        k.d[k.ndisc] = D.kp.d[q];
+        k.dpre[k.ndisc + 1] = k.dpre[k.ndisc] + (D.kp.dpre[q + 1] - D.kp.dpre[q]);
         ++k.ndisc;
       }
       placed = true;
@@ -1004,10 +1044,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   cudaError_t e = cudaGraphCreate(&gr, 0);
   if (e != cudaSuccess) return cuda_fail(e, "cudaGraphCreate");
   std::vector<std::vector<cudaGraphNode_t>> nodes_of(nsub);
-  std::vector<std::vector<int>> leaf_subs(S.nfrag);
-  for (int i = 0; i < nsub; ++i)
-    if (g.out_ch[S.subs[i].node].empty()) leaf_subs[S.subs[i].frag].push_back(i);
-  std::vector<int> last_of_node(g.nodes.size(), -1);
+  const std::vector<std::vector<int>> edges = dag_edges(P);
   auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, cudaGraphNode_t* node) -> ktiler_status {
     kfn_t fn = launch_fn(L);
     int64_t grid = 0;
@@ -1027,12 +1064,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   size_t li = 0;
   for (int i = 0; i < nsub; ++i) {
     std::vector<cudaGraphNode_t> deps;
-    for (int d : S.sub_deps[i]) deps.insert(deps.end(), nodes_of[d].begin(), nodes_of[d].end());
-    const int prev = last_of_node[S.subs[i].node];
-    if (prev >= 0) deps.insert(deps.end(), nodes_of[prev].begin(), nodes_of[prev].end());
-    const int f = S.subs[i].frag;
-    if (S.sub_deps[i].empty() && f >= window)
-      for (int j : leaf_subs[f - window]) deps.insert(deps.end(), nodes_of[j].begin(), nodes_of[j].end());
+    for (int d : edges[i]) deps.insert(deps.end(), nodes_of[d].begin(), nodes_of[d].end());
     std::sort(deps.begin(), deps.end());
     deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
     for (; li < P->launches.size() && P->launches[li].sub == i; ++li) {
@@ -1044,7 +1076,6 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
       }
       nodes_of[i].push_back(nd);
     }
-    last_of_node[S.subs[i].node] = i;
   }
   for (Launch& D : P->dag_disc) {
     std::vector<cudaGraphNode_t> deps;
@@ -1474,7 +1505,7 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
       p->pp.tb = p->tb;
     } else {
       for (auto& L : p->launches)
-        if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar)
+        if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar && L.kp.stage_bytes)
           L.kp.use_tmap = make_tmap(p->g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
       if (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN) {
         ktiler_status s = setup_chain(p);
