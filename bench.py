@@ -57,7 +57,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ktiler", choices=["ktiler", "reference"])
     ap.add_argument("--workload", default="batch64_8k", choices=sorted(WORKLOADS))
-    ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain"])
+    ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
     ap.add_argument("--l2-fraction", type=float, default=1.0)

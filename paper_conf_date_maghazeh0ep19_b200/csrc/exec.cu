@@ -32,11 +32,12 @@ namespace {
 
 using ktd::DBuf;
 constexpr int MAXR = 4, MAXD = 8;
-constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+1 control warp)
+constexpr int PCOMP_WARPS = 8;  // compute warps per persistent CTA (+ producer + publisher warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
-constexpr int PERSIST_THREADS = PCOMP_THREADS + 32;
+constexpr int PERSIST_THREADS = PCOMP_THREADS + 64;
+constexpr int PSTAGES = 3;       // staging ring depth
 constexpr int MAXDEAD = 64;
-constexpr int PERSIST_MINB_DEFAULT = 4;
+constexpr int PERSIST_MINB_DEFAULT = 2;
 
 struct LRect {
   int32_t x0, y0, z0, x1, y1, z1;
@@ -72,6 +73,7 @@ struct KParams {
   int64_t lid;          // launch index (trace id)
   uint32_t box_bytes;   // bytes one tensor-TMA box delivers
   int32_t use_tmap;
+  int32_t in_stream;    // input is a graph input: load it evict-first
   DBuf in, out;
   int32_t tw, th;
   float T;
@@ -243,7 +245,7 @@ __global__ void __launch_bounds__(256, (OP == 1 || OP == 3) ? 3 : 4) op_kernel(c
       if (p.use_tmap) {
         if (tid == 0) {
           s_tile[slot] = t;
-          ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot]);
+          ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot], p.in_stream != 0);
         }
       } else {
         if (tid == 0) s_tile[slot] = t;
@@ -349,6 +351,7 @@ struct PNode {
   CUtensorMap tmap;  // input tile map (tensor TMA), valid if use_tmap
   uint32_t box_bytes;
   int32_t use_tmap;
+  int32_t in_stream;  // input is a graph input: load it evict-first
   DBuf in, out;
   int32_t op, scalar, tw, th;
   float T;
@@ -464,10 +467,7 @@ __device__ __forceinline__ void ctl_wait(const PParams& p, const TInfo& a, unsig
 // the last reader of a block drops that block's lines from L2 without write-back.
 __device__ __forceinline__ void ctl_release(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
   const PNode& nd = *a.nd;
-  if (lane == 0) {
-    __threadfence();
-    st_release(p.flags + nd.flag0 + (a.t.z * nd.gy + a.by) * nd.gx + a.bx, epoch);
-  }
+  if (lane == 0) st_release(p.flags + nd.flag0 + (a.t.z * nd.gy + a.by) * nd.gx + a.bx, epoch);
   if (!(p.discard && nd.disc_in)) return;
   for (int base = 0; base < a.ndep; base += 32) {
     const int i = base + lane;
@@ -501,155 +501,115 @@ __device__ __forceinline__ void ctl_release(const PParams& p, const TInfo& a, un
   }
 }
 
-// Persistent executor.  One launch runs the whole schedule: tiles are taken in schedule
-// order from an atomic ticket (deadlock-free: producers precede consumers and each CTA
-// handles its tickets in order, so the smallest unfinished ticket is always runnable).
-// Warp specialization inside a CTA:
-//   control warp  takes tickets, waits for a tile's producer flags (acquire), streams its
-//                 input tile into one of two shared buffers with TMA bulk copies (one per
-//                 row, completing on that buffer's mbarrier), and — once the compute
-//                 warps signal on a named barrier that a buffer's tile is done — publishes
-//                 the tile's flag (release) and retires dead producer lines (discard);
-//   compute warps wait on the buffer's mbarrier, compute the tile from shared memory and
-//                 arrive (non-blocking) on the buffer's named barrier.
-// So the input of tile i+1 streams while tile i computes, and no compute warp ever waits
-// on a fence, a flag or an atomic.  The control warp never waits on a producer flag while
-// it holds an unreleased tile of its own.
+// Persistent executor.  One launch runs the whole schedule.  Ticket t (a tile, in the
+// order of the descriptor table: the schedule's total order, optionally skewed) belongs
+// to CTA t mod G, and every CTA runs its tickets in order — no ticket atomics.  Deadlock-
+// free: a tile's producers have smaller tickets, so the smallest unfinished ticket is
+// always runnable and its CTA reaches it (all its smaller tickets are finished).
+// Warp specialization inside a CTA, around a PSTAGES-deep ring of staging buffers:
+//   producer warp   for each of its tickets: wait until the ring slot is free (s_empty,
+//                   released by the publisher), wait (acquire) for the tile's producer
+//                   flags, stream the input tile into the slot with one TMA (s_full);
+//   compute warps   wait on s_full, compute the tile from shared memory, arrive
+//                   (non-blocking) on the slot's named barrier;
+//   publisher warp  syncs on that barrier, frees the slot, publishes the tile's flag
+//                   (gpu-scope release) and retires dead producer lines (reader counts).
+// So the dependency wait and TMA latency of later tiles, and the release of earlier ones,
+// overlap the compute of the current tile: no compute warp waits on a flag or a fence.
 template <int MINB>
 __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const __grid_constant__ PParams p) {
-  __shared__ __align__(8) uint64_t s_full[2];
-  __shared__ uint64_t s_desc[2];
-  __shared__ TInfo s_ti[2];  // decoded tile of each buffer (control warp -> compute warps)
+  __shared__ __align__(8) uint64_t s_full[PSTAGES];
+  __shared__ __align__(8) uint64_t s_empty[PSTAGES];
+  __shared__ uint64_t s_desc[PSTAGES];
+  __shared__ TInfo s_ti[PSTAGES];  // decoded tile of each slot (producer -> compute warps)
   __shared__ unsigned int s_epoch;
   __shared__ uint64_t s_tc0, s_tq0;  // trace timestamps (kept out of registers)
   extern __shared__ __align__(128) uint8_t ktsm[];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     s_epoch = *(volatile unsigned int*)&p.ctrl->epoch;
-    ktd::mbar_init(&s_full[0], 1);
-    ktd::mbar_init(&s_full[1], 1);
+    for (int s = 0; s < PSTAGES; ++s) {
+      ktd::mbar_init(&s_full[s], 1);
+      ktd::mbar_init(&s_empty[s], 1);
+    }
     ktd::fence_proxy_async();
   }
   __syncthreads();
   const unsigned int epoch = s_epoch;
+  const int64_t G = gridDim.x;
   if (warp == PCOMP_WARPS) {
-    // ------------------------------ control warp ------------------------------
-    int64_t tq = 0;        // lane 0: next ticket (grabbed one tile ahead)
-    uint64_t dq = 0;       // lane 0: its descriptor
-    if (lane == 0) {
-      tq = atomicAdd(&p.ctrl->ticket, 1u);
-      dq = tq < p.total ? p.desc[tq] : 0;
-    }
-    // the tile in flight in "this" buffer (b) and in the "other" one (b ^ 1); swapped
-    // every iteration, so no runtime-indexed arrays (they would live in local memory)
-    uint64_t d_this = 0, d_other = 0;
-    bool u_this = false, u_other = false;
-    // Reorder window: up to 4 taken-but-unstaged tickets, oldest first.  The control warp
-    // stages the oldest one whose producers are complete, so a not-yet-ready consumer does
-    // not idle the CTA; if none is ready it waits for the oldest (always runnable once
-    // every smaller ticket is done, so the executor stays deadlock-free).
-    uint64_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
-    int nw = 0;
-    bool more = true;
-    int b = 0;
-    for (;; b ^= 1) {
-      while (nw < 4 && more) {  // refill the window (one grab in steady state)
-        const int64_t t = __shfl_sync(FULL, tq, 0);
-        const uint64_t d = __shfl_sync(FULL, dq, 0);
-        if (t >= p.total) {
-          more = false;
-          break;
-        }
+    // ------------------------------ producer warp ------------------------------
+    int s = 0;
+    unsigned ph = 0;  // bit s: parity of slot s's current use
+    for (int64_t t = blockIdx.x, k = 0;; t += G, ++k) {
+      if (k >= PSTAGES) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
+      if (t >= p.total) {
         if (lane == 0) {
-          tq = atomicAdd(&p.ctrl->ticket, 1u);
-          dq = tq < p.total ? p.desc[tq] : 0;
-        }
-        if (nw == 0) w0 = d; else if (nw == 1) w1 = d; else if (nw == 2) w2 = d; else w3 = d;
-        ++nw;
-      }
-      // buffer b is free once the compute warps are done with the tile two back
-      if (u_this) {
-        nbar_sync(1 + b, PERSIST_THREADS);
-        ctl_release(p, decode(p, d_this), epoch, lane);
-        u_this = false;
-      }
-      if (nw == 0) {
-        if (lane == 0) {
-          s_desc[b] = DESC_STOP;
-          mbar_arrive(&s_full[b]);
+          s_desc[s] = DESC_STOP;
+          mbar_arrive(&s_full[s]);
         }
         break;
       }
       if (p.tb.rec && lane == 0) s_tq0 = gtimer();
-      int ch = -1;
-      if (ctl_probe(p, decode(p, w0), epoch, lane)) ch = 0;
-      else if (nw > 1 && ctl_probe(p, decode(p, w1), epoch, lane)) ch = 1;
-      else if (nw > 2 && ctl_probe(p, decode(p, w2), epoch, lane)) ch = 2;
-      else if (nw > 3 && ctl_probe(p, decode(p, w3), epoch, lane)) ch = 3;
-      if (ch < 0) {
-        if (u_other) {  // never wait while holding an unreleased tile
-          nbar_sync(1 + (b ^ 1), PERSIST_THREADS);
-          ctl_release(p, decode(p, d_other), epoch, lane);
-          u_other = false;
-        }
-        ctl_wait(p, decode(p, w0), epoch, lane);
-        ch = 0;
-      }
-      const uint64_t d = ch == 0 ? w0 : (ch == 1 ? w1 : (ch == 2 ? w2 : w3));
-      if (ch <= 0) w0 = w1;
-      if (ch <= 1) w1 = w2;
-      if (ch <= 2) w2 = w3;
-      --nw;
+      const uint64_t d = p.desc[t];
       const TInfo a = decode(p, d);
-      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+      ctl_wait(p, a, epoch, lane);
+      uint8_t* buf = ktsm + s * p.stage_bytes;
       if (lane == 0) {
-        s_desc[b] = d;
-        s_ti[b] = a;
+        s_desc[s] = d;
+        s_ti[s] = a;
       }
       if (a.nd->scalar) {
-        if (lane == 0) mbar_arrive(&s_full[b]);
+        if (lane == 0) mbar_arrive(&s_full[s]);
       } else {
         ktd::fence_proxy_async();
         if (a.nd->use_tmap) {
-          if (lane == 0) ktd::stage_issue_tmap(a.nd->op, &a.nd->tmap, a.nd->box_bytes, a.nd->in, a.t, buf, &s_full[b]);
+          if (lane == 0)
+            ktd::stage_issue_tmap(a.nd->op, &a.nd->tmap, a.nd->box_bytes, a.nd->in, a.t, buf, &s_full[s], a.nd->in_stream != 0);
         } else {
-          ktd::stage_issue(a.nd->op, a.nd->in, a.t, buf, &s_full[b], lane);
+          ktd::stage_issue(a.nd->op, a.nd->in, a.t, buf, &s_full[s], lane);
         }
       }
       if (p.tb.rec && lane == 0) trace_put(p.tb, d, 1, s_tq0, gtimer());
-      // swap roles for the next iteration (which stages into b ^ 1)
-      d_this = d_other;
-      u_this = u_other;
-      d_other = d;
-      u_other = true;
+      ph ^= 1u << s;
+      s = s + 1 == PSTAGES ? 0 : s + 1;
     }
-    // drain: the tile in the other buffer (if any) is the last one in flight
-    if (u_other) {
-      nbar_sync(1 + (b ^ 1), PERSIST_THREADS);
-      ctl_release(p, decode(p, d_other), epoch, lane);
+  } else if (warp == PCOMP_WARPS + 1) {
+    // ------------------------------ publisher warp ------------------------------
+    int s = 0;
+    for (int64_t t = blockIdx.x; t < p.total; t += G) {
+      nbar_sync(1 + s, PCOMP_THREADS + 32);  // the compute warps are done with slot s
+      const uint64_t d = s_desc[s];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_empty[s]);  // the producer may refill slot s
+      ctl_release(p, decode(p, d), epoch, lane);
+      s = s + 1 == PSTAGES ? 0 : s + 1;
     }
   } else {
     // ------------------------------ compute warps ------------------------------
-    unsigned ph = 0;  // bit b = phase parity of buffer b's mbarrier
-    for (int b = 0;; b ^= 1) {
-      ktd::mbar_wait(&s_full[b], (ph >> b) & 1u);
-      ph ^= 1u << b;
-      if (s_desc[b] == DESC_STOP) break;
+    int s = 0;
+    unsigned ph = 0;
+    for (;;) {
+      ktd::mbar_wait(&s_full[s], (ph >> s) & 1u);
+      ph ^= 1u << s;
+      if (s_desc[s] == DESC_STOP) break;
       if (p.tb.rec && tid == 0) s_tc0 = gtimer();
-      const TInfo a = s_ti[b];
+      const TInfo a = s_ti[s];
       const PNode& nd = *a.nd;
-      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
+      uint8_t* buf = ktsm + s * p.stage_bytes;
       if (nd.scalar) {
         ktd::scalar_tile(nd.op, nd.in, nd.out, a.t, nd.T, PCOMP_THREADS, tid);
       } else {
         if ((nd.op == 1 || nd.op == 3) && ktd::needs_fix(nd.op, nd.in, a.t)) {
           ktd::stage_fix(nd.op, nd.in, a.t, buf, PCOMP_THREADS, tid);
-          nbar_sync(3, PCOMP_THREADS);
+          nbar_sync(4, PCOMP_THREADS);
         }
         ktd::compute_tile(nd.op, nd.out, a.t, buf, nd.T, PCOMP_THREADS, tid);
       }
-      if (p.tb.rec && tid == 0) trace_put(p.tb, s_desc[b], 2, s_tc0, gtimer());
-      nbar_arrive(1 + b, PERSIST_THREADS);
+      if (p.tb.rec && tid == 0) trace_put(p.tb, s_desc[s], 2, s_tc0, gtimer());
+      __threadfence_block();  // this thread's tile writes before the hand-off (cumulative release)
+      nbar_arrive(1 + s, PCOMP_THREADS + 32);
+      s = s + 1 == PSTAGES ? 0 : s + 1;
     }
   }
   __syncthreads();
@@ -767,7 +727,8 @@ void build_launches(ktiler_plan_s* P) {
   const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
   // GRAPH_DAG and GRAPH_CHAIN keep each sub-kernel's discard list apart (dag_disc, sub =
   // the list's sub-kernel): DAG makes them graph nodes, CHAIN attaches them to later launches
-  const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN;
+  const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN ||
+                   P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE;
   std::vector<DRect> pending;
   auto flush_disc_only = [&](size_t keep) {
     while (pending.size() > keep) {
@@ -812,6 +773,7 @@ void build_launches(ktiler_plan_s* P) {
         L.n = const_cast<kt::Node*>(&n);
         L.kp.in = dbuf(g.bufs[r.buf]);
         L.kp.out = dbuf(g.bufs[w.buf]);
+        L.kp.in_stream = !g.written_by_node(r.buf);
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
         L.kp.T = n.T;
@@ -869,6 +831,27 @@ std::vector<std::vector<int>> dag_edges(const ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const int nsub = (int)S.subs.size();
   const int window = P->pol.window > 0 ? P->pol.window : 2;
+  if (P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE) {
+    // wave(sub) = fragment + node depth; every sub-kernel of wave w depends on every
+    // sub-kernel of the previous non-empty wave (a barrier).  Producers sit at a smaller
+    // depth in the same or an earlier fragment, hence in an earlier wave.
+    std::vector<int> depth(g.nodes.size(), 0);
+    for (int v : g.topo)
+      for (auto& c : g.in_ch[v]) depth[v] = std::max(depth[v], depth[c.u] + 1);
+    int dmax = 0;
+    for (int d : depth) dmax = std::max(dmax, d);
+    std::vector<std::vector<int>> waves(S.nfrag + dmax + 1);
+    for (int i = 0; i < nsub; ++i) waves[S.subs[i].frag + depth[S.subs[i].node]].push_back(i);
+    std::vector<std::vector<int>> e(nsub);
+    const std::vector<int>* prev = nullptr;
+    for (auto& w : waves) {
+      if (w.empty()) continue;
+      if (prev)
+        for (int i : w) e[i] = *prev;
+      prev = &w;
+    }
+    return e;
+  }
   std::vector<std::vector<int>> leaf_subs(S.nfrag), e(nsub);
   for (int i = 0; i < nsub; ++i)
     if (g.out_ch[S.subs[i].node].empty()) leaf_subs[S.subs[i].frag].push_back(i);
@@ -1012,7 +995,12 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
   // tile by default, so concurrent sub-kernels interleave at tile granularity
   static const int tpc_env = getenv("KTILER_TILES_PER_CTA") ? atoi(getenv("KTILER_TILES_PER_CTA")) : -1;
   const bool chain = P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN;
-  const int tpc = tpc_env >= 0 ? tpc_env : ((P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || chain) ? 1 : 0);
+  // Default: a launch much larger than the device (the untiled kernels) gets 2 tiles per
+  // CTA and leaves the balancing to the hardware scheduler; smaller ones (sub-kernels) get
+  // one resident wave of CTAs that grid-stride over the tiles (fewer CTA setups, no
+  // partial last wave).  GRAPH_CHAIN: one tile per CTA (fine-grained flags).  Measured on
+  // 64 x 8K; KTILER_TILES_PER_CTA overrides.
+  const int tpc = tpc_env >= 0 ? tpc_env : (chain ? 1 : (L.blocks > 8 * L.resident ? 2 : 0));
   if (L.node >= 0 && !L.n->scalar) {
     if (tpc > 0) grid = (grid + tpc - 1) / tpc;
     else grid = std::min<int64_t>(grid, L.resident);
@@ -1023,8 +1011,11 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
     L.resident = 0;
     return prep_launch(P, L, fn, grid_out);
   }
-  // (GRAPH_CHAIN: the launch's own CTAs share its discards; extra CTAs would only spin)
-  if (L.kp.ndisc && !chain) grid = std::max<int64_t>(grid, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+  // The launch's own CTAs share its discard lines (grid-stride): enlarging the grid for
+  // them would turn multi-tile CTAs into one- or zero-tile CTAs that pay the CTA setup.
+  // Discard-only launches size their grid to the lines.
+  if (L.node < 0 && L.kp.ndisc) grid = std::max<int64_t>(1, std::min<int64_t>(1184, (L.kp.dpre[L.kp.ndisc] + 255) / 256));
+  (void)chain;
   *grid_out = grid;
   return KTILER_OK;
 }
@@ -1295,14 +1286,15 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
       q.disc_in = (ib.d.flags & KTILER_BUF_INTERNAL) && discardable(ib);
     }
     q.use_tmap = !n.scalar && make_tmap(g, n, &q.tmap, &q.box_bytes);
+    q.in_stream = !g.written_by_node(r.buf);
   }
   int nsm = 0, occ = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
   {
-    // registers vs CTAs per SM (KTILER_PERSIST_MINB = 2, 3 or 4 minimum resident CTAs)
+    // registers vs CTAs per SM (KTILER_PERSIST_MINB = 2 or 3 minimum resident CTAs)
     const char* ev = getenv("KTILER_PERSIST_MINB");
     int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
-    P->pfn = mb >= 5 ? persistent_kernel<5> : (mb == 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>));
+    P->pfn = mb >= 3 ? persistent_kernel<3> : persistent_kernel<2>;
   }
   P->psmem = 0;
   for (auto& n : g.nodes) {
@@ -1310,7 +1302,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     if (!n.scalar) P->psmem = std::max(P->psmem, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
   }
   P->pp.stage_bytes = P->psmem;
-  P->psmem *= 2;
+  P->psmem *= PSTAGES;
   if (P->psmem > 32 * 1024) {
     cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
@@ -1404,7 +1396,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
   kt::Graph* G = kt::graph_of(gh);
   ktiler_status s = G->finalize();
   if (s) return s;
-  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_CHAIN)
+  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_WAVE)
     return fail(KTILER_E_INVALID, "unknown exec_mode");
   if (cache_bytes == 0) {
     int dev = 0, l2 = 0;
@@ -1426,7 +1418,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
     }
     kt::compute_discards(P->g, P->s);
     build_launches(P);
-    if (pol->exec_mode == KTILER_EXEC_GRAPH_DAG) fold_dag_discards(P);
+    if (pol->exec_mode == KTILER_EXEC_GRAPH_DAG || pol->exec_mode == KTILER_EXEC_GRAPH_WAVE) fold_dag_discards(P);
   } catch (const std::bad_alloc&) {
     delete P;
     return fail(KTILER_E_NOMEM, "host allocation failed while planning");
@@ -1529,9 +1521,10 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
       if (s) return s;
       break;
     }
-    case KTILER_EXEC_GRAPH_DAG: {
+    case KTILER_EXEC_GRAPH_DAG:
+    case KTILER_EXEC_GRAPH_WAVE: {
       if (!p->exec) {
-        if (p->has_custom) return fail(KTILER_E_UNSUPPORTED, "GRAPH_DAG runs built-in ops only");
+        if (p->has_custom) return fail(KTILER_E_UNSUPPORTED, "GRAPH_DAG / GRAPH_WAVE run built-in ops only");
         cudaGraph_t gr = nullptr;
         ktiler_status s = build_dag(p, &gr);
         if (s) return s;

@@ -202,16 +202,26 @@ __device__ __forceinline__ void stage_issue(int op, const DBuf& in, const Tile& 
 // is the whole staged window (stage_geo at full tile size), so out-of-image rows/columns
 // of a halo come back zero-filled and are fixed by stage_fix (replicate).  box_bytes is the
 // full box (also for ragged edge tiles, whose extra bytes are ignored).
+// evict_first: the tile's lines are L2 eviction candidates first (a streamed graph input).
 __device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map, unsigned box_bytes, const DBuf& in,
-                                                 const Tile& t, uint8_t* sm, uint64_t* m) {
+                                                 const Tile& t, uint8_t* sm, uint64_t* m, bool evict_first = false) {
   const StageGeo g = stage_geo(op, in, t);
   mbar_arrive_expect(m, box_bytes);
   const int x = (int)(g.xb0 >> 2), y = (int)g.ry0, z = (int)t.z;
-  asm volatile(
-      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
-          smem_u32(sm)),
-      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(m))
-      : "memory");
+  if (evict_first) {
+    const uint64_t pol = policy_evict_first();
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, "
+        "%3, %4}], [%5], %6;" ::"r"(smem_u32(sm)),
+        "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(m)), "l"(pol)
+        : "memory");
+  } else {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::"r"(
+            smem_u32(sm)),
+        "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(m))
+        : "memory");
+  }
 }
 
 // After the copies landed (stencils only): replicate-fill the halo outside the image —

@@ -88,6 +88,14 @@ struct Graph {
   int64_t total_blocks = 0;
   bool finalized = false;
 
+  // Does any node write buffer b?  (false: a graph input)
+  bool written_by_node(int b) const {
+    for (auto& n : nodes)
+      for (auto& a : n.acc)
+        if (a.buf == b && a.mode == KTILER_WRITE) return true;
+    return false;
+  }
+
   ktiler_status finalize();  // validate + derive; idempotent
 
   PRect access_rect(int node, int acc, int64_t bx, int64_t by) const;

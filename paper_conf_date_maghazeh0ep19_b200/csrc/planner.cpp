@@ -48,7 +48,17 @@ struct Partitioner {
   Schedule& out;
   int64_t nfrag = 0;
 
-  Partitioner(const Graph& G, Schedule& o) : g(G), out(o) {}
+  std::vector<uint8_t> counted;  // per buffer: do its lines count against the budget
+
+  Partitioner(const Graph& G, Schedule& o, bool resident_only) : g(G), out(o) {
+    counted.assign(g.bufs.size(), 1);
+    if (resident_only) {  // only intermediates: written by one node and read by another
+      std::vector<uint8_t> w(g.bufs.size(), 0), r(g.bufs.size(), 0);
+      for (auto& n : g.nodes)
+        for (auto& a : n.acc) (a.mode == KTILER_WRITE ? w : r)[a.buf] = 1;
+      for (size_t b = 0; b < g.bufs.size(); ++b) counted[b] = w[b] && r[b];
+    }
+  }
 
   int node_of(int64_t gid) const {
     int v = 0;
@@ -71,6 +81,7 @@ struct Partitioner {
     if (budget_lines < 0) return;
     for (int a = 0; a < (int)g.nodes[v].acc.size(); ++a)
       g.for_each_line_range(v, a, bx, by, bz, [&](int buf, int64_t l0, int64_t l1) {
+        if (!counted[buf]) return;
         const int64_t base = g.bufs[buf].line0;
         auto& bm = bits[buf];
         for (int64_t l = l0 - base; l < l1 - base;) {
@@ -341,10 +352,11 @@ ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragmen
   double frac = pol.l2_fraction > 0 ? pol.l2_fraction : 1.0;
   out.budget = (int64_t)std::floor((double)cache_bytes * frac);
   bool force = (pol.flags & KTILER_PF_FORCE_MINIMAL) != 0;
+  const bool resident = (pol.flags & KTILER_PF_RESIDENT_BUDGET) != 0;
   switch (pol.kind) {
     case KTILER_FRAG_NONE: untiled(g, out); return KTILER_OK;
     case KTILER_FRAG_BUDGET: {
-      Partitioner p(g, out);
+      Partitioner p(g, out, resident);
       p.budget_lines = out.budget / 128;
       p.rows_cap = 0;
       p.force_minimal = force;
@@ -361,7 +373,7 @@ ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragmen
       int64_t rows = pol.rows;
       if (pol.kind == KTILER_FRAG_BALANCED) {
         Schedule tmp;
-        Partitioner p(g, tmp);
+        Partitioner p(g, tmp, resident);
         p.budget_lines = out.budget / 128;
         p.rows_cap = 0;
         p.force_minimal = force;
@@ -370,7 +382,7 @@ ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragmen
         rows = (leaf_rows + tmp.nfrag - 1) / std::max<int64_t>(1, tmp.nfrag);
       }
       if (rows < 1) return fail(KTILER_E_INVALID, "ROWS policy needs rows >= 1");
-      Partitioner p(g, out);
+      Partitioner p(g, out, resident);
       p.budget_lines = -1;
       p.rows_cap = rows * leaf_gx;
       p.force_minimal = true;

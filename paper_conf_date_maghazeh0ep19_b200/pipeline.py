@@ -17,17 +17,19 @@ block dependencies in closed form from the declared footprints.
 """
 from __future__ import annotations
 
+import json
+import os
 import struct
 
 from . import ktiler as K
 
 # op -> (tile w, tile h, threads per block) for the vector variant
 B200_GEOMETRY = {
-    "gray": (256, 32, 256),    # 512 items of 16 px; 24.6 KB staged rgb
+    "gray": (256, 32, 128),    # 512 items of 16 px (4 per thread); 24.6 KB staged rgb
     "blur": (256, 64, 128),    # 128 column strips x 8 rows; 19.6 KB staged halo tile
-    "down": (256, 32, 256),    # 512 items; 16 KB staged blur rows
+    "down": (256, 32, 128),    # 512 items (4 per thread); 16 KB staged blur rows
     "sobel": (256, 64, 256),   # 256 strips x 4 rows; 19 KB halo tile
-    "thresh": (256, 16, 256),  # 256 items; 16 KB staged f32
+    "thresh": (256, 16, 64),   # 256 items (4 per thread); 16 KB staged f32
 }
 
 
@@ -115,6 +117,8 @@ class Pipeline:
             raise ValueError("down2 needs even W and H (SURVEY A3)")
         self.W, self.H, self.F, self.T = W, H, frames, T
         geo = dict(B200_GEOMETRY)
+        if os.environ.get("KTILER_GEOMETRY"):  # experiments: JSON {node: [tw, th, threads]}
+            geo.update({k: tuple(v) for k, v in json.loads(os.environ["KTILER_GEOMETRY"]).items()})
         geo.update(geometry or {})
         self.geometry = geo
         b = _GraphBuilder(device, pitch_align, bases)

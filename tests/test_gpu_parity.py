@@ -97,6 +97,7 @@ MODES = [
     dict(exec_mode="dag", window=1),
     dict(exec_mode="dag", window=4),
     dict(exec_mode="chain"),
+    dict(exec_mode="wave"),
 ]
 POLICIES = [
     dict(kind="none"),
@@ -105,6 +106,7 @@ POLICIES = [
     dict(kind="rows", rows=1),
     dict(kind="rows", rows=3),
     dict(kind="balanced", cache_bytes=200 * 1024),
+    dict(kind="budget", cache_bytes=60 * 1024, resident_budget=True),
 ]
 
 
@@ -141,7 +143,7 @@ def test_replay_is_idempotent():
     """A plan executes many times (GRAPH replays, persistent epochs) with identical output."""
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
     W, H, F = 1024, 128, 1
-    for mode in ("graph", "persistent", "chain"):
+    for mode in ("graph", "persistent", "chain", "wave"):
         p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
         a = synth.uniform(1, W, H, F)
         b = synth.scene(2, W, H, F)
@@ -254,7 +256,7 @@ def test_trace_records(mode):
 
 
 @pytest.mark.parametrize("world", [2, 4])
-@pytest.mark.parametrize("mode", ["graph", "dag"])
+@pytest.mark.parametrize("mode", ["graph", "dag", "wave"])
 def test_strips_on_one_gpu(world, mode):
     """§8(e) strip path, GPU side: each rank's extended strip (owned rows + the halo the
     exchange delivers) through libktiler; concatenated owned masks == whole-image oracle."""
