@@ -69,6 +69,18 @@ def summarise(rec, launches, pix):
         gaps = starts[1:] - ends[:-1]
         out["launch_gap_us_median"] = round(float(np.median(gaps)) / 1e3, 2) if len(gaps) else 0.0
         out["launch_overlap_frac"] = round(float((gaps < 0).mean()), 3) if len(gaps) else 0.0
+        # per node: median launch span and median gap from the previous launch's end
+        lnode = np.array([launches[i][1] for i in order])
+        per_span, per_gap = {}, {}
+        for v in sorted(set(lnode.tolist())):
+            m = lnode == v
+            name = NODES[v] if 0 <= v < len(NODES) else "discard"
+            per_span[name] = round(float(np.median((ends - starts)[m])) / 1e3, 2)
+            gm = m[1:]
+            if gm.any():
+                per_gap[name] = round(float(np.median(gaps[gm])) / 1e3, 2)
+        out["node_launch_span_us"] = per_span
+        out["node_gap_before_us"] = per_gap
     for kind, name in ((3, "ready_to_computed"), (4, "publish")):
         kk = rec[rec["kind"] == kind]
         if len(kk):
