@@ -403,7 +403,7 @@ class Tiling:
     footprint_lines: list  # per fragment: |lines(newSubKBlks)|
 
 
-def cluster_tile(g: OGraph, tr: Trace, budget_bytes: int, cluster=None) -> Tiling:
+def cluster_tile(g: OGraph, tr: Trace, budget_bytes: int, cluster=None, et=None) -> Tiling:
     """Alg. 2 for the cluster ``cluster`` (default: all nodes).
 
     Readings: A11 CheckCacheConst counts |union of lines read or written by
@@ -414,9 +414,10 @@ def cluster_tile(g: OGraph, tr: Trace, budget_bytes: int, cluster=None) -> Tilin
     dependency set is inside toBeAssigned U assigned, iterated to a fixpoint; A15
     toBeAssigned accumulates across successful iterations and is emptied only at l.24; A16
     when no leaf block is left, newSubKBlks is committed; A17 one sub-kernel per node per
-    commit, in topological order, empty ones omitted; A18 l.23 -> INF.  Cost: the
-    performance tables are outside the hot path, so CO_i
-    here counts sub-kernels — it only matters for the INF signal.
+    commit, in topological order, empty ones omitted; A18 l.23 -> INF.  Cost (l.19):
+    ``et(v, n_blocks, hot)`` = the performance-table time of a sub-kernel of node v with n
+    blocks, hot iff one of v's producers is in the cluster; without ``et``
+    CO_i counts sub-kernels (it then only matters for the INF signal).
     """
     nodes = list(range(len(g.nodes))) if cluster is None else sorted(cluster)
     in_cluster = set(nodes)
@@ -492,7 +493,10 @@ def cluster_tile(g: OGraph, tr: Trace, budget_bytes: int, cluster=None) -> Tilin
             if newSub[v]:
                 T.append((v, sorted(g.block_of(b)[1] for b in newSub[v])))
                 frag.append(nfrag)
-                CO += 1
+                if et is None:
+                    CO += 1
+                else:  # l.19: ET(subKer_v, C_i, perfTables)
+                    CO += et(v, len(newSub[v]), any(p in in_cluster for p in g.producers(v)))
                 assigned.update(newSub[v])
                 changed = True
         if changed:
@@ -543,6 +547,105 @@ def cluster_tile(g: OGraph, tr: Trace, budget_bytes: int, cluster=None) -> Tilin
             newSub = {v: set() for v in nodes}
             new_lines = 0
     return Tiling(T, frag, CO, fps)
+
+
+# ---------------------------------------------------------------------------------------
+# O-13: Alg. 1 Application Tiling with performance tables
+# ---------------------------------------------------------------------------------------
+def et_lookup(table, n: int, hot: bool) -> float:
+    """Performance-table lookup ("for the missing points, the duration is
+    obtained by interpolation"; reading A35): ``table`` = (block counts, cold ms, hot ms);
+    linear between points, the first point's time below the table, the last point's
+    per-block rate above it."""
+    ns, cold, hot_t = table
+    t = hot_t if hot else cold
+    if n <= ns[0]:
+        return t[0]
+    for k in range(1, len(ns)):
+        if n <= ns[k]:
+            return t[k - 1] + (t[k] - t[k - 1]) * (n - ns[k - 1]) / (ns[k] - ns[k - 1])
+    return t[-1] * n / ns[-1]
+
+
+def quotient_is_acyclic(edges, cluster_of) -> bool:
+    """A partition is valid iff its clusters can be totally ordered with no back-dependency
+    (PAPER.md:247–257): the graph of clusters (edges between different clusters) is
+    acyclic."""
+    nodes = set(cluster_of.values())
+    adj = {c: set() for c in nodes}
+    for u, v in edges:
+        if cluster_of[u] != cluster_of[v]:
+            adj[cluster_of[u]].add(cluster_of[v])
+    state = {}
+
+    def dfs(c):
+        state[c] = 1
+        for d in adj[c]:
+            if state.get(d) == 1 or (d not in state and not dfs(d)):
+                return False
+        state[c] = 2
+        return True
+    return all(c in state or dfs(c) for c in nodes)
+
+
+def application_tiling(g: OGraph, tr: Trace, budget_bytes: int, tables: dict, weights: dict, thld: float):
+    """Alg. 1, line by line.  ``tables[v]`` = performance table of node v
+    (see et_lookup); ``weights[(u, v)]`` = edge weight (None: derived as the time v saves
+    when that input is cached, ET_cold(N) - ET_hot(N)).  Reading A22: weight
+    > thld strict; ties by (src, dst); an edge whose ends already share a cluster is dropped.
+    Returns (clusters in execution order, their costs, schedule [(node, blocks, cluster)])."""
+    n = len(g.nodes)
+    et = lambda v, k, hot: et_lookup(tables[v], k, hot)  # noqa: E731
+    P = {i: [i] for i in range(n)}  # l.1–5: C_i = {v_i}
+    T = {i: None for i in range(n)}  # None = the kernel untiled (T_i = {kernel(v_i)})
+    CO = {i: et(i, g.nblocks(i), False) for i in range(n)}  # kerExeTimes
+    cluster_of = {i: i for i in range(n)}
+    edges = [(u, v) for v in range(n) for u in g.producers(v)]
+    w = {}
+    for (u, v) in edges:
+        wv = weights.get((u, v))
+        w[(u, v)] = et(v, g.nblocks(v), False) - et(v, g.nblocks(v), True) if wv is None else wv
+    cand = sorted([e for e in edges if w[e] > thld], key=lambda e: (-w[e], e[0], e[1]))  # l.6–7
+    eix = 0
+    while eix < len(cand):  # l.8
+        u, v = cand[eix]  # l.9
+        a, b = cluster_of[u], cluster_of[v]  # l.10
+        if a == b:
+            cand.pop(eix)
+            eix = 0
+            continue
+        merged = sorted(P[a] + P[b])  # l.11 (node ids are in topological order)
+        tmp_of = dict(cluster_of)  # l.12
+        for x in P[b]:
+            tmp_of[x] = a
+        if quotient_is_acyclic(edges, tmp_of):  # l.13
+            til = cluster_tile(g, tr, budget_bytes, cluster=merged, et=et)  # l.14
+            if til.cost < CO[a] + CO[b]:  # l.15
+                cluster_of = tmp_of
+                P[a] = merged
+                del P[b]
+                T[a], CO[a] = til, til.cost
+                del T[b], CO[b]
+            cand.pop(eix)  # l.16
+            eix = 0
+        else:
+            eix += 1  # l.18
+    # l.21–23: the clusters' tiling sequences in a topological order of the clusters
+    order, done = [], set()
+    while len(order) < len(P):
+        ready = [c for c in P if c not in done and all(cluster_of[p] in done or cluster_of[p] == c
+                                                       for x in P[c] for p in g.producers(x))]
+        c = min(ready, key=lambda c: P[c][0])
+        order.append(c)
+        done.add(c)
+    sched = []
+    for k, c in enumerate(order):
+        if T[c] is None:
+            v = P[c][0]
+            sched.append((v, g.blocks(v), k))
+        else:
+            sched.extend((v, blocks, k) for (v, blocks) in T[c].seq)
+    return [P[c] for c in order], [CO[c] for c in order], sched
 
 
 # ---------------------------------------------------------------------------------------

@@ -853,8 +853,16 @@ std::vector<std::vector<int>> dag_edges(const ktiler_plan_s* P) {
     return e;
   }
   std::vector<std::vector<int>> leaf_subs(S.nfrag), e(nsub);
-  for (int i = 0; i < nsub; ++i)
-    if (g.out_ch[S.subs[i].node].empty()) leaf_subs[S.subs[i].frag].push_back(i);
+  // leaf = no consumer inside the sub-kernel's cluster (Alg. 1 partitions; else the graph)
+  std::vector<std::vector<uint8_t>> member(S.clusters.size(), std::vector<uint8_t>(g.nodes.size(), 0));
+  for (size_t c = 0; c < S.clusters.size(); ++c)
+    for (int v : S.clusters[c]) member[c][v] = 1;
+  for (int i = 0; i < nsub; ++i) {
+    const int v = S.subs[i].node, c = S.subs[i].cluster;
+    bool leaf = true;
+    for (const kt::Chan& ch : g.out_ch[v]) leaf = leaf && !(c < (int)member.size() && member[c][ch.v]);
+    if (leaf) leaf_subs[S.subs[i].frag].push_back(i);
+  }
   std::vector<int> last_of_node(g.nodes.size(), -1);
   for (int i = 0; i < nsub; ++i) {
     e[i].assign(S.sub_deps[i].begin(), S.sub_deps[i].end());
@@ -1452,7 +1460,7 @@ ktiler_status ktiler_plan_get_subkernel(ktiler_plan_t p, int64_t i, ktiler_subke
   out->fragment = sk.frag;
   out->n_blocks = sk.nblocks;
   out->n_rects = (int32_t)sk.rects.size();
-  out->pad = 0;
+  out->cluster = sk.cluster;
   out->footprint_bytes = sk.footprint;
   if (rects)
     for (int32_t k = 0; k < cap && k < (int32_t)sk.rects.size(); ++k) {
@@ -1603,6 +1611,166 @@ ktiler_status ktiler_execute_host(ktiler_plan_t p, const ktiler_host_copy* in, i
     s = copy(outc[i], false);
     if (s) return s;
   }
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_num_clusters(ktiler_plan_t p, int32_t* n) {
+  if (!p || !n) return fail(KTILER_E_INVALID, "NULL argument");
+  *n = (int32_t)p->s.clusters.size();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_plan_get_cluster(ktiler_plan_t p, int32_t i, int32_t* nodes, int32_t cap, int32_t* n_nodes,
+                                      double* cost_ms) {
+  if (!p || !n_nodes) return fail(KTILER_E_INVALID, "NULL argument");
+  if (i < 0 || i >= (int32_t)p->s.clusters.size()) return fail(KTILER_E_INVALID, "cluster index out of range");
+  const std::vector<int>& c = p->s.clusters[i];
+  *n_nodes = (int32_t)c.size();
+  if (nodes)
+    for (int32_t k = 0; k < cap && k < (int32_t)c.size(); ++k) nodes[k] = c[k];
+  if (cost_ms) *cost_ms = p->s.cluster_cost[i];
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_calibrate(ktiler_graph_t gh, int32_t node, int32_t npts, const int64_t* nb, int32_t reps,
+                               double* ms_cold, double* ms_hot) {
+  if (!gh || !nb || !ms_cold || !ms_hot || npts < 1 || reps < 1) return fail(KTILER_E_INVALID, "bad argument");
+  kt::Graph* G = kt::graph_of(gh);
+  ktiler_status s = G->finalize();
+  if (s) return s;
+  if (node < 0 || node >= (int)G->nodes.size()) return fail(KTILER_E_INVALID, "node out of range");
+  if (G->nodes[node].op == KTILER_OP_CUSTOM) return fail(KTILER_E_UNSUPPORTED, "calibration runs built-in ops only");
+  ktiler_plan_s P;  // launch context (STREAM semantics)
+  P.g = *G;
+  P.pol.exec_mode = KTILER_EXEC_STREAM;
+  cudaError_t e = cudaGetDevice(&P.device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  int l2 = 0;
+  cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, P.device);
+  const size_t flush_bytes = (size_t)std::max(l2, 1 << 20) * 2;
+  void* flush = nullptr;
+  if ((e = cudaMalloc(&flush, flush_bytes)) != cudaSuccess) return cuda_fail(e, "cudaMalloc (L2 flush)");
+  cudaStream_t st = nullptr;
+  cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  const kt::Graph& g = P.g;
+  const kt::Node& n = g.nodes[node];
+  // the first k blocks of a node in (x, y, z) order as at most 3 rects
+  auto first_rects = [](const kt::Node& v, int64_t k) {
+    std::vector<kt::Rect6> r;
+    const int64_t gx = v.gx(), gy = v.gy(), per = gx * gy;
+    const int64_t fz = k / per, rem = k % per, rows = rem / gx, tail = rem % gx;
+    if (fz) r.push_back({0, 0, 0, (int32_t)gx, (int32_t)gy, (int32_t)fz});
+    if (rows) r.push_back({0, 0, (int32_t)fz, (int32_t)gx, (int32_t)rows, (int32_t)fz + 1});
+    if (tail) r.push_back({0, (int32_t)rows, (int32_t)fz, (int32_t)tail, (int32_t)rows + 1, (int32_t)fz + 1});
+    return r;
+  };
+  // device-side spans (first CTA start -> last CTA end) through the tracer
+  const int64_t tcap = 1 << 18;
+  void* tmem = nullptr;
+  if ((e = cudaMalloc(&tmem, (size_t)tcap * sizeof(ktiler_trace_record) + 256)) != cudaSuccess)
+    return cuda_fail(e, "cudaMalloc (calibration trace)");
+  TraceBuf tb{(ktiler_trace_record*)tmem, (unsigned long long*)((char*)tmem + (size_t)tcap * sizeof(ktiler_trace_record)),
+              tcap};
+  std::vector<ktiler_trace_record> rec;
+  auto read_span = [&](uint64_t id, uint64_t* t0, uint64_t* t1) -> bool {  // after a sync
+    unsigned long long cnt = 0;
+    cudaMemcpy(&cnt, tb.n, sizeof(cnt), cudaMemcpyDeviceToHost);
+    const int64_t k = std::min<int64_t>((int64_t)cnt, tcap);
+    rec.resize((size_t)k);
+    if (k) cudaMemcpy(rec.data(), tb.rec, (size_t)k * sizeof(ktiler_trace_record), cudaMemcpyDeviceToHost);
+    *t0 = ~0ull;
+    *t1 = 0;
+    for (auto& r : rec)
+      if (r.kind == 0 && r.id == id) {
+        *t0 = std::min(*t0, r.t0_ns);
+        *t1 = std::max(*t1, r.t1_ns);
+      }
+    return *t1 > 0;
+  };
+  auto launch_rects = [&](int v, const std::vector<kt::Rect6>& rects, int64_t trace_id, int times = 1) -> ktiler_status {
+    kt::SubKernel sk;
+    sk.node = v;
+    sk.rects = rects;
+    for (auto& q : rects) sk.nblocks += q.count();
+    ktiler_plan_s Q;
+    Q.g = g;
+    Q.pol.exec_mode = KTILER_EXEC_STREAM;
+    Q.device = P.device;
+    Q.s.subs.push_back(sk);
+    Q.s.discards.resize(1);
+    Q.s.nfrag = 1;
+    build_launches(&Q);
+    for (auto& L : Q.launches) {
+      if (L.node >= 0 && !L.n->scalar && L.kp.stage_bytes) {
+        L.n = &Q.g.nodes[L.node];
+        L.kp.use_tmap = make_tmap(Q.g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
+      }
+      if (trace_id >= 0) {
+        L.kp.tb = tb;
+        L.kp.lid = trace_id;
+      }
+    }
+    ktiler_status r = enqueue(&Q, st);
+    for (int k = 1; k < times && !r; ++k) {  // back to back: no host work in between
+      for (auto& L : Q.launches) ++L.kp.lid;
+      r = enqueue(&Q, st);
+    }
+    return r;
+  };
+  std::vector<double> ts;
+  ktiler_status rs = KTILER_OK;
+  // inter-launch gap of back-to-back launches (last CTA end -> next first CTA start):
+  // every sub-kernel of a replayed schedule pays it once ("inter-launch gap")
+  double gap_ms = 0;
+  {
+    const std::vector<kt::Rect6> one = first_rects(n, std::min<int64_t>(n.nblocks, n.gx()));
+    std::vector<double> gaps;
+    for (int r = 0; r < reps + 1 && !rs; ++r) {
+      cudaMemsetAsync(tb.n, 0, sizeof(unsigned long long), st);
+      rs = launch_rects(node, one, 2, 2);  // trace ids 2 and 3
+      cudaStreamSynchronize(st);
+      uint64_t a0, a1, b0, b1;
+      if (r && read_span(2, &a0, &a1) && read_span(3, &b0, &b1) && b0 > a1) gaps.push_back((double)(b0 - a1) * 1e-6);
+    }
+    std::sort(gaps.begin(), gaps.end());
+    gap_ms = gaps.empty() ? 0 : gaps[gaps.size() / 2];
+  }
+  for (int k = 0; k < npts && !rs; ++k) {
+    const int64_t m = std::min<int64_t>(std::max<int64_t>(1, nb[k]), n.nblocks);
+    const std::vector<kt::Rect6> rects = first_rects(n, m);
+    // producer blocks the first m blocks read: per channel, the bounding block range
+    std::vector<std::pair<int, std::vector<kt::Rect6>>> prod;
+    for (const kt::Chan& c : g.in_ch[node]) {
+      std::vector<kt::Rect6> pr;
+      for (auto& q : rects) {
+        kt::BRange a = g.producers(c, q.x0, q.y0), b = g.producers(c, q.x1 - 1, q.y1 - 1);
+        pr.push_back({(int32_t)a.x0, (int32_t)a.y0, q.z0, (int32_t)b.x1, (int32_t)b.y1, q.z1});
+      }
+      prod.push_back({c.u, pr});
+    }
+    for (int hot = 0; hot < 2 && !rs; ++hot) {
+      ts.clear();
+      for (int r = 0; r < reps + 1 && !rs; ++r) {  // +1: untimed warm-up
+        cudaMemsetAsync(flush, r & 0xFF, flush_bytes, st);
+        if (hot)
+          for (auto& pp : prod)
+            if (!rs) rs = launch_rects(pp.first, pp.second, -1);
+        cudaMemsetAsync(tb.n, 0, sizeof(unsigned long long), st);
+        if (!rs) rs = launch_rects(node, rects, 1);
+        cudaStreamSynchronize(st);
+        uint64_t t0, t1;
+        if (r && read_span(1, &t0, &t1)) ts.push_back((double)(t1 - t0) * 1e-6 + gap_ms);
+      }
+      std::sort(ts.begin(), ts.end());
+      (hot ? ms_hot : ms_cold)[k] = ts.empty() ? 0 : ts[ts.size() / 2];
+    }
+  }
+  cudaFree(tmem);
+  cudaStreamDestroy(st);
+  cudaFree(flush);
+  if (rs) return rs;
+  if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "calibration");
+  kt::clear_error();
   return KTILER_OK;
 }
 

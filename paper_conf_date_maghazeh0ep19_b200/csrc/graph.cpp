@@ -346,6 +346,23 @@ ktiler_status ktiler_add_edge(ktiler_graph_t g, int32_t src, int32_t dst, int32_
   return KTILER_OK;
 }
 
+ktiler_status ktiler_set_perf_table(ktiler_graph_t g, int32_t node, int32_t npts, const int64_t* nb, const double* cold,
+                                    const double* hot) {
+  if (!g || !nb || !cold || !hot) return fail(KTILER_E_INVALID, "NULL argument");
+  if (node < 0 || node >= (int)g->g.nodes.size()) return fail(KTILER_E_INVALID, "node out of range");
+  if (npts < 1) return fail(KTILER_E_INVALID, "a performance table needs at least one point");
+  for (int k = 0; k < npts; ++k) {
+    if (nb[k] < 1 || (k && nb[k] <= nb[k - 1])) return fail(KTILER_E_INVALID, "block counts must be positive and increasing");
+    if (!(cold[k] >= 0) || !(hot[k] >= 0)) return fail(KTILER_E_INVALID, "times must be >= 0");
+  }
+  Node& n = g->g.nodes[node];
+  n.perf_n.assign(nb, nb + npts);
+  n.perf_cold.assign(cold, cold + npts);
+  n.perf_hot.assign(hot, hot + npts);
+  clear_error();
+  return KTILER_OK;
+}
+
 ktiler_status ktiler_graph_block_deps(ktiler_graph_t g, int32_t node, int32_t bx, int32_t by, int32_t bz, int32_t* out,
                                       int64_t cap, int64_t* n) {
   if (!g || !n) return fail(KTILER_E_INVALID, "NULL argument");

@@ -48,6 +48,22 @@ struct Node {
   int64_t gid0 = 0;  // first global block id
   float T = 200.f;
   bool scalar = false;  // one thread per pixel variant
+  // performance table: execution time (ms) of a sub-kernel of perf_n[k]
+  // blocks with its input cold (HBM) / hot (produced by tiling, in L2); empty = none
+  std::vector<int64_t> perf_n;
+  std::vector<double> perf_cold, perf_hot;
+  // ET lookup (A35): piecewise linear in the block count, the first point's time below
+  // the table, the last point's per-block rate above it
+  double et(int64_t n, bool hot) const {
+    const std::vector<double>& t = hot ? perf_hot : perf_cold;
+    const size_t m = perf_n.size();
+    if (m == 0) return (double)n;
+    if (n <= perf_n[0]) return t[0];
+    for (size_t k = 1; k < m; ++k)
+      if (n <= perf_n[k])
+        return t[k - 1] + (t[k] - t[k - 1]) * (double)(n - perf_n[k - 1]) / (double)(perf_n[k] - perf_n[k - 1]);
+    return t[m - 1] * (double)n / (double)perf_n[m - 1];
+  }
   int64_t gx() const { return grid[0]; }
   int64_t gy() const { return grid[1]; }
   int64_t gz() const { return grid[2]; }
@@ -132,6 +148,7 @@ struct Rect6 {
 
 struct SubKernel {
   int32_t node = 0, frag = 0;
+  int32_t cluster = 0;    // Alg. 1 cluster (0 when the whole graph is one cluster)
   int64_t nblocks = 0;
   int64_t footprint = 0;  // bytes, of the fragment
   std::vector<Rect6> rects;
@@ -158,6 +175,10 @@ struct Schedule {
   // that reads the dying blocks (a discard may only run after all of them) — GRAPH_DAG
   std::vector<std::vector<int32_t>> sub_deps;
   std::vector<std::vector<int32_t>> discard_readers;
+  // Alg. 1: the clusters in execution order and their costs (ms, from
+  // the performance tables); one cluster of every node for the other policies
+  std::vector<std::vector<int>> clusters;
+  std::vector<double> cluster_cost;
 };
 
 ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out);

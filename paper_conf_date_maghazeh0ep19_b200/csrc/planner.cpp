@@ -19,6 +19,8 @@
 // Scale: O(blocks x deps) time and one byte per block + one bit per memory line, so
 // 64 x 8K frames (2.6 M blocks) or a 65536^2 image plan in well under a second.
 #include <algorithm>
+#include <climits>
+#include <cstdint>
 #include <chrono>
 #include <cmath>
 
@@ -49,8 +51,13 @@ struct Partitioner {
   int64_t nfrag = 0;
 
   std::vector<uint8_t> counted;  // per buffer: do its lines count against the budget
+  std::vector<uint8_t> in_c;     // per node: member of the cluster being tiled
+  int32_t cluster_id = 0;
+  double cost = 0;               // CO_i (PAPER.md:305 l.19): sum of ET over committed sub-kernels
+  bool use_et = false;
 
   Partitioner(const Graph& G, Schedule& o, bool resident_only) : g(G), out(o) {
+    in_c.assign(g.nodes.size(), 1);
     counted.assign(g.bufs.size(), 1);
     if (resident_only) {  // only intermediates: written by one node and read by another
       std::vector<uint8_t> w(g.bufs.size(), 0), r(g.bufs.size(), 0);
@@ -118,6 +125,7 @@ struct Partitioner {
       int64_t bx, by, bz;
       coords(v, gid, bx, by, bz);
       for (const Chan& c : g.in_ch[v]) {
+        if (!in_c[c.u]) continue;  // intra-cluster dependencies only (A13)
         BRange r = g.producers(c, bx, by);
         for (int64_t y = r.y0; y < r.y1; ++y)
           for (int64_t x = r.x0; x < r.x1; ++x) {
@@ -134,6 +142,7 @@ struct Partitioner {
   bool deps_covered(int v, int64_t bx, int64_t by, int64_t bz) const {
     bool any = false;
     for (const Chan& c : g.in_ch[v]) {
+      if (!in_c[c.u]) continue;
       BRange r = g.producers(c, bx, by);
       for (int64_t y = r.y0; y < r.y1; ++y)
         for (int64_t x = r.x0; x < r.x1; ++x) {
@@ -153,6 +162,7 @@ struct Partitioner {
       int64_t px, py, pz;
       coords(u, gid, px, py, pz);
       for (const Chan& c : g.out_ch[u]) {
+        if (!in_c[c.v]) continue;
         BRange r = g.consumers(c, px, py);
         for (int64_t y = r.y0; y < r.y1; ++y)
           for (int64_t x = r.x0; x < r.x1; ++x) {
@@ -187,7 +197,13 @@ struct Partitioner {
       SubKernel sk;
       sk.node = v;
       sk.frag = (int32_t)nfrag;
+      sk.cluster = cluster_id;
       sk.nblocks = (int64_t)per[v].size();
+      if (use_et) {  // l.19: ET(subKer_v, C_i, perfTables) — hot iff an input is produced in the cluster
+        bool hot = false;
+        for (const Chan& c : g.in_ch[v]) hot = hot || in_c[c.u];
+        cost += g.nodes[v].et(sk.nblocks, hot);
+      }
       sk.footprint = fp_lines * 128;
       to_rects(v, per[v], sk.rects);
       out.subs.push_back(std::move(sk));
@@ -254,16 +270,26 @@ struct Partitioner {
   ktiler_status run() {
     const int nn = (int)g.nodes.size();
     st.assign(g.total_blocks, 0);
+    int64_t cluster_blocks = 0;
+    for (int v = 0; v < nn; ++v) {
+      if (in_c[v]) cluster_blocks += g.nodes[v].nblocks;
+      else std::fill(st.begin() + g.nodes[v].gid0, st.begin() + g.nodes[v].gid0 + g.nodes[v].nblocks, (uint8_t)2);
+    }
+    nfrag = out.nfrag;  // fragments are numbered across clusters
     if (budget_lines >= 0) {
       bits.resize(g.bufs.size());
       for (size_t b = 0; b < g.bufs.size(); ++b) bits[b].assign((g.bufs[b].nlines + 63) / 64, 0);
     }
     leaf_node.assign(nn, 0);
-    for (int v = 0; v < nn; ++v)
-      if (g.out_ch[v].empty()) {
+    for (int v : g.topo) {  // leaves of the cluster: no consumer inside it
+      if (!in_c[v]) continue;
+      bool leaf = true;
+      for (const Chan& c : g.out_ch[v]) leaf = leaf && !in_c[c.v];
+      if (leaf) {
         leaf_node[v] = 1;
         leaves.push_back(v);
       }
+    }
     cursor.assign(nn, 0);
     scan.assign(nn, 0);
     int64_t assigned = 0;
@@ -278,6 +304,7 @@ struct Partitioner {
       if (picked.empty()) {
         // A16b: blocks no leaf block depends on act as bottom blocks, last node first
         for (int v : rev) {
+          if (!in_c[v]) continue;
           const Node& n = g.nodes[v];
           for (int64_t l = 0; l < n.nblocks; ++l)
             if (st[n.gid0 + l] == 0) {
@@ -289,7 +316,7 @@ struct Partitioner {
       }
       if (picked.empty()) {
         // A16: every block is in assigned U toBeAssigned -> commit newSubKBlks
-        if (new_len == 0 && assigned < g.total_blocks) return fail(KTILER_E_UNTILEABLE, "internal: nothing to commit");
+        if (new_len == 0 && assigned < cluster_blocks) return fail(KTILER_E_UNTILEABLE, "internal: nothing to commit");
         if (new_len) commit(new_len, new_lines);
         break;
       }
@@ -345,6 +372,170 @@ static void untiled(const Graph& g, Schedule& out) {
   out.max_footprint = fp;
 }
 
+// Alg. 1 Application Tiling.  Starts from singleton
+// clusters whose cost is the kernel's default (untiled, cold-input) execution time, takes
+// the candidate edges (weight > thld; weight < 0 = derived from the performance tables as
+// the time the consumer saves when that input is cached), highest weight
+// first (ties: src id, dst id), merges the two clusters at the ends of the current edge
+// when the partition stays valid (the quotient graph of clusters is acyclic),
+// tiles the merged cluster with Alg. 2 and keeps it iff CO_m < CO_a + CO_b; the edge is
+// then removed and the scan restarts at the top (l.16), an invalid merge moves to the
+// next edge (l.18).  The schedule concatenates the clusters' tiling sequences in a
+// topological order of the clusters; an unmerged node runs untiled (l.2: T_i = kernel).
+static const double ALG1_INF = 1e300;
+
+static bool quotient_acyclic(const Graph& g, const std::vector<int>& cl) {
+  const int nn = (int)g.nodes.size();
+  std::vector<std::vector<int>> adj(nn);
+  std::vector<int> indeg(nn, 0), present(nn, 0);
+  for (int v = 0; v < nn; ++v) present[cl[v]] = 1;
+  for (int v = 0; v < nn; ++v)
+    for (const Chan& c : g.out_ch[v])
+      if (cl[c.u] != cl[c.v]) {
+        adj[cl[c.u]].push_back(cl[c.v]);
+        ++indeg[cl[c.v]];
+      }
+  std::vector<int> q;
+  int seen = 0, total = 0;
+  for (int c = 0; c < nn; ++c)
+    if (present[c]) {
+      ++total;
+      if (!indeg[c]) q.push_back(c);
+    }
+  while (!q.empty()) {
+    int c = q.back();
+    q.pop_back();
+    ++seen;
+    for (int d : adj[c])
+      if (--indeg[d] == 0) q.push_back(d);
+  }
+  return seen == total;
+}
+
+static ktiler_status alg1(Graph& g, int64_t budget_lines, double thld, bool resident, Schedule& out) {
+  const int nn = (int)g.nodes.size();
+  for (int v = 0; v < nn; ++v)
+    if (g.nodes[v].perf_n.empty())
+      return fail(KTILER_E_STATE, "KTILER_FRAG_ALG1 needs a performance table for every node (ktiler_set_perf_table)");
+  std::vector<int> pos(nn);
+  for (int i = 0; i < nn; ++i) pos[g.topo[i]] = i;
+  std::vector<int> cl(nn);
+  std::vector<std::vector<int>> members(nn);
+  std::vector<double> CO(nn);
+  for (int v = 0; v < nn; ++v) {  // l.1–5
+    cl[v] = v;
+    members[v] = {v};
+    CO[v] = g.nodes[v].et(g.nodes[v].nblocks, false);
+  }
+  struct Cand {
+    double w;
+    int src, dst;
+  };
+  std::vector<Cand> cand;  // l.6–7
+  for (const Edge& e : g.edges) {
+    const Node& d = g.nodes[e.dst];
+    const double w = e.w >= 0 ? (double)e.w : d.et(d.nblocks, false) - d.et(d.nblocks, true);
+    if (w > thld) cand.push_back({w, e.src, e.dst});
+  }
+  std::stable_sort(cand.begin(), cand.end(), [](const Cand& a, const Cand& b) {
+    if (a.w != b.w) return a.w > b.w;
+    if (a.src != b.src) return a.src < b.src;
+    return a.dst < b.dst;
+  });
+  auto tile = [&](const std::vector<int>& mem, int32_t cid, Schedule& into, double* cost) -> ktiler_status {
+    Partitioner p(g, into, resident);
+    std::fill(p.in_c.begin(), p.in_c.end(), (uint8_t)0);
+    for (int v : mem) p.in_c[v] = 1;
+    p.budget_lines = budget_lines;
+    p.rows_cap = 0;
+    p.force_minimal = false;
+    p.use_et = true;
+    p.cluster_id = cid;
+    ktiler_status st = p.run();
+    *cost = st ? ALG1_INF : p.cost;
+    return st;
+  };
+  size_t eix = 0;
+  while (eix < cand.size()) {  // l.8
+    const int a = cl[cand[eix].src], b = cl[cand[eix].dst];  // l.10
+    if (a == b) {  // both ends already in one cluster (A22)
+      cand.erase(cand.begin() + (long)eix);
+      eix = 0;
+      continue;
+    }
+    std::vector<int> merged = members[a];  // l.11 MergeOrder: topological order
+    merged.insert(merged.end(), members[b].begin(), members[b].end());
+    std::sort(merged.begin(), merged.end(), [&](int x, int y) { return pos[x] < pos[y]; });
+    std::vector<int> cl2 = cl;  // l.12–13
+    for (int v : members[b]) cl2[v] = a;
+    if (!quotient_acyclic(g, cl2)) {
+      ++eix;  // l.18
+      continue;
+    }
+    Schedule tmp;  // l.14
+    double com = 0;
+    tile(merged, 0, tmp, &com);
+    if (com < CO[a] + CO[b]) {  // l.15
+      cl = cl2;
+      members[a] = merged;
+      members[b].clear();
+      CO[a] = com;
+    }
+    cand.erase(cand.begin() + (long)eix);  // l.16
+    eix = 0;
+  }
+  kt::clear_error();
+  // l.21–24: clusters in a topological order of the quotient graph
+  std::vector<int> order;
+  {
+    std::vector<int> indeg(nn, 0);
+    std::vector<std::vector<int>> adj(nn);
+    for (int v = 0; v < nn; ++v)
+      for (const Chan& c : g.out_ch[v])
+        if (cl[c.u] != cl[c.v]) {
+          adj[cl[c.u]].push_back(cl[c.v]);
+          ++indeg[cl[c.v]];
+        }
+    std::vector<int> ready;
+    for (int c = 0; c < nn; ++c)
+      if (!members[c].empty() && !indeg[c]) ready.push_back(c);
+    while (!ready.empty()) {  // smallest topological position first (deterministic)
+      auto it = std::min_element(ready.begin(), ready.end(),
+                                 [&](int x, int y) { return pos[members[x][0]] < pos[members[y][0]]; });
+      const int c = *it;
+      ready.erase(it);
+      order.push_back(c);
+      for (int d : adj[c])
+        if (--indeg[d] == 0) ready.push_back(d);
+    }
+  }
+  for (int c : order) {
+    const int32_t cid = (int32_t)out.clusters.size();
+    if (members[c].size() == 1) {
+      const int v = members[c][0];
+      const Node& n = g.nodes[v];
+      SubKernel sk;
+      sk.node = v;
+      sk.frag = (int32_t)out.nfrag++;
+      sk.cluster = cid;
+      sk.nblocks = n.nblocks;
+      int64_t fp = 0;
+      for (auto& a : n.acc) fp += g.bufs[a.buf].nlines * 128;
+      sk.footprint = fp;
+      sk.rects.push_back({0, 0, 0, (int32_t)n.gx(), (int32_t)n.gy(), (int32_t)n.gz()});
+      out.subs.push_back(sk);
+      out.max_footprint = std::max(out.max_footprint, fp);
+    } else {
+      double cost = 0;
+      ktiler_status st = tile(members[c], cid, out, &cost);
+      if (st) return st;
+    }
+    out.clusters.push_back(members[c]);
+    out.cluster_cost.push_back(CO[c]);
+  }
+  return KTILER_OK;
+}
+
 ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out) {
   ktiler_status s = g.finalize();
   if (s) return s;
@@ -353,7 +544,13 @@ ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragmen
   out.budget = (int64_t)std::floor((double)cache_bytes * frac);
   bool force = (pol.flags & KTILER_PF_FORCE_MINIMAL) != 0;
   const bool resident = (pol.flags & KTILER_PF_RESIDENT_BUDGET) != 0;
+  if (pol.kind != KTILER_FRAG_ALG1) {
+    std::vector<int> all(g.topo.begin(), g.topo.end());
+    out.clusters.push_back(all);
+    out.cluster_cost.push_back(0.0);
+  }
   switch (pol.kind) {
+    case KTILER_FRAG_ALG1: return alg1(g, out.budget / 128, pol.alg1_thld, resident, out);
     case KTILER_FRAG_NONE: untiled(g, out); return KTILER_OK;
     case KTILER_FRAG_BUDGET: {
       Partitioner p(g, out, resident);
@@ -432,6 +629,14 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
     std::sort(dep.begin(), dep.end());
     dep.erase(std::unique(dep.begin(), dep.end()), dep.end());
   }
+  // Lines are discarded only where tiling keeps them in L2: producer and last reader in
+  // the same cluster, and that cluster tiled into more than one fragment (an untiled
+  // intermediate has left L2 long before its last reader ends).
+  std::vector<int32_t> cf0(s.clusters.size() + 1, INT32_MAX), cf1(s.clusters.size() + 1, -1);
+  for (const SubKernel& sk : s.subs) {
+    cf0[sk.cluster] = std::min(cf0[sk.cluster], sk.frag);
+    cf1[sk.cluster] = std::max(cf1[sk.cluster], sk.frag);
+  }
   for (int u = 0; u < (int)g.nodes.size(); ++u) {
     const Node& n = g.nodes[u];
     const Access& w = n.acc[n.wacc];
@@ -454,7 +659,10 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
             rd.push_back(sc);
           }
       }
-      if (last >= 0) {
+      const int32_t own = sub_of[n.gid0 + l];
+      const int32_t c = own >= 0 ? s.subs[own].cluster : -1;
+      const bool tiled = c >= 0 && last >= 0 && s.subs[last].cluster == c && cf1[c] > cf0[c];
+      if (last >= 0 && tiled) {
         dead[last].push_back(l);
         auto& R = s.discard_readers[last];
         R.insert(R.end(), rd.begin(), rd.end());

@@ -18,14 +18,15 @@ OK, E_INVALID, E_CYCLE, E_UNTILEABLE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 
 BUF_INTERNAL = 1
 READ, WRITE = 1, 2
 OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM = range(6)
-FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE = range(4)
+FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1 = range(5)
 EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE = range(7)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL, PF_RESIDENT_BUDGET = 1, 2, 4, 8
 
 EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
               "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG, "chain": EXEC_GRAPH_CHAIN,
               "wave": EXEC_GRAPH_WAVE}
-FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE}
+FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE,
+              "alg1": FRAG_ALG1}
 
 
 SELFTEST_SQRT = 0
@@ -68,12 +69,12 @@ class KernelDesc(ctypes.Structure):
 class Policy(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("l2_fraction", ctypes.c_double), ("rows", ctypes.c_int64),
                 ("exec_mode", ctypes.c_int32), ("flags", ctypes.c_uint32), ("persistent_ctas", ctypes.c_int32),
-                ("pipeline_skew", ctypes.c_int32), ("window", ctypes.c_int32)]
+                ("pipeline_skew", ctypes.c_int32), ("window", ctypes.c_int32), ("alg1_thld", ctypes.c_double)]
 
 
 class SubKernelInfo(ctypes.Structure):
     _fields_ = [("node", ctypes.c_int32), ("fragment", ctypes.c_int32), ("n_blocks", ctypes.c_int64),
-                ("n_rects", ctypes.c_int32), ("pad", ctypes.c_int32), ("footprint_bytes", ctypes.c_int64)]
+                ("n_rects", ctypes.c_int32), ("cluster", ctypes.c_int32), ("footprint_bytes", ctypes.c_int64)]
 
 
 class PlanStats(ctypes.Structure):
@@ -98,7 +99,8 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_graph_block_deps", "ktiler_graph_block_lines", "ktiler_plan", "ktiler_plan_destroy",
            "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
            "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
-           "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest"]
+           "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest", "ktiler_plan_num_clusters",
+           "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate"]
 
 _LIB = None
 
@@ -136,6 +138,10 @@ def lib() -> ctypes.CDLL:
         "ktiler_trace_read": ([vp, vp, i64, P(i64)], st),
         "ktiler_plan_get_launch": ([vp, i64, P(i32), P(i32), P(i64)], st),
         "ktiler_selftest": ([i32, P(i64)], st),
+        "ktiler_plan_num_clusters": ([vp, P(i32)], st),
+        "ktiler_plan_get_cluster": ([vp, i32, P(i32), i32, P(i32), P(ctypes.c_double)], st),
+        "ktiler_set_perf_table": ([vp, i32, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double)], st),
+        "ktiler_calibrate": ([vp, i32, i32, P(i64), i32, P(ctypes.c_double), P(ctypes.c_double)], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -220,14 +226,28 @@ class Graph:
         _check(lib().ktiler_graph_block_lines(self._h, node, bx, by, bz, arr, n.value, ctypes.byref(n)))
         return list(arr[:n.value])
 
+    def set_perf_table(self, node: int, nblocks, ms_cold, ms_hot) -> None:
+        """Performance table of a node for the ALG1 policy."""
+        n = len(nblocks)
+        _check(lib().ktiler_set_perf_table(self._h, node, n, (ctypes.c_int64 * n)(*nblocks),
+                                           (ctypes.c_double * n)(*ms_cold), (ctypes.c_double * n)(*ms_hot)))
+
+    def calibrate(self, node: int, nblocks, reps: int = 5):
+        """Measure a node's performance table on the current device -> (cold, hot) lists (ms)."""
+        n = len(nblocks)
+        c, h = (ctypes.c_double * n)(), (ctypes.c_double * n)()
+        _check(lib().ktiler_calibrate(self._h, node, n, (ctypes.c_int64 * n)(*nblocks), reps, c, h))
+        return list(c), list(h)
+
     def plan(self, cache_bytes: int = 0, kind: str | int = "budget", l2_fraction: float = 1.0, rows: int = 1,
              exec_mode: str | int = "graph", discard: bool = False, pdl: bool = False, force_minimal: bool = False,
-             persistent_ctas: int = 0, skew: int = 0, window: int = 0, resident_budget: bool = False) -> "Plan":
+             persistent_ctas: int = 0, skew: int = 0, window: int = 0, resident_budget: bool = False,
+             alg1_thld: float = 0.0) -> "Plan":
         k = FRAG_KINDS[kind] if isinstance(kind, str) else kind
         m = EXEC_MODES[exec_mode] if isinstance(exec_mode, str) else exec_mode
         flags = (PF_DISCARD_DEAD if discard else 0) | (PF_PDL if pdl else 0) | (PF_FORCE_MINIMAL if force_minimal else 0) \
             | (PF_RESIDENT_BUDGET if resident_budget else 0)
-        pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew, window)
+        pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew, window, alg1_thld)
         h = ctypes.c_void_p()
         _check(lib().ktiler_plan(self._h, cache_bytes, ctypes.byref(pol), ctypes.byref(h)))
         return Plan(h, self)
@@ -270,9 +290,22 @@ class Plan:
             _check(lib().ktiler_plan_get_subkernel(self._h, i, ctypes.byref(info), None, 0))
             arr = (ctypes.c_int32 * (6 * max(1, info.n_rects)))()
             _check(lib().ktiler_plan_get_subkernel(self._h, i, ctypes.byref(info), arr, info.n_rects))
-            out.append({"node": info.node, "fragment": info.fragment, "n_blocks": info.n_blocks,
+            out.append({"node": info.node, "fragment": info.fragment, "n_blocks": info.n_blocks, "cluster": info.cluster,
                         "footprint_bytes": info.footprint_bytes,
                         "rects": [tuple(arr[6 * k:6 * k + 6]) for k in range(info.n_rects)]})
+        return out
+
+    def clusters(self):
+        """[(node ids, estimated cost ms)] in execution order (Alg. 1 partition)."""
+        n = ctypes.c_int32()
+        _check(lib().ktiler_plan_num_clusters(self._h, ctypes.byref(n)))
+        out = []
+        for i in range(n.value):
+            cnt, cost = ctypes.c_int32(), ctypes.c_double()
+            _check(lib().ktiler_plan_get_cluster(self._h, i, None, 0, ctypes.byref(cnt), ctypes.byref(cost)))
+            arr = (ctypes.c_int32 * max(1, cnt.value))()
+            _check(lib().ktiler_plan_get_cluster(self._h, i, arr, cnt.value, ctypes.byref(cnt), ctypes.byref(cost)))
+            out.append((list(arr[:cnt.value]), cost.value))
         return out
 
     def stats(self) -> dict:

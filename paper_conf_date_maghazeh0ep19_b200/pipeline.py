@@ -69,6 +69,7 @@ class _GraphBuilder:
         self.g = K.Graph()
         self.bufs = {}  # name -> (id, W, H, F, elem, pitch)
         self.nodes = {}
+        self.grids = {}
         self.pitch_align = pitch_align
         self.bases = bases or {}
 
@@ -92,6 +93,7 @@ class _GraphBuilder:
                dict(buf=did, mode=K.WRITE, ax=tw, ay=th)]
         nid = self.g.add_kernel(op, grid, block, acc, params)
         self.nodes[name] = nid
+        self.grids[name] = grid
         return nid
 
     def view(self, name):
@@ -140,10 +142,11 @@ class Pipeline:
                  params=struct.pack("f", T))
         n = b.nodes
         bu = b.bufs
-        b.g.add_edge(n["gray"], n["blur"], bu["gray"][0])
-        b.g.add_edge(n["blur"], n["down"], bu["blur"][0])
-        b.g.add_edge(n["down"], n["sobel"], bu["down"][0])
-        b.g.add_edge(n["sobel"], n["thresh"], bu["sob"][0])
+        # edge weights < 0: derived from the performance tables by Alg. 1 (include/ktiler.h)
+        b.g.add_edge(n["gray"], n["blur"], bu["gray"][0], -1.0)
+        b.g.add_edge(n["blur"], n["down"], bu["blur"][0], -1.0)
+        b.g.add_edge(n["down"], n["sobel"], bu["down"][0], -1.0)
+        b.g.add_edge(n["sobel"], n["thresh"], bu["sob"][0], -1.0)
         self.plan_obj = None
 
     @property
@@ -156,6 +159,26 @@ class Pipeline:
     def plan(self, cache_bytes: int = 0, **policy) -> K.Plan:
         self.plan_obj = self.b.g.plan(cache_bytes, **policy)
         return self.plan_obj
+
+    def calibrate(self, reps: int = 5, max_points: int = 8) -> dict:
+        """Self-calibrated performance tables on the current
+        device: each node's time for row bands of 1, 2, 4, ... block rows up to the whole
+        grid, input cold and hot (ktiler_calibrate), installed with ktiler_set_perf_table.
+        Returns {node name: (block counts, cold ms, hot ms)}."""
+        out = {}
+        for name in self.NODE_ORDER:
+            gx, gy, gz = self.b.grids[name]
+            total = gx * gy * gz
+            pts, k = [], gx
+            while k < total and len(pts) < max_points - 1:
+                pts.append(k)
+                k *= 4
+            pts.append(total)
+            nid = self.b.nodes[name]
+            cold, hot = self.graph.calibrate(nid, pts, reps)
+            self.graph.set_perf_table(nid, pts, cold, hot)
+            out[name] = (pts, cold, hot)
+        return out
 
     def run(self, stream: int | None = None) -> None:
         if self.plan_obj is None:
@@ -203,7 +226,7 @@ class Motivational:
         else:
             b.kernel("A", K.OP_GRAY, "in", "intm", B200_GEOMETRY["gray"][:2], B200_GEOMETRY["gray"][2])
             b.kernel("B", K.OP_DOWN2, "intm", "out", B200_GEOMETRY["down"][:2], B200_GEOMETRY["down"][2], scale=2)
-        b.g.add_edge(b.nodes["A"], b.nodes["B"], b.bufs["intm"][0])
+        b.g.add_edge(b.nodes["A"], b.nodes["B"], b.bufs["intm"][0], -1.0)
         self.plan_obj = None
 
     @property

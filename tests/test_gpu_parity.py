@@ -279,3 +279,23 @@ def test_selftest_sqrt_exhaustive():
     """The Sobel magnitude's fast sqrt equals __fsqrt_rn on every integer of its domain."""
     from paper_conf_date_maghazeh0ep19_b200 import ktiler
     assert ktiler.selftest(ktiler.SELFTEST_SQRT) == 0
+
+
+def test_alg1_calibrated_plan():
+    """§8(f) f1 on the device: self-calibrated performance tables (ktiler_calibrate), an
+    Alg. 1 plan from them, executed bit-exact; cold times grow with the block count."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 1024, 256, 2
+    rgb = synth.scene(31, W, H, F)
+    p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
+    p.view("rgb").copy_(torch.from_numpy(rgb))
+    tabs = p.calibrate(reps=2, max_points=4)
+    for name, (pts, cold, hot) in tabs.items():
+        assert len(pts) == len(cold) == len(hot) and all(t > 0 for t in cold + hot)
+        assert cold[-1] >= cold[0]
+    for mode in ("graph", "dag"):
+        plan = p.plan(64 * 1024, kind="alg1", exec_mode=mode, discard=True)
+        assert sorted(v for c, _ in plan.clusters() for v in c) == [0, 1, 2, 3, 4]
+        p.run()
+        torch.cuda.synchronize()
+        assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(rgb, T=40.0)["mask"])
