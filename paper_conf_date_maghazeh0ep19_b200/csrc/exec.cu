@@ -32,12 +32,12 @@ namespace {
 
 using ktd::DBuf;
 constexpr int MAXR = 4, MAXD = 8;
-constexpr int PCOMP_WARPS = 8;  // compute warps per persistent CTA (+ producer + publisher warp)
+constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+ producer + publisher warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
 constexpr int PERSIST_THREADS = PCOMP_THREADS + 64;
-constexpr int PSTAGES = 3;       // staging ring depth
-constexpr int MAXDEAD = 64;
-constexpr int PERSIST_MINB_DEFAULT = 2;
+constexpr int PSTAGES_MAX = 6;   // staging ring depth (slots that fit the CTA's share of smem)
+constexpr int PERSIST_MINB_DEFAULT = 3;
+constexpr int PMAX_NODES = 8;
 
 struct LRect {
   int32_t x0, y0, z0, x1, y1, z1;
@@ -347,6 +347,20 @@ __global__ void discard_kernel(const __grid_constant__ KParams p) {
 // ------------------------------------------------------------------------------------
 // persistent executor
 // ------------------------------------------------------------------------------------
+// One launch runs the whole schedule.  The schedule's sub-kernels are replayed as a
+// stream of tickets in a (skewed) total order that respects every dependency
+// (PAPER.md:271): a ticket is one block (tile) of a sub-kernel, or one chunk of a discard
+// list.  Ticket i belongs to CTA i mod G (static, no ticket atomics); the host lays each
+// CTA's tickets out contiguously so a warp fetches 32 of them with one coalesced load.
+// Synchronisation is per SUB-KERNEL, not per block: each sub-kernel (and each discard
+// list) is a "group" whose tickets may start once the completion counters of the groups
+// it depends on (Schedule::sub_deps, the block-level dependencies PAPER.md:173–193
+// aggregated per sub-kernel; for discards: every reader of the lines) have reached
+// epoch x their tile counts.  With the skewed order a consumer sub-kernel is issued about
+// one pipeline step after its producer, so the check almost never waits; and a CTA
+// re-checks only when its next ticket belongs to another group.
+// Deadlock-free: a group's dependencies have all their tickets earlier in the order, so
+// the smallest unfinished ticket is always runnable and its CTA reaches it.
 struct PNode {
   CUtensorMap tmap;  // input tile map (tensor TMA), valid if use_tmap
   uint32_t box_bytes;
@@ -355,261 +369,266 @@ struct PNode {
   DBuf in, out;
   int32_t op, scalar, tw, th;
   float T;
-  int32_t gx, gy;
-  int64_t flag0;
-  int32_t pu, disc_in;
-  int64_t rax, ray, rox, roy;
-  int32_t rhl, rhr, rht, rhb;
-  int64_t wax, way;
-  int32_t pgx, pgy;
-  int64_t pflag0;
-  const uint8_t* expect;  // per producer block: number of reader blocks
-  int64_t ptw, pth;       // producer output tile (for discards)
 };
 struct PCtrl {
-  unsigned int ticket, done, epoch, pad;
+  unsigned int done, epoch, pad0, pad1;
 };
-// Tile descriptor of ticket t: node (4 bits) | bz (12) | by (24) | bx (24).
-__host__ __device__ inline uint64_t pack_tile(uint64_t node, uint64_t bx, uint64_t by, uint64_t bz) {
-  return (node << 60) | (bz << 48) | (by << 24) | bx;
+struct PDep {
+  int32_t sub;       // counter index (= sub-kernel id)
+  uint32_t ntiles;   // its tiles per execute
+};
+struct PChunk {      // one discard ticket: lines [l0, l0 + n) of rect d (row-major, lpr per row)
+  int32_t d;
+  int32_t n;
+  int64_t l0;
+};
+// Ticket descriptor: kind (4 bits: node id, or PK_DISCARD) | group (20) | payload (40).
+// Tile payload: bz (12) | by (14) | bx (14); discard payload: chunk index.
+constexpr uint64_t PK_DISCARD = 15, PK_STOP = 14;
+__host__ __device__ inline uint64_t pack_ticket(uint64_t kind, uint64_t group, uint64_t payload) {
+  return (kind << 60) | (group << 40) | payload;
+}
+__host__ __device__ inline uint64_t tile_payload(uint64_t bx, uint64_t by, uint64_t bz) {
+  return (bz << 28) | (by << 14) | bx;
 }
 struct PParams {
   const PNode* nodes;
-  const uint64_t* desc;  // one descriptor per ticket, in schedule order
-  int32_t discard;
+  const uint64_t* desc;     // [G][per_cta] tickets, STOP-padded
+  int64_t per_cta;
+  const int32_t* dep_off;   // CSR over groups
+  const PDep* deps;
+  const DRect* drects;
+  const PChunk* chunks;
+  int32_t nsub;             // groups < nsub are sub-kernels (counted); the rest discard lists
   int32_t pad;
-  int64_t total;
-  unsigned int* flags;
-  unsigned int* rc;
+  unsigned int* cnt;        // completion counters, one per sub-kernel
   PCtrl* ctrl;
-  int64_t stage_bytes;  // one staging buffer (the kernel double-buffers)
+  int64_t stage_bytes;      // one ring slot
+  int32_t nslots;
+  int32_t nnodes;
   TraceBuf tb;
 };
 
-
-// Producer blocks i in [0, n) with [a*i, a*(i+1)) meeting [lo, hi) (write footprints have no
-// offsets or halos for built-ins).  32-bit: pixel coordinates are < 2^31.
-__device__ __forceinline__ void hit(int a, int lo, int hi, int n, int& i0, int& i1) {
-  i0 = lo > 0 ? lo / a : 0;
-  i1 = min(n, (hi + a - 1) / a);
-  if (i1 < i0) i1 = i0;
-}
-
-// Decoded ticket: node, block, its output rect, and the producer-block range of its read
-// footprint (the closed-form dependency of the affine maps).  Computed
-// once per tile by the control warp and handed to the compute warps in shared memory.
-struct TInfo {
-  const PNode* nd;
-  ktd::Tile t;
-  int bx, by, px0, py0, pw, ndep;
-};
-
-__device__ __forceinline__ TInfo decode(const PParams& p, uint64_t dsc) {
-  TInfo r;
-  r.nd = p.nodes + (dsc >> 60);
-  const PNode& nd = *r.nd;
-  r.by = (int)((dsc >> 24) & 0xFFFFFF);
-  r.bx = (int)(dsc & 0xFFFFFF);
-  const int tw = nd.tw, th = nd.th, W = (int)nd.out.W, H = (int)nd.out.H;
-  r.t.z = (int64_t)((dsc >> 48) & 0xFFF);
-  r.t.x0 = tw * r.bx;
-  r.t.y0 = th * r.by;
-  r.t.x1 = min(tw * r.bx + tw, W);
-  r.t.y1 = min(th * r.by + th, H);
-  r.t.fw = tw;
-  r.t.pad = 0;
-  int px0 = 0, px1 = 0, py0 = 0, py1 = 0;
-  if (nd.pu >= 0) {
-    const int rax = (int)nd.rax, ray = (int)nd.ray, rox = (int)nd.rox, roy = (int)nd.roy;
-    const int rx0 = max(0, rax * r.bx + rox - nd.rhl), rx1 = min((int)nd.in.W, rax * (r.bx + 1) + rox + nd.rhr);
-    const int ry0 = max(0, ray * r.by + roy - nd.rht), ry1 = min((int)nd.in.H, ray * (r.by + 1) + roy + nd.rhb);
-    hit((int)nd.wax, rx0, rx1, nd.pgx, px0, px1);
-    hit((int)nd.way, ry0, ry1, nd.pgy, py0, py1);
-  }
-  r.px0 = px0;
-  r.py0 = py0;
-  r.pw = px1 - px0;
-  r.ndep = r.pw * (py1 - py0);
-  return r;
-}
-
-__device__ __forceinline__ const unsigned int* dep_flag(const PParams& p, const TInfo& a, int i) {
-  const PNode& nd = *a.nd;
-  const int dy = i / a.pw;
-  return p.flags + nd.pflag0 + ((int64_t)a.t.z * nd.pgy + a.py0 + dy) * nd.pgx + a.px0 + (i - dy * a.pw);
-}
-
-// ---- persistent executor: warp-specialized (PCOMP_WARPS compute warps + 1 control warp) ----
-__device__ __forceinline__ void nbar_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 __device__ __forceinline__ void nbar_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 __device__ __forceinline__ void mbar_arrive(uint64_t* m) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(ktd::smem_u32(m)) : "memory");
 }
-constexpr uint64_t DESC_STOP = ~0ull;
+__device__ __forceinline__ bool mbar_test(uint64_t* m, unsigned parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred P;\n mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n selp.u32 %0, 1, 0, P;\n}"
+      : "=r"(ok)
+      : "r"(ktd::smem_u32(m)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void red_release_add(unsigned int* p, unsigned int v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 constexpr unsigned FULL = 0xFFFFFFFFu;
 
-// Control warp: are all producer blocks of a complete?  (one poll per flag, warp-uniform)
-__device__ __forceinline__ bool ctl_probe(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
-  bool ok = true;
-  for (int i = lane; i < a.ndep; i += 32) ok &= (ld_acquire(dep_flag(p, a, i)) == epoch);
-  return __all_sync(FULL, ok);
+__device__ __forceinline__ ktd::Tile ticket_tile(const PNode& nd, uint64_t d) {
+  const int bx = (int)(d & 0x3FFF), by = (int)((d >> 14) & 0x3FFF);
+  ktd::Tile t;
+  t.z = (int64_t)((d >> 28) & 0xFFF);
+  t.x0 = (int64_t)nd.tw * bx;
+  t.y0 = (int64_t)nd.th * by;
+  t.x1 = min(t.x0 + nd.tw, nd.out.W);
+  t.y1 = min(t.y0 + nd.th, nd.out.H);
+  t.fw = nd.tw;
+  t.pad = 0;
+  return t;
 }
-__device__ __forceinline__ void ctl_wait(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
-  for (int i = lane; i < a.ndep; i += 32) {
-    const unsigned int* f = dep_flag(p, a, i);
-    while (ld_acquire(f) != epoch) __nanosleep(32);
+
+// Producer warp: wait until every dependency group of `group` is complete this epoch.
+// Polls are relaxed (no L1 invalidation per poll); one acquire once they are satisfied.
+__device__ __forceinline__ unsigned int ld_relaxed(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void wait_group(const PParams& p, int group, unsigned epoch, int lane) {
+  const int a = p.dep_off[group], b = p.dep_off[group + 1];
+  for (int i = a + lane; i < b; i += 32) {
+    const PDep dp = p.deps[i];
+    const unsigned target = epoch * dp.ntiles;
+    if ((int)(ld_relaxed(p.cnt + dp.sub) - target) < 0) {
+      while ((int)(ld_relaxed(p.cnt + dp.sub) - target) < 0) __nanosleep(100);
+    }
+    (void)ld_acquire(p.cnt + dp.sub);
   }
   __syncwarp();
 }
-
-// Control warp, after the compute warps finished tile a (named barrier): publish its
-// completion flag (gpu-scope release), then count it as a reader of its producer blocks;
-// the last reader of a block drops that block's lines from L2 without write-back.
-__device__ __forceinline__ void ctl_release(const PParams& p, const TInfo& a, unsigned epoch, int lane) {
-  const PNode& nd = *a.nd;
-  if (lane == 0) st_release(p.flags + nd.flag0 + (a.t.z * nd.gy + a.by) * nd.gx + a.bx, epoch);
-  if (!(p.discard && nd.disc_in)) return;
-  for (int base = 0; base < a.ndep; base += 32) {
-    const int i = base + lane;
-    int64_t pl = 0;
-    bool dead = false;
-    if (i < a.ndep) {
-      const int dy = i / a.pw;
-      pl = ((int64_t)a.t.z * nd.pgy + a.py0 + dy) * nd.pgx + a.px0 + (i - dy * a.pw);
-      const unsigned int old = atomicAdd(p.rc + nd.pflag0 + pl, 1u);
-      dead = old + 1 == nd.expect[pl];
-      if (dead) p.rc[nd.pflag0 + pl] = 0;
-    }
-    unsigned mask = __ballot_sync(FULL, dead);
-    const int eb = nd.op == 4 ? 4 : 1;  // element bytes of the producer output (= our input)
-    while (mask) {
-      const int j = __ffs(mask) - 1;
-      mask &= mask - 1;
-      const int q = (int)(__shfl_sync(FULL, pl, j) - (int64_t)a.t.z * nd.pgy * nd.pgx);  // within the frame
-      const int qy = q / nd.pgx, qx = q - qy * nd.pgx;
-      const int ax0 = (int)nd.ptw * qx, ax1 = min(ax0 + (int)nd.ptw, (int)nd.in.W);
-      const int ay0 = (int)nd.pth * qy, ay1 = min(ay0 + (int)nd.pth, (int)nd.in.H);
-      const uint8_t* fb = nd.in.p + a.t.z * nd.in.fstride;
-      // lines fully inside [ax0*eb, ax1*eb) of each row (the buffer pitch is a multiple of 128)
-      const int l0 = (ax0 * eb + 127) >> 7, l1 = (ax1 * eb) >> 7, lpr = l1 > l0 ? l1 - l0 : 0;
-      const int n = lpr * (ay1 - ay0);
-      for (int k = lane; k < n; k += 32) {
-        const int dy = k / lpr;
-        ktd::discard_line(fb + (int64_t)(ay0 + dy) * nd.in.pitch + 128 * (l0 + k - dy * lpr));
-      }
-    }
-  }
+// mbarrier wait that suspends between probes (off the compute warps' critical path)
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* m, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred P;\n KT_WS_%=:\n mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n @!P bra KT_WS_%=;\n}" ::"r"(
+          ktd::smem_u32(m)),
+      "r"(parity), "r"(1000000u)
+      : "memory");
 }
 
-// Persistent executor.  One launch runs the whole schedule.  Ticket t (a tile, in the
-// order of the descriptor table: the schedule's total order, optionally skewed) belongs
-// to CTA t mod G, and every CTA runs its tickets in order — no ticket atomics.  Deadlock-
-// free: a tile's producers have smaller tickets, so the smallest unfinished ticket is
-// always runnable and its CTA reaches it (all its smaller tickets are finished).
-// Warp specialization inside a CTA, around a PSTAGES-deep ring of staging buffers:
-//   producer warp   for each of its tickets: wait until the ring slot is free (s_empty,
-//                   released by the publisher), wait (acquire) for the tile's producer
-//                   flags, stream the input tile into the slot with one TMA (s_full);
-//   compute warps   wait on s_full, compute the tile from shared memory, arrive
-//                   (non-blocking) on the slot's named barrier;
-//   publisher warp  syncs on that barrier, frees the slot, publishes the tile's flag
-//                   (gpu-scope release) and retires dead producer lines (reader counts).
-// So the dependency wait and TMA latency of later tiles, and the release of earlier ones,
-// overlap the compute of the current tile: no compute warp waits on a flag or a fence.
+// Warp roles: PCOMP_WARPS compute warps, one producer warp (dependency check + TMA issue
+// into a ring of nslots staging slots), one publisher warp (publishes finished tiles to
+// the sub-kernel counters with one gpu-scope release per run of consecutive tiles of the
+// same sub-kernel).  The compute warps free a slot themselves (s_empty), so neither a
+// dependency poll nor a release fence ever sits between a finished tile and the refill of
+// its slot.  The publisher reads finished tiles from its own queue (PUBQ entries, s_done
+// barriers); the producer keeps at most PUBQ - nslots tickets ahead of it, so a queue
+// entry is never overwritten before it is published.
+constexpr int PUBQ = 32;
 template <int MINB>
 __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const __grid_constant__ PParams p) {
-  __shared__ __align__(8) uint64_t s_full[PSTAGES];
-  __shared__ __align__(8) uint64_t s_empty[PSTAGES];
-  __shared__ uint64_t s_desc[PSTAGES];
-  __shared__ TInfo s_ti[PSTAGES];  // decoded tile of each slot (producer -> compute warps)
+  __shared__ __align__(8) uint64_t s_full[PSTAGES_MAX];
+  __shared__ __align__(8) uint64_t s_empty[PSTAGES_MAX];
+  __shared__ __align__(8) uint64_t s_done[PUBQ];
+  __shared__ uint64_t s_desc[PSTAGES_MAX];
+  __shared__ ktd::Tile s_tile[PSTAGES_MAX];
+  __shared__ int32_t s_pub[PUBQ];          // group of finished tile k (k mod PUBQ)
+  __shared__ volatile int32_t s_pubk;      // tiles the publisher has consumed
+  __shared__ __align__(64) PNode s_nodes[PMAX_NODES];
   __shared__ unsigned int s_epoch;
-  __shared__ uint64_t s_tc0, s_tq0;  // trace timestamps (kept out of registers)
   extern __shared__ __align__(128) uint8_t ktsm[];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int S = p.nslots;
+  for (int i = tid; i < p.nnodes * (int)(sizeof(PNode) / 4); i += blockDim.x)
+    reinterpret_cast<uint32_t*>(s_nodes)[i] = reinterpret_cast<const uint32_t*>(p.nodes)[i];
   if (tid == 0) {
     s_epoch = *(volatile unsigned int*)&p.ctrl->epoch;
-    for (int s = 0; s < PSTAGES; ++s) {
+    s_pubk = 0;
+    for (int s = 0; s < S; ++s) {
       ktd::mbar_init(&s_full[s], 1);
-      ktd::mbar_init(&s_empty[s], 1);
+      ktd::mbar_init(&s_empty[s], PCOMP_THREADS);
     }
+    for (int q = 0; q < PUBQ; ++q) ktd::mbar_init(&s_done[q], PCOMP_THREADS);
     ktd::fence_proxy_async();
   }
   __syncthreads();
   const unsigned int epoch = s_epoch;
-  const int64_t G = gridDim.x;
+  const uint64_t* my = p.desc + (int64_t)blockIdx.x * p.per_cta;
   if (warp == PCOMP_WARPS) {
     // ------------------------------ producer warp ------------------------------
-    int s = 0;
+    int s = 0, ok_group = -1;
     unsigned ph = 0;  // bit s: parity of slot s's current use
-    for (int64_t t = blockIdx.x, k = 0;; t += G, ++k) {
-      if (k >= PSTAGES) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
-      if (t >= p.total) {
+    uint64_t batch = 0;
+    for (int64_t k = 0;; ++k) {
+      if ((k & 31) == 0) batch = k + lane < p.per_cta ? my[k + lane] : pack_ticket(PK_STOP, 0, 0);
+      const uint64_t d = __shfl_sync(FULL, batch, (int)(k & 31));
+      const uint64_t kind = d >> 60;
+      if (k >= S) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
+      while ((int)k - s_pubk > PUBQ - PSTAGES_MAX) __nanosleep(200);  // publisher queue bound
+      if (kind == PK_STOP) {
         if (lane == 0) {
-          s_desc[s] = DESC_STOP;
+          s_desc[s] = d;
           mbar_arrive(&s_full[s]);
         }
         break;
       }
-      if (p.tb.rec && lane == 0) s_tq0 = gtimer();
-      const uint64_t d = p.desc[t];
-      const TInfo a = decode(p, d);
-      ctl_wait(p, a, epoch, lane);
-      uint8_t* buf = ktsm + s * p.stage_bytes;
+      const uint64_t tq0 = p.tb.rec ? gtimer() : 0;
+      const int group = (int)((d >> 40) & 0xFFFFF);
+      if (group != ok_group) {
+        wait_group(p, group, epoch, lane);
+        ok_group = group;
+      }
       if (lane == 0) {
         s_desc[s] = d;
-        s_ti[s] = a;
-      }
-      if (a.nd->scalar) {
-        if (lane == 0) mbar_arrive(&s_full[s]);
-      } else {
-        ktd::fence_proxy_async();
-        if (a.nd->use_tmap) {
-          if (lane == 0)
-            ktd::stage_issue_tmap(a.nd->op, &a.nd->tmap, a.nd->box_bytes, a.nd->in, a.t, buf, &s_full[s], a.nd->in_stream != 0);
+        if (kind == PK_DISCARD) {
+          mbar_arrive(&s_full[s]);
         } else {
-          ktd::stage_issue(a.nd->op, a.nd->in, a.t, buf, &s_full[s], lane);
+          const PNode& nd = s_nodes[kind];
+          const ktd::Tile t = ticket_tile(nd, d);
+          s_tile[s] = t;
+          if (nd.scalar) {
+            mbar_arrive(&s_full[s]);
+          } else {
+            ktd::fence_proxy_async();
+            ktd::stage_issue_tmap(nd.op, &p.nodes[kind].tmap, nd.box_bytes, nd.in, t, ktsm + s * p.stage_bytes,
+                                  &s_full[s], nd.in_stream != 0);
+          }
+          if (p.tb.rec) trace_put(p.tb, d, 1, tq0, gtimer());
         }
       }
-      if (p.tb.rec && lane == 0) trace_put(p.tb, d, 1, s_tq0, gtimer());
+      __syncwarp();
       ph ^= 1u << s;
-      s = s + 1 == PSTAGES ? 0 : s + 1;
+      s = s + 1 == S ? 0 : s + 1;
     }
   } else if (warp == PCOMP_WARPS + 1) {
     // ------------------------------ publisher warp ------------------------------
-    int s = 0;
-    for (int64_t t = blockIdx.x; t < p.total; t += G) {
-      nbar_sync(1 + s, PCOMP_THREADS + 32);  // the compute warps are done with slot s
-      const uint64_t d = s_desc[s];
+    unsigned ph = 0;    // bit q: parity of queue entry q
+    int cur = -1;       // sub-kernel of the pending run
+    unsigned pend = 0;  // finished tiles not yet published
+    for (int k = 0;; ++k) {
+      const int q = k & (PUBQ - 1);
+      const unsigned par = (ph >> q) & 1u;
+      if (pend && !mbar_test(&s_done[q], par)) {  // nothing more finished right now: publish
+        if (lane == 0) red_release_add(p.cnt + cur, pend);
+        pend = 0;
+      }
+      mbar_wait_sleep(&s_done[q], par);
+      const int group = s_pub[q];
       __syncwarp();
-      if (lane == 0) mbar_arrive(&s_empty[s]);  // the producer may refill slot s
-      ctl_release(p, decode(p, d), epoch, lane);
-      s = s + 1 == PSTAGES ? 0 : s + 1;
+      if (lane == 0) s_pubk = k + 1;
+      ph ^= 1u << q;
+      if (group < 0) break;            // STOP
+      if (group >= p.nsub) continue;   // discard chunk: nobody waits on it
+      if (group != cur && pend) {
+        if (lane == 0) red_release_add(p.cnt + cur, pend);
+        pend = 0;
+      }
+      cur = group;
+      ++pend;
     }
+    if (pend && lane == 0) red_release_add(p.cnt + cur, pend);
   } else {
     // ------------------------------ compute warps ------------------------------
     int s = 0;
     unsigned ph = 0;
-    for (;;) {
+    for (int k = 0;; ++k) {
       ktd::mbar_wait(&s_full[s], (ph >> s) & 1u);
       ph ^= 1u << s;
-      if (s_desc[s] == DESC_STOP) break;
-      if (p.tb.rec && tid == 0) s_tc0 = gtimer();
-      const TInfo a = s_ti[s];
-      const PNode& nd = *a.nd;
-      uint8_t* buf = ktsm + s * p.stage_bytes;
-      if (nd.scalar) {
-        ktd::scalar_tile(nd.op, nd.in, nd.out, a.t, nd.T, PCOMP_THREADS, tid);
-      } else {
-        if ((nd.op == 1 || nd.op == 3) && ktd::needs_fix(nd.op, nd.in, a.t)) {
-          ktd::stage_fix(nd.op, nd.in, a.t, buf, PCOMP_THREADS, tid);
-          nbar_sync(4, PCOMP_THREADS);
-        }
-        ktd::compute_tile(nd.op, nd.out, a.t, buf, nd.T, PCOMP_THREADS, tid);
+      const uint64_t d = s_desc[s];
+      const uint64_t kind = d >> 60;
+      if (kind == PK_STOP) {
+        if (tid == 0) s_pub[k & (PUBQ - 1)] = -1;
+        mbar_arrive(&s_done[k & (PUBQ - 1)]);
+        break;
       }
-      if (p.tb.rec && tid == 0) trace_put(p.tb, s_desc[s], 2, s_tc0, gtimer());
-      __threadfence_block();  // this thread's tile writes before the hand-off (cumulative release)
-      nbar_arrive(1 + s, PCOMP_THREADS + 32);
-      s = s + 1 == PSTAGES ? 0 : s + 1;
+      const uint64_t tc0 = p.tb.rec ? gtimer() : 0;
+      if (kind == PK_DISCARD) {
+        const PChunk c = p.chunks[d & 0xFFFFFFFFFFull];
+        const DRect& r = p.drects[c.d];
+        const int64_t h = r.y1 - r.y0;
+        for (int64_t i = tid; i < c.n; i += PCOMP_THREADS) {
+          const int64_t j = c.l0 + i, row = j / r.lpr, l = j - row * r.lpr;
+          const int64_t z = r.z0 + row / h, y = r.y0 + row % h;
+          ktd::discard_line(r.base + z * r.fstride + y * r.pitch + r.lb0 + 128 * l);
+        }
+        mbar_arrive(&s_empty[s]);
+        if (tid == 0) s_pub[k & (PUBQ - 1)] = (int32_t)((d >> 40) & 0xFFFFF);
+        mbar_arrive(&s_done[k & (PUBQ - 1)]);
+      } else {
+        const PNode& nd = s_nodes[kind];
+        const ktd::Tile t = s_tile[s];
+        uint8_t* buf = ktsm + s * p.stage_bytes;
+        if (nd.scalar) {
+          ktd::scalar_tile(nd.op, nd.in, nd.out, t, nd.T, PCOMP_THREADS, tid);
+        } else {
+          if ((nd.op == 1 || nd.op == 3) && ktd::needs_fix(nd.op, nd.in, t)) {
+            ktd::stage_fix(nd.op, nd.in, t, buf, PCOMP_THREADS, tid);
+            nbar_sync(1, PCOMP_THREADS);
+          }
+          ktd::compute_tile(nd.op, nd.out, t, buf, nd.T, PCOMP_THREADS, tid);
+        }
+        mbar_arrive(&s_empty[s]);  // this thread is done with the slot
+        if (tid == 0) {
+          if (p.tb.rec) trace_put(p.tb, d, 2, tc0, gtimer());
+          s_pub[k & (PUBQ - 1)] = (int32_t)((d >> 40) & 0xFFFFF);
+        }
+        // every compute thread arrives (release.cta) after its tile writes; the publisher
+        // acquires the completed phase before its gpu-scope release (cumulative)
+        mbar_arrive(&s_done[k & (PUBQ - 1)]);
+      }
+      s = s + 1 == S ? 0 : s + 1;
     }
   }
   __syncthreads();
@@ -617,7 +636,6 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
     __threadfence();
     unsigned int old = atomicAdd(&p.ctrl->done, 1u);
     if (old == gridDim.x - 1) {
-      p.ctrl->ticket = 0;
       p.ctrl->done = 0;
       __threadfence();
       atomicAdd(&p.ctrl->epoch, 1u);
@@ -679,6 +697,7 @@ struct ktiler_plan_s {
   void* dmem = nullptr;
   PParams pp{};
   int pctas = 0;
+  int pminb = 2;
   int psmem = 0;
   void (*pfn)(PParams) = nullptr;
   int64_t skew = 0;
@@ -1238,35 +1257,19 @@ ktiler_status setup_chain(ktiler_plan_s* P) {
 
 ktiler_status setup_persistent(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
+  const kt::Schedule& S = P->s;
   const int nn = (int)g.nodes.size();
+  const int nsub = (int)S.subs.size();
   for (auto& n : g.nodes)
     if (n.op == KTILER_OP_CUSTOM) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode runs built-in ops only");
-  // flags: one u32 per block of every node; rc: reader counters, same indexing
-  std::vector<int64_t> flag0(nn);
-  int64_t nflags = 0;
-  for (int v = 0; v < nn; ++v) {
-    flag0[v] = nflags;
-    nflags += g.nodes[v].nblocks;
-  }
-  // expected reader counts per producer block (u8)
-  std::vector<uint8_t> expect(nflags, 0);
-  for (int u = 0; u < nn; ++u) {
-    const kt::Node& n = g.nodes[u];
-    for (int64_t l = 0; l < n.nblocks; ++l) {
-      int64_t px = l % n.gx(), py = (l / n.gx()) % n.gy();
-      int64_t cnt = 0;
-      for (auto& c : g.out_ch[u]) {
-        kt::BRange r = g.consumers(c, px, py);
-        cnt += (r.x1 - r.x0) * (r.y1 - r.y0);
-      }
-      expect[flag0[u] + l] = (uint8_t)std::min<int64_t>(cnt, 255);
-    }
-  }
+  if (nn > PMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: at most 8 nodes");
   std::vector<PNode> pn(nn);
   for (int v = 0; v < nn; ++v) {
     const kt::Node& n = g.nodes[v];
     const kt::Access& w = n.acc[n.wacc];
     const kt::Access& r = n.acc[n.racc];
+    if (n.gx() >= (1 << 14) || n.gy() >= (1 << 14) || n.gz() > 4096)
+      return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: grid exceeds the ticket (2^14 blocks per axis, 4096 frames)");
     PNode& q = pn[v];
     std::memset(&q, 0, sizeof(q));
     q.in = dbuf(g.bufs[r.buf]);
@@ -1276,121 +1279,160 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     q.tw = (int32_t)w.ax;
     q.th = (int32_t)w.ay;
     q.T = n.T;
-    q.gx = (int32_t)n.gx();
-    q.gy = (int32_t)n.gy();
-    q.flag0 = flag0[v];
-    q.pu = -1;
-    for (auto& c : g.in_ch[v]) {
-      const kt::Node& u = g.nodes[c.u];
-      const kt::Access& uw = u.acc[c.w];
-      q.pu = c.u;
-      q.rax = r.ax; q.ray = r.ay; q.rox = r.ox; q.roy = r.oy;
-      q.rhl = r.hl; q.rhr = r.hr; q.rht = r.ht; q.rhb = r.hb;
-      q.wax = uw.ax; q.way = uw.ay;
-      q.pgx = (int32_t)u.gx(); q.pgy = (int32_t)u.gy();
-      q.pflag0 = flag0[c.u];
-      q.ptw = uw.ax; q.pth = uw.ay;
-      const kt::Buffer& ib = g.bufs[c.buf];
-      q.disc_in = (ib.d.flags & KTILER_BUF_INTERNAL) && discardable(ib);
-    }
     q.use_tmap = !n.scalar && make_tmap(g, n, &q.tmap, &q.box_bytes);
+    if (!n.scalar && !q.use_tmap) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: input tile map unavailable");
     q.in_stream = !g.written_by_node(r.buf);
   }
-  int nsm = 0, occ = 0;
+  int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
   {
-    // registers vs CTAs per SM (KTILER_PERSIST_MINB = 2 or 3 minimum resident CTAs)
     const char* ev = getenv("KTILER_PERSIST_MINB");
-    int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
-    P->pfn = mb >= 3 ? persistent_kernel<3> : persistent_kernel<2>;
+    const int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
+    P->pfn = mb >= 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>);
+    P->pminb = mb >= 4 ? 4 : (mb == 3 ? 3 : 2);
   }
-  P->psmem = 0;
+  int slot = 0;
   for (auto& n : g.nodes) {
     const kt::Access& w = n.acc[n.wacc];
-    if (!n.scalar) P->psmem = std::max(P->psmem, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
+    if (!n.scalar) slot = std::max(slot, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
   }
-  P->pp.stage_bytes = P->psmem;
-  P->psmem *= PSTAGES;
-  if (P->psmem > 32 * 1024) {
+  // ring depth: as many slots as fit the shared memory of MINB CTAs per SM (2..PSTAGES_MAX)
+  int smem_sm = 0;
+  cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
+  const int per_cta = smem_sm / P->pminb - 2048;  // static smem + per-CTA reserve
+  int nslots = slot ? std::min(PSTAGES_MAX, std::max(2, per_cta / slot)) : 2;
+  if (const char* ev = getenv("KTILER_PERSIST_SLOTS")) nslots = std::min(PSTAGES_MAX, std::max(2, atoi(ev)));
+  P->psmem = std::max(slot, 128) * nslots;
+  if (P->psmem > 48 * 1024) {
     cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
   }
+  int occ = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, P->pfn, PERSIST_THREADS, P->psmem);
-  P->pctas = P->pol.persistent_ctas > 0 ? P->pol.persistent_ctas : nsm * std::max(1, occ);
-  // Ticket order.  skew < 0: the emitted (fragment-major) order.  skew = k > 0: software
+  if (occ < 1) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: kernel does not fit an SM");
+  P->pctas = P->pol.persistent_ctas > 0 ? std::min(P->pol.persistent_ctas, nsm * occ) : nsm * occ;
+  // Group order.  skew < 0: the emitted (fragment-major) order.  skew = k > 0: software
   // pipeline over fragments — the sub-kernel of fragment f at node depth d is issued at
   // step f + d*k, deepest node first within a step.  A consumer's producers sit in
   // fragments <= f at smaller depth, hence at strictly earlier steps: still a valid total
-  // order, and about k fragments of tiles separate a tile from its
-  // producers, so a CTA rarely waits.
+  // order, and k steps of other work separate a sub-kernel from its
+  // producers, so the dependency check rarely waits.
   std::vector<int> depth(nn, 0);
   int dmax = 0;
   for (int v : g.topo)
     for (auto& c : g.in_ch[v]) depth[v] = std::max(depth[v], depth[c.u] + 1);
   for (int v = 0; v < nn; ++v) dmax = std::max(dmax, depth[v]);
-  const int64_t nfrag = P->s.nfrag;
+  const int64_t nfrag = S.nfrag;
   std::vector<std::vector<int>> by_frag(nfrag, std::vector<int>(nn, -1));
-  int64_t tiles = 0;
-  for (size_t i = 0; i < P->s.subs.size(); ++i) {
-    by_frag[P->s.subs[i].frag][P->s.subs[i].node] = (int)i;
-    tiles += P->s.subs[i].nblocks;
-  }
+  for (int i = 0; i < nsub; ++i) by_frag[S.subs[i].frag][S.subs[i].node] = i;
   int64_t k = P->pol.pipeline_skew;
-  if (k == 0) {
-    int64_t per_frag = std::max<int64_t>(1, tiles / std::max<int64_t>(1, nfrag));
-    k = std::max<int64_t>(1, (3 * (int64_t)P->pctas + 2 * per_frag - 1) / (2 * per_frag));
-  }
+  if (k == 0) k = 1;
   P->skew = k;
   std::vector<int> order;
   if (k < 0) {
-    for (size_t i = 0; i < P->s.subs.size(); ++i) order.push_back((int)i);
+    for (int i = 0; i < nsub; ++i) order.push_back(i);
   } else {
     std::vector<int> rtopo(g.topo.rbegin(), g.topo.rend());
-    for (int64_t s = 0; s < nfrag + dmax * k; ++s)
+    for (int64_t st = 0; st < nfrag + dmax * k; ++st)
       for (int v : rtopo) {
-        int64_t f = s - depth[v] * k;
+        const int64_t f = st - depth[v] * k;
         if (f >= 0 && f < nfrag && by_frag[f][v] >= 0) order.push_back(by_frag[f][v]);
       }
   }
-  // per-ticket tile descriptors, in ticket order (blocks of one sub-kernel in rect order)
-  std::vector<uint64_t> desc;
-  desc.reserve(tiles);
-  for (int oi : order) {
-    const kt::SubKernel& sk = P->s.subs[oi];
-    if (g.nodes[sk.node].gz() > 4096 || g.nodes[sk.node].gy() >= (1 << 24) || g.nodes[sk.node].gx() >= (1 << 24) || nn > 16)
-      return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: grid exceeds the tile descriptor (16 nodes, 4096 frames, 2^24 blocks per axis)");
+  // Discard lists (groups nsub + si): after the last of their readers, one pipeline step
+  // (nn sub-kernels) later so the readers have finished by the time the chunks are reached.
+  const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
+  std::vector<int> pos(nsub, 0);
+  for (size_t i = 0; i < order.size(); ++i) pos[order[i]] = (int)i;
+  std::vector<std::vector<int>> disc_after(order.size() + 1);
+  std::vector<DRect> drects;
+  std::vector<std::vector<int>> drect_of(nsub);
+  if (disc) {
+    for (int si = 0; si < nsub; ++si) {
+      for (auto& dd : S.discards[si]) {
+        if (!discardable(g.bufs[dd.buf])) continue;
+        DRect dr = drect(g, dd);
+        if (dr.lpr <= 0) continue;
+        drect_of[si].push_back((int)drects.size());
+        drects.push_back(dr);
+      }
+      if (drect_of[si].empty()) continue;
+      int last = pos[si];
+      for (int r : S.discard_readers[si]) last = std::max(last, pos[r]);
+      disc_after[std::min<size_t>(order.size(), (size_t)last + (size_t)nn)].push_back(si);
+    }
+  }
+  // groups' dependency lists (CSR) and the tickets in global order
+  const int ngroups = 2 * nsub;
+  if (ngroups >= (1 << 20)) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: too many sub-kernels");
+  std::vector<int32_t> dep_off(ngroups + 1, 0);
+  std::vector<PDep> deps;
+  for (int gi = 0; gi < ngroups; ++gi) {
+    const std::vector<int32_t>& src = gi < nsub ? S.sub_deps[gi] : S.discard_readers[gi - nsub];
+    for (int32_t u : src) deps.push_back(PDep{u, (uint32_t)S.subs[u].nblocks});
+    dep_off[gi + 1] = (int32_t)deps.size();
+  }
+  std::vector<uint64_t> tickets;
+  std::vector<PChunk> chunks;
+  constexpr int64_t CHUNK_LINES = 2048;  // 256 KB of dead lines per discard ticket
+  auto emit_discards = [&](int si) {
+    for (int di : drect_of[si]) {
+      const DRect& r = drects[di];
+      const int64_t lines = r.lpr * (int64_t)(r.y1 - r.y0) * (r.z1 - r.z0);
+      for (int64_t l0 = 0; l0 < lines; l0 += CHUNK_LINES) {
+        tickets.push_back(pack_ticket(PK_DISCARD, (uint64_t)(nsub + si), chunks.size()));
+        chunks.push_back(PChunk{di, (int32_t)std::min(CHUNK_LINES, lines - l0), l0});
+      }
+    }
+  };
+  for (size_t i = 0; i <= order.size(); ++i) {
+    for (int si : disc_after[i]) emit_discards(si);
+    if (i == order.size()) break;
+    const kt::SubKernel& sk = S.subs[order[i]];
     for (auto& r : sk.rects)
       for (int64_t z = r.z0; z < r.z1; ++z)
         for (int64_t y = r.y0; y < r.y1; ++y)
-          for (int64_t x = r.x0; x < r.x1; ++x) desc.push_back(pack_tile(sk.node, x, y, z));
+          for (int64_t x = r.x0; x < r.x1; ++x)
+            tickets.push_back(pack_ticket((uint64_t)sk.node, (uint64_t)order[i], tile_payload(x, y, z)));
   }
-  const int64_t t0 = (int64_t)desc.size();
-  // one device allocation: ctrl | flags | rc | expect | nodes | desc
+  // per-CTA contiguous ticket lists (ticket i -> CTA i mod G, in order), STOP-padded
+  const int64_t G = P->pctas, T = (int64_t)tickets.size();
+  const int64_t per = (T + G - 1) / G + 1;
+  std::vector<uint64_t> desc((size_t)(G * per), pack_ticket(PK_STOP, 0, 0));
+  for (int64_t i = 0; i < T; ++i) desc[(size_t)((i % G) * per + i / G)] = tickets[(size_t)i];
+  // one device allocation: ctrl | counters | dep_off | deps | drects | chunks | nodes | desc
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
-  size_t o_ctrl = 0, o_flags = al(sizeof(PCtrl)), o_rc = o_flags + al(nflags * 4), o_exp = o_rc + al(nflags * 4);
-  size_t o_nodes = o_exp + al(nflags), o_desc = o_nodes + al(pn.size() * sizeof(PNode));
-  size_t total = o_desc + al(desc.size() * sizeof(uint64_t));
+  size_t o_ctrl = 0, o_cnt = al(sizeof(PCtrl)), o_doff = o_cnt + al((size_t)nsub * 4 + 4);
+  size_t o_deps = o_doff + al(dep_off.size() * 4), o_dr = o_deps + al(deps.size() * sizeof(PDep) + 8);
+  size_t o_ch = o_dr + al(drects.size() * sizeof(DRect) + 8), o_nodes = o_ch + al(chunks.size() * sizeof(PChunk) + 8);
+  size_t o_desc = o_nodes + al(pn.size() * sizeof(PNode)), total = o_desc + al(desc.size() * sizeof(uint64_t));
   char* d = nullptr;
   cudaError_t e = cudaMalloc(&d, total);
   if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (persistent tables)");
   P->dmem = d;
-  for (auto& q : pn) q.expect = (const uint8_t*)(d + o_exp) + q.pflag0;
-  PCtrl c0{0, 0, 1, 0};
+  PCtrl c0{0, 1, 0, 0};
   if ((e = cudaMemset(d, 0, total)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
   cudaMemcpy(d + o_ctrl, &c0, sizeof(c0), cudaMemcpyHostToDevice);
-  cudaMemcpy(d + o_exp, expect.data(), expect.size(), cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_doff, dep_off.data(), dep_off.size() * 4, cudaMemcpyHostToDevice);
+  if (!deps.empty()) cudaMemcpy(d + o_deps, deps.data(), deps.size() * sizeof(PDep), cudaMemcpyHostToDevice);
+  if (!drects.empty()) cudaMemcpy(d + o_dr, drects.data(), drects.size() * sizeof(DRect), cudaMemcpyHostToDevice);
+  if (!chunks.empty()) cudaMemcpy(d + o_ch, chunks.data(), chunks.size() * sizeof(PChunk), cudaMemcpyHostToDevice);
   cudaMemcpy(d + o_nodes, pn.data(), pn.size() * sizeof(PNode), cudaMemcpyHostToDevice);
   if ((e = cudaMemcpy(d + o_desc, desc.data(), desc.size() * sizeof(uint64_t), cudaMemcpyHostToDevice)) != cudaSuccess)
     return cuda_fail(e, "cudaMemcpy (persistent tables)");
-  // expect for nodes is indexed by the producer's local id: expect base + pflag0 was set
-  // above; the kernel adds the producer-local index.
   P->pp.nodes = (const PNode*)(d + o_nodes);
   P->pp.desc = (const uint64_t*)(d + o_desc);
-  P->pp.discard = (P->pol.flags & KTILER_PF_DISCARD_DEAD) ? 1 : 0;
-  P->pp.total = t0;
-  P->pp.flags = (unsigned int*)(d + o_flags);
-  P->pp.rc = (unsigned int*)(d + o_rc);
+  P->pp.per_cta = per;
+  P->pp.dep_off = (const int32_t*)(d + o_doff);
+  P->pp.deps = (const PDep*)(d + o_deps);
+  P->pp.drects = (const DRect*)(d + o_dr);
+  P->pp.chunks = (const PChunk*)(d + o_ch);
+  P->pp.nsub = nsub;
+  P->pp.cnt = (unsigned int*)(d + o_cnt);
   P->pp.ctrl = (PCtrl*)(d + o_ctrl);
+  P->pp.stage_bytes = std::max(slot, 128);
+  P->pp.nslots = nslots;
+  P->pp.nnodes = nn;
   return KTILER_OK;
 }
 
