@@ -34,9 +34,8 @@ using ktd::DBuf;
 constexpr int MAXR = 4, MAXD = 8;
 constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+ producer + publisher warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
-constexpr int PERSIST_THREADS = PCOMP_THREADS + 64;
-constexpr int PSTAGES_MAX = 6;   // staging ring depth (slots that fit the CTA's share of smem)
-constexpr int PERSIST_MINB_DEFAULT = 3;
+constexpr int PSTAGES_MAX = 12;   // staging ring depth (slots that fit the CTA's share of smem)
+constexpr int PERSIST_GROUPS_DEFAULT = 4;
 constexpr int PMAX_NODES = 8;
 
 struct LRect {
@@ -382,9 +381,13 @@ struct PChunk {      // one discard ticket: lines [l0, l0 + n) of rect d (row-ma
   int32_t n;
   int64_t l0;
 };
-// Ticket descriptor: kind (4 bits: node id, or PK_DISCARD) | group (20) | payload (40).
+// Ticket descriptor: kind (4 bits: node id, or PK_DISCARD) | check (1) | group (19) |
+// payload (40).  check = first ticket of its group in this CTA's list: the producer warp
+// verifies the group's dependencies there (and only there).
 // Tile payload: bz (12) | by (14) | bx (14); discard payload: chunk index.
-constexpr uint64_t PK_DISCARD = 15, PK_STOP = 14;
+constexpr uint64_t PK_DISCARD = 15, PK_STOP = 14, PK_CHECK = 1ull << 59;
+constexpr int PGROUP_BITS = 19;
+__host__ __device__ inline int ticket_group(uint64_t d) { return (int)((d >> 40) & ((1u << PGROUP_BITS) - 1)); }
 __host__ __device__ inline uint64_t pack_ticket(uint64_t kind, uint64_t group, uint64_t payload) {
   return (kind << 60) | (group << 40) | payload;
 }
@@ -468,24 +471,26 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* m, unsigned parity) {
       : "memory");
 }
 
-// Warp roles: PCOMP_WARPS compute warps, one producer warp (dependency check + TMA issue
-// into a ring of nslots staging slots), one publisher warp (publishes finished tiles to
-// the sub-kernel counters with one gpu-scope release per run of consecutive tiles of the
-// same sub-kernel).  The compute warps free a slot themselves (s_empty), so neither a
-// dependency poll nor a release fence ever sits between a finished tile and the refill of
-// its slot.  The publisher reads finished tiles from its own queue (PUBQ entries, s_done
-// barriers); the producer keeps at most PUBQ - nslots tickets ahead of it, so a queue
-// entry is never overwritten before it is published.
-constexpr int PUBQ = 32;
-template <int MINB>
-__global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const __grid_constant__ PParams p) {
+// Warp roles: NG compute groups of PCOMP_WARPS warps, one producer warp (dependency check
+// + TMA issue into a ring of nslots staging slots shared by the groups), one publisher
+// warp (publishes finished tiles to the sub-kernel counters with one gpu-scope release
+// per run of consecutive tiles of the same sub-kernel).  Ticket k of the CTA uses slot
+// k mod nslots and compute group k mod NG, so the groups share one pool of slots (a group
+// busy with a long tile does not hold prefetch slots idle).  The compute warps free a
+// slot themselves (s_empty), so neither a dependency poll nor a release fence ever sits
+// between a finished tile and the refill of its slot.  The publisher reads finished
+// tiles from its own queue (PUBQ entries, s_done barriers); the producer keeps at most
+// PUBQ - PSTAGES_MAX tickets ahead of it, so a queue entry is never reused early.
+constexpr int PUBQ = 64;
+template <int NG, int MINB>
+__global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kernel(const __grid_constant__ PParams p) {
   __shared__ __align__(8) uint64_t s_full[PSTAGES_MAX];
   __shared__ __align__(8) uint64_t s_empty[PSTAGES_MAX];
   __shared__ __align__(8) uint64_t s_done[PUBQ];
   __shared__ uint64_t s_desc[PSTAGES_MAX];
   __shared__ ktd::Tile s_tile[PSTAGES_MAX];
-  __shared__ int32_t s_pub[PUBQ];          // group of finished tile k (k mod PUBQ)
-  __shared__ volatile int32_t s_pubk;      // tiles the publisher has consumed
+  __shared__ int32_t s_pub[PUBQ];          // group of finished ticket k (k mod PUBQ)
+  __shared__ volatile int32_t s_pubk;      // tickets the publisher has consumed
   __shared__ __align__(64) PNode s_nodes[PMAX_NODES];
   __shared__ unsigned int s_epoch;
   extern __shared__ __align__(128) uint8_t ktsm[];
@@ -506,30 +511,30 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
   __syncthreads();
   const unsigned int epoch = s_epoch;
   const uint64_t* my = p.desc + (int64_t)blockIdx.x * p.per_cta;
-  if (warp == PCOMP_WARPS) {
+  if (warp == NG * PCOMP_WARPS) {
     // ------------------------------ producer warp ------------------------------
-    int s = 0, ok_group = -1;
+    int s = 0, stops = 0;
     unsigned ph = 0;  // bit s: parity of slot s's current use
     uint64_t batch = 0;
     for (int64_t k = 0;; ++k) {
       if ((k & 31) == 0) batch = k + lane < p.per_cta ? my[k + lane] : pack_ticket(PK_STOP, 0, 0);
       const uint64_t d = __shfl_sync(FULL, batch, (int)(k & 31));
-      const uint64_t kind = d >> 60;
       if (k >= S) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
       while ((int)k - s_pubk > PUBQ - PSTAGES_MAX) __nanosleep(200);  // publisher queue bound
-      if (kind == PK_STOP) {
+      const uint64_t kind = d >> 60;
+      if (kind == PK_STOP) {  // one STOP per compute group: tickets k .. k+NG-1
         if (lane == 0) {
           s_desc[s] = d;
           mbar_arrive(&s_full[s]);
         }
-        break;
+        __syncwarp();
+        if (++stops == NG) break;
+        ph ^= 1u << s;
+        s = s + 1 == S ? 0 : s + 1;
+        continue;
       }
       const uint64_t tq0 = p.tb.rec ? gtimer() : 0;
-      const int group = (int)((d >> 40) & 0xFFFFF);
-      if (group != ok_group) {
-        wait_group(p, group, epoch, lane);
-        ok_group = group;
-      }
+      if (d & PK_CHECK) wait_group(p, ticket_group(d), epoch, lane);
       if (lane == 0) {
         s_desc[s] = d;
         if (kind == PK_DISCARD) {
@@ -552,25 +557,29 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
       ph ^= 1u << s;
       s = s + 1 == S ? 0 : s + 1;
     }
-  } else if (warp == PCOMP_WARPS + 1) {
+  } else if (warp == NG * PCOMP_WARPS + 1) {
     // ------------------------------ publisher warp ------------------------------
-    unsigned ph = 0;    // bit q: parity of queue entry q
-    int cur = -1;       // sub-kernel of the pending run
-    unsigned pend = 0;  // finished tiles not yet published
+    unsigned long long ph = 0;  // bit q: parity of queue entry q
+    int cur = -1;               // sub-kernel of the pending run
+    unsigned pend = 0;          // finished tiles not yet published
+    int stops = 0;
     for (int k = 0;; ++k) {
       const int q = k & (PUBQ - 1);
-      const unsigned par = (ph >> q) & 1u;
+      const unsigned par = (unsigned)(ph >> q) & 1u;
       if (pend && !mbar_test(&s_done[q], par)) {  // nothing more finished right now: publish
         if (lane == 0) red_release_add(p.cnt + cur, pend);
         pend = 0;
       }
-      mbar_wait_sleep(&s_done[q], par);
+      while (!mbar_test(&s_done[q], par)) __nanosleep(64);
       const int group = s_pub[q];
       __syncwarp();
       if (lane == 0) s_pubk = k + 1;
-      ph ^= 1u << q;
-      if (group < 0) break;            // STOP
-      if (group >= p.nsub) continue;   // discard chunk: nobody waits on it
+      ph ^= 1ull << q;
+      if (group < 0) {  // STOP of one compute group
+        if (++stops == NG) break;
+        continue;
+      }
+      if (group >= p.nsub) continue;  // discard chunk: nobody waits on it
       if (group != cur && pend) {
         if (lane == 0) red_release_add(p.cnt + cur, pend);
         pend = 0;
@@ -580,17 +589,17 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
     }
     if (pend && lane == 0) red_release_add(p.cnt + cur, pend);
   } else {
-    // ------------------------------ compute warps ------------------------------
-    int s = 0;
-    unsigned ph = 0;
-    for (int k = 0;; ++k) {
-      ktd::mbar_wait(&s_full[s], (ph >> s) & 1u);
-      ph ^= 1u << s;
+    // ------------------------------ compute groups ------------------------------
+    const int cg = warp / PCOMP_WARPS, gtid = tid - cg * PCOMP_THREADS;
+    for (int k = cg;; k += NG) {
+      const int s = k % S;
+      ktd::mbar_wait(&s_full[s], (unsigned)(k / S) & 1u);
       const uint64_t d = s_desc[s];
       const uint64_t kind = d >> 60;
+      const int q = k & (PUBQ - 1);
       if (kind == PK_STOP) {
-        if (tid == 0) s_pub[k & (PUBQ - 1)] = -1;
-        mbar_arrive(&s_done[k & (PUBQ - 1)]);
+        if (gtid == 0) s_pub[q] = -1;
+        mbar_arrive(&s_done[q]);
         break;
       }
       const uint64_t tc0 = p.tb.rec ? gtimer() : 0;
@@ -598,37 +607,31 @@ __global__ void __launch_bounds__(PERSIST_THREADS, MINB) persistent_kernel(const
         const PChunk c = p.chunks[d & 0xFFFFFFFFFFull];
         const DRect& r = p.drects[c.d];
         const int64_t h = r.y1 - r.y0;
-        for (int64_t i = tid; i < c.n; i += PCOMP_THREADS) {
+        for (int64_t i = gtid; i < c.n; i += PCOMP_THREADS) {
           const int64_t j = c.l0 + i, row = j / r.lpr, l = j - row * r.lpr;
           const int64_t z = r.z0 + row / h, y = r.y0 + row % h;
           ktd::discard_line(r.base + z * r.fstride + y * r.pitch + r.lb0 + 128 * l);
         }
-        mbar_arrive(&s_empty[s]);
-        if (tid == 0) s_pub[k & (PUBQ - 1)] = (int32_t)((d >> 40) & 0xFFFFF);
-        mbar_arrive(&s_done[k & (PUBQ - 1)]);
       } else {
         const PNode& nd = s_nodes[kind];
         const ktd::Tile t = s_tile[s];
         uint8_t* buf = ktsm + s * p.stage_bytes;
         if (nd.scalar) {
-          ktd::scalar_tile(nd.op, nd.in, nd.out, t, nd.T, PCOMP_THREADS, tid);
+          ktd::scalar_tile(nd.op, nd.in, nd.out, t, nd.T, PCOMP_THREADS, gtid);
         } else {
           if ((nd.op == 1 || nd.op == 3) && ktd::needs_fix(nd.op, nd.in, t)) {
-            ktd::stage_fix(nd.op, nd.in, t, buf, PCOMP_THREADS, tid);
-            nbar_sync(1, PCOMP_THREADS);
+            ktd::stage_fix(nd.op, nd.in, t, buf, PCOMP_THREADS, gtid, 1 + NG + cg);
+            nbar_sync(1 + cg, PCOMP_THREADS);
           }
-          ktd::compute_tile(nd.op, nd.out, t, buf, nd.T, PCOMP_THREADS, tid);
+          ktd::compute_tile(nd.op, nd.out, t, buf, nd.T, PCOMP_THREADS, gtid);
         }
-        mbar_arrive(&s_empty[s]);  // this thread is done with the slot
-        if (tid == 0) {
-          if (p.tb.rec) trace_put(p.tb, d, 2, tc0, gtimer());
-          s_pub[k & (PUBQ - 1)] = (int32_t)((d >> 40) & 0xFFFFF);
-        }
-        // every compute thread arrives (release.cta) after its tile writes; the publisher
-        // acquires the completed phase before its gpu-scope release (cumulative)
-        mbar_arrive(&s_done[k & (PUBQ - 1)]);
+        if (p.tb.rec && gtid == 0) trace_put(p.tb, d, 2, tc0, gtimer());
       }
-      s = s + 1 == S ? 0 : s + 1;
+      mbar_arrive(&s_empty[s]);  // this thread is done with the slot
+      if (gtid == 0) s_pub[q] = ticket_group(d);
+      // every compute thread arrives (release.cta) after its tile writes; the publisher
+      // acquires the completed phase before its gpu-scope release (cumulative)
+      mbar_arrive(&s_done[q]);
     }
   }
   __syncthreads();
@@ -698,6 +701,8 @@ struct ktiler_plan_s {
   PParams pp{};
   int pctas = 0;
   int pminb = 2;
+  int pgroups = 1;
+  int pthreads = 0;
   int psmem = 0;
   void (*pfn)(PParams) = nullptr;
   int64_t skew = 0;
@@ -1286,37 +1291,52 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
   {
-    const char* ev = getenv("KTILER_PERSIST_MINB");
-    const int mb = ev ? atoi(ev) : PERSIST_MINB_DEFAULT;
-    P->pfn = mb >= 4 ? persistent_kernel<4> : (mb == 3 ? persistent_kernel<3> : persistent_kernel<2>);
-    P->pminb = mb >= 4 ? 4 : (mb == 3 ? 3 : 2);
+    // KTILER_PERSIST_GROUPS: compute groups per CTA (4 -> one CTA per SM; 2 -> two; 1 ->
+    // three single-group CTAs)
+    const char* ev = getenv("KTILER_PERSIST_GROUPS");
+    const int ng = ev ? atoi(ev) : PERSIST_GROUPS_DEFAULT;
+    if (ng >= 4) { P->pfn = persistent_kernel<4, 1>; P->pminb = 1; P->pgroups = 4; }
+    else if (ng == 2) { P->pfn = persistent_kernel<2, 2>; P->pminb = 2; P->pgroups = 2; }
+    else { P->pfn = persistent_kernel<1, 3>; P->pminb = 3; P->pgroups = 1; }
+    P->pthreads = P->pgroups * PCOMP_THREADS + 64;
   }
   int slot = 0;
   for (auto& n : g.nodes) {
     const kt::Access& w = n.acc[n.wacc];
     if (!n.scalar) slot = std::max(slot, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
   }
-  // ring depth: as many slots as fit the shared memory of MINB CTAs per SM (2..PSTAGES_MAX)
-  int smem_sm = 0;
+  // ring depth: as many slots as fit the shared memory of MINB CTAs per SM, a multiple of
+  // the compute groups (slot s always serves group s mod NG, so every waiter on a slot's
+  // barrier has consumed the slot's previous use itself: no parity aliasing)
+  int smem_sm = 0, smem_blk = 0;
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
-  const int per_cta = smem_sm / P->pminb - 2048;  // static smem + per-CTA reserve
-  int nslots = slot ? std::min(PSTAGES_MAX, std::max(2, per_cta / slot)) : 2;
-  if (const char* ev = getenv("KTILER_PERSIST_SLOTS")) nslots = std::min(PSTAGES_MAX, std::max(2, atoi(ev)));
+  cudaDeviceGetAttribute(&smem_blk, cudaDevAttrMaxSharedMemoryPerBlockOptin, P->device);
+  cudaFuncAttributes fa{};
+  cudaFuncGetAttributes(&fa, (const void*)P->pfn);
+  const int per_cta = std::min(smem_sm / P->pminb - 1024, smem_blk) - (int)fa.sharedSizeBytes;
+  const int ngr = P->pgroups;
+  int nslots = slot ? std::min(PSTAGES_MAX, std::max(2 * ngr, per_cta / slot)) : 2 * ngr;
+  if (const char* ev = getenv("KTILER_PERSIST_SLOTS")) nslots = std::min(PSTAGES_MAX, std::max(ngr, atoi(ev)));
+  nslots -= nslots % ngr;
   P->psmem = std::max(slot, 128) * nslots;
+  if (P->psmem + (int)fa.sharedSizeBytes > smem_blk)
+    return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: staging slots exceed shared memory");
   if (P->psmem > 48 * 1024) {
     cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
   }
   int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, P->pfn, PERSIST_THREADS, P->psmem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, P->pfn, P->pthreads, P->psmem);
   if (occ < 1) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: kernel does not fit an SM");
   P->pctas = P->pol.persistent_ctas > 0 ? std::min(P->pol.persistent_ctas, nsm * occ) : nsm * occ;
-  // Group order.  skew < 0: the emitted (fragment-major) order.  skew = k > 0: software
-  // pipeline over fragments — the sub-kernel of fragment f at node depth d is issued at
-  // step f + d*k, deepest node first within a step.  A consumer's producers sit in
-  // fragments <= f at smaller depth, hence at strictly earlier steps: still a valid total
-  // order, and k steps of other work separate a sub-kernel from its
-  // producers, so the dependency check rarely waits.
+  // Ticket order, in pipeline steps.  skew < 0: the emitted (fragment-major) order, one
+  // sub-kernel per step.  skew = k > 0: software pipeline over fragments — the
+  // sub-kernel of fragment f at node depth d runs in step f + d*k.  A consumer's
+  // producers sit in fragments <= f at smaller depth, hence in steps at least k earlier:
+  // still a valid total order, and the sub-kernels of one step never
+  // depend on each other, so their tiles are interleaved evenly (memory-bound and
+  // ALU-bound tiles of different fragments share every SM) and a step only waits for
+  // the step k before it.
   std::vector<int> depth(nn, 0);
   int dmax = 0;
   for (int v : g.topo)
@@ -1328,23 +1348,29 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   int64_t k = P->pol.pipeline_skew;
   if (k == 0) k = 1;
   P->skew = k;
-  std::vector<int> order;
+  const char* ie = getenv("KTILER_PERSIST_INTERLEAVE");
+  const bool interleave = k > 0 && (!ie || atoi(ie) != 0);
+  std::vector<std::vector<int>> steps;  // sub-kernels per step
+  std::vector<int> step_of(nsub, 0);
   if (k < 0) {
-    for (int i = 0; i < nsub; ++i) order.push_back(i);
+    for (int i = 0; i < nsub; ++i) steps.push_back({i});
   } else {
     std::vector<int> rtopo(g.topo.rbegin(), g.topo.rend());
-    for (int64_t st = 0; st < nfrag + dmax * k; ++st)
+    for (int64_t st = 0; st < nfrag + dmax * k; ++st) {
+      steps.emplace_back();
       for (int v : rtopo) {
         const int64_t f = st - depth[v] * k;
-        if (f >= 0 && f < nfrag && by_frag[f][v] >= 0) order.push_back(by_frag[f][v]);
+        if (f >= 0 && f < nfrag && by_frag[f][v] >= 0) steps.back().push_back(by_frag[f][v]);
       }
+    }
   }
-  // Discard lists (groups nsub + si): after the last of their readers, one pipeline step
-  // (nn sub-kernels) later so the readers have finished by the time the chunks are reached.
+  for (size_t st = 0; st < steps.size(); ++st)
+    for (int i : steps[st]) step_of[i] = (int)st;
+  // Discard lists (groups nsub + si): |skew| steps after the step of their last reader, so
+  // the readers have finished by the time the chunks are reached.
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
-  std::vector<int> pos(nsub, 0);
-  for (size_t i = 0; i < order.size(); ++i) pos[order[i]] = (int)i;
-  std::vector<std::vector<int>> disc_after(order.size() + 1);
+  const int dlag = (int)std::max<int64_t>(1, k < 0 ? nn : k);
+  std::vector<std::vector<int>> disc_in(steps.size() + dlag + 1);
   std::vector<DRect> drects;
   std::vector<std::vector<int>> drect_of(nsub);
   if (disc) {
@@ -1357,14 +1383,14 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
         drects.push_back(dr);
       }
       if (drect_of[si].empty()) continue;
-      int last = pos[si];
-      for (int r : S.discard_readers[si]) last = std::max(last, pos[r]);
-      disc_after[std::min<size_t>(order.size(), (size_t)last + (size_t)nn)].push_back(si);
+      int last = step_of[si];
+      for (int r : S.discard_readers[si]) last = std::max(last, step_of[r]);
+      disc_in[std::min<size_t>(disc_in.size() - 1, (size_t)last + dlag)].push_back(si);
     }
   }
-  // groups' dependency lists (CSR) and the tickets in global order
+  // groups' dependency lists (CSR)
   const int ngroups = 2 * nsub;
-  if (ngroups >= (1 << 20)) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: too many sub-kernels");
+  if (ngroups >= (1 << PGROUP_BITS)) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: too many sub-kernels");
   std::vector<int32_t> dep_off(ngroups + 1, 0);
   std::vector<PDep> deps;
   for (int gi = 0; gi < ngroups; ++gi) {
@@ -1372,34 +1398,63 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     for (int32_t u : src) deps.push_back(PDep{u, (uint32_t)S.subs[u].nblocks});
     dep_off[gi + 1] = (int32_t)deps.size();
   }
+  // the tickets in global order: per step, each member's tickets spread evenly over the
+  // step (key (j + 1/2) / n), discard chunks likewise
   std::vector<uint64_t> tickets;
   std::vector<PChunk> chunks;
   constexpr int64_t CHUNK_LINES = 2048;  // 256 KB of dead lines per discard ticket
-  auto emit_discards = [&](int si) {
-    for (int di : drect_of[si]) {
-      const DRect& r = drects[di];
-      const int64_t lines = r.lpr * (int64_t)(r.y1 - r.y0) * (r.z1 - r.z0);
-      for (int64_t l0 = 0; l0 < lines; l0 += CHUNK_LINES) {
-        tickets.push_back(pack_ticket(PK_DISCARD, (uint64_t)(nsub + si), chunks.size()));
-        chunks.push_back(PChunk{di, (int32_t)std::min(CHUNK_LINES, lines - l0), l0});
-      }
-    }
+  std::vector<std::pair<double, uint64_t>> keyed;
+  auto put = [&](std::vector<uint64_t>& v) {
+    const double n = (double)v.size();
+    for (size_t j = 0; j < v.size(); ++j) keyed.push_back({interleave ? (j + 0.5) / n : 0.0, v[j]});
   };
-  for (size_t i = 0; i <= order.size(); ++i) {
-    for (int si : disc_after[i]) emit_discards(si);
-    if (i == order.size()) break;
-    const kt::SubKernel& sk = S.subs[order[i]];
-    for (auto& r : sk.rects)
-      for (int64_t z = r.z0; z < r.z1; ++z)
-        for (int64_t y = r.y0; y < r.y1; ++y)
-          for (int64_t x = r.x0; x < r.x1; ++x)
-            tickets.push_back(pack_ticket((uint64_t)sk.node, (uint64_t)order[i], tile_payload(x, y, z)));
+  std::vector<uint64_t> tmp;
+  for (size_t st = 0; st < disc_in.size(); ++st) {
+    keyed.clear();
+    for (int si : disc_in[st]) {
+      tmp.clear();
+      for (int di : drect_of[si]) {
+        const DRect& r = drects[di];
+        const int64_t lines = r.lpr * (int64_t)(r.y1 - r.y0) * (r.z1 - r.z0);
+        for (int64_t l0 = 0; l0 < lines; l0 += CHUNK_LINES) {
+          tmp.push_back(pack_ticket(PK_DISCARD, (uint64_t)(nsub + si), chunks.size()));
+          chunks.push_back(PChunk{di, (int32_t)std::min(CHUNK_LINES, lines - l0), l0});
+        }
+      }
+      put(tmp);
+    }
+    if (st < steps.size())
+      for (int si : steps[st]) {
+        tmp.clear();
+        const kt::SubKernel& sk = S.subs[si];
+        for (auto& r : sk.rects)
+          for (int64_t z = r.z0; z < r.z1; ++z)
+            for (int64_t y = r.y0; y < r.y1; ++y)
+              for (int64_t x = r.x0; x < r.x1; ++x)
+                tmp.push_back(pack_ticket((uint64_t)sk.node, (uint64_t)si, tile_payload(x, y, z)));
+        put(tmp);
+      }
+    std::stable_sort(keyed.begin(), keyed.end(),
+                     [](const std::pair<double, uint64_t>& a, const std::pair<double, uint64_t>& b) { return a.first < b.first; });
+    for (auto& kv : keyed) tickets.push_back(kv.second);
   }
-  // per-CTA contiguous ticket lists (ticket i -> CTA i mod G, in order), STOP-padded
+  // per-CTA contiguous ticket lists (ticket i -> CTA i mod G, in order), STOP-padded; the
+  // first ticket of each group in a CTA's list carries PK_CHECK
   const int64_t G = P->pctas, T = (int64_t)tickets.size();
   const int64_t per = (T + G - 1) / G + 1;
   std::vector<uint64_t> desc((size_t)(G * per), pack_ticket(PK_STOP, 0, 0));
   for (int64_t i = 0; i < T; ++i) desc[(size_t)((i % G) * per + i / G)] = tickets[(size_t)i];
+  {
+    std::vector<int64_t> stamp(ngroups, -1);
+    for (int64_t c = 0; c < G; ++c)
+      for (int64_t j = 0; j < per; ++j) {
+        uint64_t& d = desc[(size_t)(c * per + j)];
+        if ((d >> 60) == PK_STOP) break;
+        const int gr = ticket_group(d);
+        if (stamp[gr] != c && dep_off[gr + 1] > dep_off[gr]) d |= PK_CHECK;
+        stamp[gr] = c;
+      }
+  }
   // one device allocation: ctrl | counters | dep_off | deps | drects | chunks | nodes | desc
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
   size_t o_ctrl = 0, o_cnt = al(sizeof(PCtrl)), o_doff = o_cnt + al((size_t)nsub * 4 + 4);
@@ -1612,7 +1667,7 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     case KTILER_EXEC_PERSISTENT: {
       cudaLaunchConfig_t cfg = {};
       cfg.gridDim = dim3((unsigned)p->pctas);
-      cfg.blockDim = dim3(PERSIST_THREADS);
+      cfg.blockDim = dim3((unsigned)p->pthreads);
       cfg.dynamicSmemBytes = (size_t)p->psmem;
       cfg.stream = st;
       if ((e = cudaLaunchKernelEx(&cfg, p->pfn, p->pp)) != cudaSuccess) return cuda_fail(e, "persistent launch");

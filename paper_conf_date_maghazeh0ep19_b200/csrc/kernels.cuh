@@ -228,7 +228,8 @@ __device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map,
 // columns < 0 / >= W from pixel 0 / W-1 of the same row, then rows < 0 / >= H as copies of
 // the nearest image row — so the staged window holds in[clamp(y)][clamp(x)].  All threads;
 // the caller synchronizes afterwards.  Returns quickly for interior tiles.
-__device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid) {
+__device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid,
+                                          int bar_id = 4) {
   if (op != 1 && op != 3) return;
   const StageGeo g = stage_geo(op, in, t);
   const int left = g.xb0 < 0 ? (int)(-g.xb0) : 0;                                       // columns < 0
@@ -246,7 +247,7 @@ __device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t,
     }
   }
   if (top || bfrom < g.nr) {
-    if (per) asm volatile("bar.sync 4, %0;" ::"r"(nt) : "memory");  // the nt staging threads only
+    if (per) asm volatile("bar.sync %0, %1;" ::"r"(bar_id), "r"(nt) : "memory");  // the nt staging threads only
     const int n16 = g.stride >> 4, nfix = top + (g.nr - bfrom);
     for (int i = tid; i < nfix * n16; i += nt) {
       const int j = i / n16, c = i % n16;

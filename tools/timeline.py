@@ -124,6 +124,11 @@ def summarise(rec, launches, pix):
             out["ctl_us_p90"] = round(float(np.percentile(c, 90)) / 1e3, 3)
             cn = (k1["id"] >> np.uint64(60)).astype(np.int64)
             out["ctl_us_by_node"] = {NODES[v]: round(float(c[cn == v].mean()) / 1e3, 3) for v in sorted(set(cn.tolist()))}
+            # staging issued -> compute start, per node (TMA latency + queueing behind earlier tiles)
+            i1 = {int(i): int(t) for i, t in zip(k1["id"], k1["t1"])}
+            lat = np.array([t - i1.get(int(i), t) for i, t in zip(k2["id"], k2["t0"])], dtype=np.int64)
+            out["issue_to_start_us_by_node"] = {NODES[v]: [round(float(np.percentile(lat[node == v], q)) / 1e3, 2)
+                                                           for q in (10, 50, 90)] for v in sorted(set(node.tolist()))}
         # per SM: idle between consecutive compute intervals (all CTAs of the SM merged)
         sm = k2["smid"].astype(np.int64)
         idle = []
