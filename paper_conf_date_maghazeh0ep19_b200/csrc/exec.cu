@@ -35,7 +35,7 @@ constexpr int MAXR = 4, MAXD = 8;
 constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+ producer + publisher warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
 constexpr int PSTAGES_MAX = 12;   // staging ring depth (slots that fit the CTA's share of smem)
-constexpr int PERSIST_GROUPS_DEFAULT = 4;
+constexpr int PERSIST_GROUPS_DEFAULT = 2;
 constexpr int PMAX_NODES = 8;
 
 struct LRect {
@@ -1349,7 +1349,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   if (k == 0) k = 1;
   P->skew = k;
   const char* ie = getenv("KTILER_PERSIST_INTERLEAVE");
-  const bool interleave = k > 0 && (!ie || atoi(ie) != 0);
+  const bool interleave = k > 0 && ie && atoi(ie) != 0;  // opt-in: mixed ops thrash the instruction cache
   std::vector<std::vector<int>> steps;  // sub-kernels per step
   std::vector<int> step_of(nsub, 0);
   if (k < 0) {

@@ -36,7 +36,7 @@ def main():
     pix = W * H * F
     cfgs = [dict(kind="none", exec_mode="graph"), dict(kind="budget", l2_fraction=1.0, exec_mode="dag", discard=True)]
     for fr in (0.5, 1.0):
-        for mode in ("graph", "dag"):
+        for mode in ("graph", "dag", "persistent"):
             for rb in (False, True):
                 cfgs.append(dict(kind="alg1", l2_fraction=fr, exec_mode=mode, discard=True, resident_budget=rb))
     for c in cfgs:
