@@ -370,7 +370,7 @@ struct PNode {
   float T;
 };
 struct PCtrl {
-  unsigned int done, epoch, pad0, pad1;
+  unsigned int done, epoch, ticket, pad1;  // ticket: next unclaimed ticket (dynamic mode)
 };
 struct PDep {
   int32_t sub;       // counter index (= sub-kernel id)
@@ -397,7 +397,8 @@ __host__ __device__ inline uint64_t tile_payload(uint64_t bx, uint64_t by, uint6
 struct PParams {
   const PNode* nodes;
   const uint64_t* desc;     // [G][per_cta] tickets, STOP-padded
-  int64_t per_cta;
+  int64_t per_cta;          // static: tickets per CTA list; dynamic: 0
+  int64_t total;            // dynamic: tickets in the global order
   const int32_t* dep_off;   // CSR over groups
   const PDep* deps;
   const DRect* drects;
@@ -482,6 +483,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* m, unsigned parity) {
 // tiles from its own queue (PUBQ entries, s_done barriers); the producer keeps at most
 // PUBQ - PSTAGES_MAX tickets ahead of it, so a queue entry is never reused early.
 constexpr int PUBQ = 64;
+constexpr int DYN_B = 2;  // tickets per claim (dynamic mode)
 template <int NG, int MINB>
 __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kernel(const __grid_constant__ PParams p) {
   __shared__ __align__(8) uint64_t s_full[PSTAGES_MAX];
@@ -493,9 +495,11 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
   __shared__ volatile int32_t s_pubk;      // tickets the publisher has consumed
   __shared__ __align__(64) PNode s_nodes[PMAX_NODES];
   __shared__ unsigned int s_epoch;
+  __shared__ int32_t s_okg[64];
   extern __shared__ __align__(128) uint8_t ktsm[];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int S = p.nslots;
+  if (tid < 64) s_okg[tid] = -1;
   for (int i = tid; i < p.nnodes * (int)(sizeof(PNode) / 4); i += blockDim.x)
     reinterpret_cast<uint32_t*>(s_nodes)[i] = reinterpret_cast<const uint32_t*>(p.nodes)[i];
   if (tid == 0) {
@@ -516,9 +520,22 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
     int s = 0, stops = 0;
     unsigned ph = 0;  // bit s: parity of slot s's current use
     uint64_t batch = 0;
+    const bool dyn = p.per_cta == 0;
+    // dynamic: chunks of DYN_B consecutive tickets claimed from the global counter; the
+    // claim of the next chunk is issued when a chunk starts, so its latency overlaps it
+    unsigned next = 0;
+    if (dyn && lane == 0) next = atomicAdd(&p.ctrl->ticket, (unsigned)DYN_B);
     for (int64_t k = 0;; ++k) {
-      if ((k & 31) == 0) batch = k + lane < p.per_cta ? my[k + lane] : pack_ticket(PK_STOP, 0, 0);
-      const uint64_t d = __shfl_sync(FULL, batch, (int)(k & 31));
+      if (dyn) {
+        if ((k % DYN_B) == 0) {
+          const unsigned base = __shfl_sync(FULL, next, 0);
+          if (lane == 0 && base < p.total) next = atomicAdd(&p.ctrl->ticket, (unsigned)DYN_B);
+          batch = lane < DYN_B && (int64_t)base + lane < p.total ? p.desc[base + lane] : pack_ticket(PK_STOP, 0, 0);
+        }
+      } else if ((k & 31) == 0) {
+        batch = k + lane < p.per_cta ? my[k + lane] : pack_ticket(PK_STOP, 0, 0);
+      }
+      const uint64_t d = __shfl_sync(FULL, batch, dyn ? (int)(k % DYN_B) : (int)(k & 31));
       if (k >= S) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
       while ((int)k - s_pubk > PUBQ - PSTAGES_MAX) __nanosleep(200);  // publisher queue bound
       const uint64_t kind = d >> 60;
@@ -534,7 +551,16 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
         continue;
       }
       const uint64_t tq0 = p.tb.rec ? gtimer() : 0;
-      if (d & PK_CHECK) wait_group(p, ticket_group(d), epoch, lane);
+      if (d & PK_CHECK) {
+        wait_group(p, ticket_group(d), epoch, lane);
+      } else if (dyn) {  // dynamic: a small cache of groups already verified by this CTA
+        const int gr = ticket_group(d);
+        if (s_okg[gr & 63] != gr) {
+          wait_group(p, gr, epoch, lane);
+          if (lane == 0) s_okg[gr & 63] = gr;
+          __syncwarp();
+        }
+      }
       if (lane == 0) {
         s_desc[s] = d;
         if (kind == PK_DISCARD) {
@@ -640,6 +666,7 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
     unsigned int old = atomicAdd(&p.ctrl->done, 1u);
     if (old == gridDim.x - 1) {
       p.ctrl->done = 0;
+      p.ctrl->ticket = 0;
       __threadfence();
       atomicAdd(&p.ctrl->epoch, 1u);
     }
@@ -1438,13 +1465,21 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
                      [](const std::pair<double, uint64_t>& a, const std::pair<double, uint64_t>& b) { return a.first < b.first; });
     for (auto& kv : keyed) tickets.push_back(kv.second);
   }
-  // per-CTA contiguous ticket lists (ticket i -> CTA i mod G, in order), STOP-padded; the
-  // first ticket of each group in a CTA's list carries PK_CHECK
+  // Static: per-CTA contiguous ticket lists (ticket i -> CTA i mod G, in order),
+  // STOP-padded; the first ticket of each group in a CTA's list carries PK_CHECK.
+  // Dynamic (default; KTILER_PERSIST_DYNAMIC=0 for static): the global order as is; CTAs claim chunks of it
+  // from an atomic counter (load balance), checking dependencies through a group cache.
   const int64_t G = P->pctas, T = (int64_t)tickets.size();
-  const int64_t per = (T + G - 1) / G + 1;
-  std::vector<uint64_t> desc((size_t)(G * per), pack_ticket(PK_STOP, 0, 0));
-  for (int64_t i = 0; i < T; ++i) desc[(size_t)((i % G) * per + i / G)] = tickets[(size_t)i];
-  {
+  const char* dy = getenv("KTILER_PERSIST_DYNAMIC");
+  const bool dynamic = !dy || atoi(dy) != 0;  // default on: load-balanced claims
+  if (T >= (1ll << 31)) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: more than 2^31 tickets");
+  const int64_t per = dynamic ? 0 : (T + G - 1) / G + 1;
+  std::vector<uint64_t> desc;
+  if (dynamic) {
+    desc = tickets;
+  } else {
+    desc.assign((size_t)(G * per), pack_ticket(PK_STOP, 0, 0));
+    for (int64_t i = 0; i < T; ++i) desc[(size_t)((i % G) * per + i / G)] = tickets[(size_t)i];
     std::vector<int64_t> stamp(ngroups, -1);
     for (int64_t c = 0; c < G; ++c)
       for (int64_t j = 0; j < per; ++j) {
@@ -1465,7 +1500,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   cudaError_t e = cudaMalloc(&d, total);
   if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (persistent tables)");
   P->dmem = d;
-  PCtrl c0{0, 1, 0, 0};
+  PCtrl c0{0, 1, 0, 0};  // done, epoch, ticket
   if ((e = cudaMemset(d, 0, total)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
   cudaMemcpy(d + o_ctrl, &c0, sizeof(c0), cudaMemcpyHostToDevice);
   cudaMemcpy(d + o_doff, dep_off.data(), dep_off.size() * 4, cudaMemcpyHostToDevice);
@@ -1478,6 +1513,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   P->pp.nodes = (const PNode*)(d + o_nodes);
   P->pp.desc = (const uint64_t*)(d + o_desc);
   P->pp.per_cta = per;
+  P->pp.total = T;
   P->pp.dep_off = (const int32_t*)(d + o_doff);
   P->pp.deps = (const PDep*)(d + o_deps);
   P->pp.drects = (const DRect*)(d + o_dr);
