@@ -1393,10 +1393,14 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   }
   for (size_t st = 0; st < steps.size(); ++st)
     for (int i : steps[st]) step_of[i] = (int)st;
-  // Discard lists (groups nsub + si): |skew| steps after the step of their last reader, so
-  // the readers have finished by the time the chunks are reached.
+  // Discard lists (groups nsub + si): at the end of the step of their last reader, after
+  // the step's source tiles (deepest node first: the readers come early in the step), or
+  // nn sub-kernels later in fragment-major order.  Measured on B200: the L2 writes dirty
+  // lines back on its own within microseconds, so a discard a whole step late saves
+  // nothing — dead lines must go as soon as their readers are done.
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
-  const int dlag = (int)std::max<int64_t>(1, k < 0 ? nn : k);
+  const char* dl = getenv("KTILER_PERSIST_DLAG");
+  const int dlag = k < 0 ? nn : (dl ? atoi(dl) : 0);
   std::vector<std::vector<int>> disc_in(steps.size() + dlag + 1);
   std::vector<DRect> drects;
   std::vector<std::vector<int>> drect_of(nsub);
@@ -1438,6 +1442,19 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   std::vector<uint64_t> tmp;
   for (size_t st = 0; st < disc_in.size(); ++st) {
     keyed.clear();
+    if (st < steps.size())
+      for (int si : steps[st]) {
+        tmp.clear();
+        const kt::SubKernel& sk = S.subs[si];
+        for (auto& r : sk.rects)
+          for (int64_t z = r.z0; z < r.z1; ++z)
+            for (int64_t y = r.y0; y < r.y1; ++y)
+              for (int64_t x = r.x0; x < r.x1; ++x)
+                tmp.push_back(pack_ticket((uint64_t)sk.node, (uint64_t)si, tile_payload(x, y, z)));
+        put(tmp);
+      }
+    // the step's discard chunks after its tiles (non-interleaved): the lines die as soon
+    // as possible while the readers (a step earlier) have had a whole step to finish
     for (int si : disc_in[st]) {
       tmp.clear();
       for (int di : drect_of[si]) {
@@ -1450,17 +1467,6 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
       }
       put(tmp);
     }
-    if (st < steps.size())
-      for (int si : steps[st]) {
-        tmp.clear();
-        const kt::SubKernel& sk = S.subs[si];
-        for (auto& r : sk.rects)
-          for (int64_t z = r.z0; z < r.z1; ++z)
-            for (int64_t y = r.y0; y < r.y1; ++y)
-              for (int64_t x = r.x0; x < r.x1; ++x)
-                tmp.push_back(pack_ticket((uint64_t)sk.node, (uint64_t)si, tile_payload(x, y, z)));
-        put(tmp);
-      }
     std::stable_sort(keyed.begin(), keyed.end(),
                      [](const std::pair<double, uint64_t>& a, const std::pair<double, uint64_t>& b) { return a.first < b.first; });
     for (auto& kv : keyed) tickets.push_back(kv.second);
