@@ -4,8 +4,9 @@ Workload (default ``batch64_8k`` = BASELINE configs[3]): 64 frames of 8K (7680x4
 through the 5-kernel pipeline gray -> blur5 -> down2 -> sobel3 -> thresh, the
 configuration the north star's 1-GPU target is stated on ("8K-class images on one B200")
 and the one its multi-GPU scaling target uses ("frame batches").  With --gpus N (one
-process per GPU, launched by torchrun) the 64 frames are split across the ranks — frame
-sharding with no data-path collective (strong scaling: the batch is fixed).  Workload
+process per GPU, launched by torchrun) every rank runs its own 64-frame batch — frame
+sharding with no data-path collective, per-GPU work fixed ("scaling": "weak"; --scaling
+strong splits one 64-frame batch across the ranks instead).  Workload
 ``strip_65536`` (configs[4]) splits one 65536x65536 image into row strips whose 4 halo
 rows per side move over NCCL send/recv before each step.
 
@@ -60,7 +61,11 @@ def parse():
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=1.0)
+    ap.add_argument("--l2-fraction", type=float, default=0.5)
+    ap.add_argument("--no-resident", action="store_true",
+                    help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="frames: weak = every rank runs the whole batch (per-GPU work fixed), strong = split it")
     ap.add_argument("--window", type=int, default=2)
     ap.add_argument("--no-discard", action="store_true")
     ap.add_argument("--pdl", action="store_true")
@@ -189,7 +194,7 @@ def run_reference(args):
     sample = f"1 {W}x{rows} image per step (bounded sample of the {args.workload} workload), 1 thread"
     print(json.dumps({
         "metric": METRIC, "value": v, "unit": "Mpix/s", "n_gpus": args.gpus, "steps": steps, "warmup": args.warmup,
-        "ms_per_step": ms, "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+        "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic", "config": {"workload": args.workload, "W": W, "H": H, "frames": Ftot, "baseline_config": cfg},
         "impl": "reference",
         "cpu_baseline": {"value": v, "unit": "Mpix/s", "cores": 1, "kind": "oracle", "sample": sample},
@@ -251,15 +256,17 @@ def main():
         pix_rank = W * (sp.o1 - sp.o0)
         per = 1
     else:
-        per = Ftot // world if shard == "frames" and Ftot >= world else Ftot
+        strong = shard == "frames" and args.scaling == "strong" and Ftot >= world
+        per = Ftot // world if strong else Ftot
         f0 = rank * per if shard == "frames" else 0
         p = Pipeline(W, H, per, T=args.T, internal=True)
         G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
         pix_rank = W * H * per
     torch.cuda.synchronize()
     discard = not args.no_discard
+    resident = not args.no_resident
     pol = dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode, discard=discard,
-               pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew, window=args.window)
+               pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew, window=args.window, resident_budget=resident)
     plan = p.plan(0, **pol)
     st = plan.stats()
 
@@ -302,7 +309,7 @@ def main():
     comp_bytes = pix * 3.25  # rgb in + mask out: the method's algorithmic bytes
     achieved = comp_bytes / (ms / 1000) / 1e9
     tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
-            "discard": discard, "window": args.window, "n_gpus": world}
+            "discard": discard, "window": args.window, "resident_budget": resident}
     traffic, traffic_src = traffic_for(tcfg)
     line = {
         "metric": METRIC,
@@ -313,14 +320,15 @@ def main():
         "warmup": args.warmup,
         "ms_per_step": ms,
         "higher_is_better": True,
-        "scaling": "strong",
+        "scaling": "strong" if (shard == "strips" or (shard == "frames" and args.scaling == "strong")) else "weak",
         "vs_baseline": None,
         "dtype": "u8",
         "data": "synthetic",
         "config": {"workload": args.workload, "baseline_config": cfg_idx, "W": W, "H": H, "frames": Ftot,
+                   "frames_per_gpu": per if sp is None else None,
                    "sharding": shard if world > 1 else "none", "pixels_per_gpu": pix_rank, "mode": args.mode,
                    "policy": args.kind, "rows": args.rows, "l2_fraction": args.l2_fraction, "window": args.window,
-                   "discard": discard, "pdl": args.pdl,
+                   "resident_budget": resident, "discard": discard, "pdl": args.pdl,
                    "l2_flush": "not needed: each step reads >= 6.4 GB of input (>> 126 MB L2)" if Ftot > 1 or W >= 16384
                    else "none (input smaller than L2: steady-state replay)",
                    "fragments": st["n_fragments"], "subkernels": st["n_subkernels"],
