@@ -674,6 +674,40 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
 }
 
 // ------------------------------------------------------------------------------------
+// footprint discovery (ktiler_discover_footprint): fill / perturb / compare kernels
+// ------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t disc_hash(uint64_t x) {
+  x += 0x9E3779B97F4A7C15ull;
+  x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+  x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+  return (uint32_t)(x ^ (x >> 31));
+}
+// byte i of a region = 1 + hash % 254 (never 0 or 255: a {0,255}-valued output always
+// differs from the fill, so no written byte hides behind an equal fill value)
+__global__ void disc_fill_kernel(uint8_t* p, int64_t n, uint64_t salt) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = (uint8_t)(1 + disc_hash(salt ^ ((uint64_t)i * 0x100000001B3ull)) % 254);
+}
+// bytes [a, b) of a region: XOR with a nonzero hash byte (every byte changes)
+__global__ void disc_perturb_kernel(uint8_t* p, int64_t a, int64_t b, uint64_t salt) {
+  for (int64_t i = a + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < b; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] ^= (uint8_t)(1 + disc_hash(salt ^ ((uint64_t)i * 0x100000001B3ull)) % 255);
+}
+// written |= (cur != snap)
+__global__ void disc_diff_kernel(const uint8_t* cur, const uint8_t* snap, uint8_t* written, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    written[i] |= (uint8_t)(cur[i] != snap[i]);
+}
+// *flag |= any byte with written != 0 differs between cur and ref
+__global__ void disc_cmp_kernel(const uint8_t* cur, const uint8_t* ref, const uint8_t* written, int64_t n,
+                                unsigned int* flag) {
+  unsigned int d = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    d |= (unsigned int)(written[i] && cur[i] != ref[i]);
+  if (__syncthreads_or((int)d) && threadIdx.x == 0) atomicOr(flag, 1u);
+}
+
+// ------------------------------------------------------------------------------------
 
 // ------------------------------------------------------------------------------------
 // host side
@@ -1912,6 +1946,163 @@ ktiler_status ktiler_calibrate(ktiler_graph_t gh, int32_t node, int32_t npts, co
   cudaFree(flush);
   if (rs) return rs;
   if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "calibration");
+  kt::clear_error();
+  return KTILER_OK;
+}
+
+ktiler_status ktiler_discover_footprint(ktiler_graph_t gh, int32_t node, int32_t bx, int32_t by, int32_t bz,
+                                        int32_t trials, uint64_t seed, ktiler_footprint_rec* out, int32_t cap,
+                                        int32_t* n_out) {
+  if (!gh || !n_out || trials < 1) return fail(KTILER_E_INVALID, "bad argument");
+  kt::Graph* G = kt::graph_of(gh);
+  ktiler_status s = G->finalize();
+  if (s) return s;
+  if (node < 0 || node >= (int)G->nodes.size()) return fail(KTILER_E_INVALID, "node out of range");
+  const kt::Node& nd = G->nodes[node];
+  if (bx < 0 || by < 0 || bz < 0 || bx >= nd.gx() || by >= nd.gy() || bz >= nd.gz())
+    return fail(KTILER_E_INVALID, "block out of the node's grid");
+  // the candidate space: every byte of every buffer (nothing of the declared accesses is used)
+  const int nb = (int)G->bufs.size();
+  std::vector<int64_t> off(nb + 1, 0);
+  for (int b = 0; b < nb; ++b) {
+    if (G->bufs[b].addr % 128) return fail(KTILER_E_INVALID, "footprint discovery needs 128-B aligned buffers");
+    off[b + 1] = off[b] + ((G->bufs[b].span + 127) & ~(int64_t)127);
+  }
+  const int64_t total = off[nb];
+  if (total > ((int64_t)1 << 30)) return fail(KTILER_E_UNSUPPORTED, "footprint discovery: graph buffers exceed 1 GiB");
+  ktiler_plan_s P;  // launch context (STREAM semantics)
+  P.g = *G;
+  P.pol.exec_mode = KTILER_EXEC_STREAM;
+  cudaError_t e = cudaGetDevice(&P.device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  uint8_t *snap = nullptr, *ref = nullptr, *wr = nullptr;
+  unsigned int* flag = nullptr;
+  if ((e = cudaMalloc(&snap, (size_t)total)) != cudaSuccess || (e = cudaMalloc(&ref, (size_t)total)) != cudaSuccess ||
+      (e = cudaMalloc(&wr, (size_t)total)) != cudaSuccess || (e = cudaMalloc(&flag, 4)) != cudaSuccess) {
+    cudaFree(snap); cudaFree(ref); cudaFree(wr);
+    return cuda_fail(e, "cudaMalloc (footprint discovery)");
+  }
+  cudaStream_t st = nullptr;
+  cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  auto bufp = [&](int b) { return (uint8_t*)G->bufs[b].d.base; };
+  auto span = [&](int b) { return G->bufs[b].span; };
+  auto copy_all = [&](uint8_t* dst, bool to_buffers) {
+    for (int b = 0; b < nb; ++b)
+      if (to_buffers) cudaMemcpyAsync(bufp(b), dst + off[b], (size_t)span(b), cudaMemcpyDeviceToDevice, st);
+      else cudaMemcpyAsync(dst + off[b], bufp(b), (size_t)span(b), cudaMemcpyDeviceToDevice, st);
+  };
+  // one launch of the single block, through the same launcher as every schedule
+  kt::SubKernel sk;
+  sk.node = node;
+  sk.rects.push_back({bx, by, bz, bx + 1, by + 1, bz + 1});
+  sk.nblocks = 1;
+  P.s.subs.push_back(sk);
+  P.s.discards.resize(1);
+  P.s.nfrag = 1;
+  build_launches(&P);
+  for (auto& L : P.launches)
+    if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar && L.kp.stage_bytes) {
+      L.n = &P.g.nodes[L.node];
+      L.kp.use_tmap = make_tmap(P.g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
+    }
+  ktiler_status rs = KTILER_OK;
+  auto run_block = [&]() { if (!rs) rs = enqueue(&P, st); };
+  // 1. writes: union over `trials` independent fills of the bytes the block changed
+  cudaMemsetAsync(wr, 0, (size_t)total, st);
+  for (int t = 0; t < trials && !rs; ++t) {
+    for (int b = 0; b < nb; ++b)
+      disc_fill_kernel<<<256, 256, 0, st>>>(bufp(b), span(b), seed * 0x9E3779B97F4A7C15ull + (uint64_t)t * 1000003u + (uint64_t)b);
+    copy_all(snap, false);
+    run_block();
+    for (int b = 0; b < nb && !rs; ++b) disc_diff_kernel<<<256, 256, 0, st>>>(bufp(b), snap + off[b], wr + off[b], span(b));
+  }
+  // 2. reads: reference = trial-0 fill (snap) and its output (ref); probe(lines [a, b) of the
+  //    concatenated line space) = restore, perturb those lines, run, compare on the written bytes
+  for (int b = 0; b < nb; ++b)
+    disc_fill_kernel<<<256, 256, 0, st>>>(bufp(b), span(b), seed * 0x9E3779B97F4A7C15ull + (uint64_t)b);
+  copy_all(snap, false);
+  run_block();
+  copy_all(ref, false);
+  std::vector<int64_t> loff(nb + 1, 0);
+  for (int b = 0; b < nb; ++b) loff[b + 1] = loff[b] + (off[b + 1] - off[b]) / 128;
+  uint64_t probe_salt = seed ^ 0xD1B54A32D192ED03ull;
+  auto probe = [&](int64_t la, int64_t lb) -> bool {
+    copy_all(snap, true);
+    for (int b = 0; b < nb; ++b) {
+      const int64_t a = std::max(la, loff[b]), c = std::min(lb, loff[b + 1]);
+      if (a >= c) continue;
+      const int64_t ba = (a - loff[b]) * 128, bb = std::min((c - loff[b]) * 128, span(b));
+      if (ba < bb) disc_perturb_kernel<<<64, 256, 0, st>>>(bufp(b), ba, bb, probe_salt);
+    }
+    probe_salt = probe_salt * 6364136223846793005ull + 1442695040888963407ull;
+    run_block();
+    cudaMemsetAsync(flag, 0, 4, st);
+    for (int b = 0; b < nb; ++b)
+      disc_cmp_kernel<<<128, 256, 0, st>>>(bufp(b), ref + off[b], wr + off[b], span(b), flag);
+    unsigned int h = 0;
+    cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    return h != 0;
+  };
+  std::vector<int64_t> read_lines;
+  std::vector<std::pair<int64_t, int64_t>> stack{{0, loff[nb]}};
+  while (!stack.empty() && !rs) {
+    auto [a, b] = stack.back();
+    stack.pop_back();
+    if (!probe(a, b)) continue;
+    if (b - a == 1) {
+      read_lines.push_back(a);
+    } else {
+      const int64_t m = a + (b - a) / 2;
+      stack.push_back({m, b});
+      stack.push_back({a, m});
+    }
+  }
+  std::vector<uint8_t> hw((size_t)total);
+  if (!rs) {
+    cudaMemcpyAsync(hw.data(), wr, (size_t)total, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+  }
+  e = cudaGetLastError();
+  cudaFree(snap); cudaFree(ref); cudaFree(wr); cudaFree(flag);
+  cudaStreamDestroy(st);
+  if (rs) return rs;
+  if (e != cudaSuccess) return cuda_fail(e, "footprint discovery");
+  // records: runs of written bytes, runs of read lines (as bytes), per buffer
+  std::vector<ktiler_footprint_rec> rec;
+  for (int b = 0; b < nb; ++b)
+    for (int64_t i = 0; i < span(b);) {
+      if (!hw[(size_t)(off[b] + i)]) { ++i; continue; }
+      int64_t j = i;
+      while (j < span(b) && hw[(size_t)(off[b] + j)]) ++j;
+      rec.push_back({b, KTILER_WRITE, i, j});
+      i = j;
+    }
+  std::sort(read_lines.begin(), read_lines.end());
+  for (size_t i = 0; i < read_lines.size();) {
+    size_t j = i + 1;
+    while (j < read_lines.size() && read_lines[j] == read_lines[j - 1] + 1) ++j;
+    int b = 0;
+    while (read_lines[i] >= loff[b + 1]) ++b;
+    const int64_t first = (read_lines[i] - loff[b]) * 128;
+    const int64_t last = std::min((read_lines[j - 1] - loff[b] + 1) * 128, span(b));
+    // a run never crosses buffers: split where it does
+    int64_t k = (int64_t)i;
+    while (k < (int64_t)j) {
+      int bb = 0;
+      while (read_lines[k] >= loff[bb + 1]) ++bb;
+      int64_t e2 = k;
+      while (e2 + 1 < (int64_t)j && read_lines[e2 + 1] < loff[bb + 1]) ++e2;
+      rec.push_back({bb, KTILER_READ, (read_lines[k] - loff[bb]) * 128,
+                     std::min((read_lines[e2] - loff[bb] + 1) * 128, span(bb))});
+      k = e2 + 1;
+    }
+    (void)first; (void)last;
+    i = j;
+  }
+  *n_out = (int32_t)rec.size();
+  if (out)
+    for (int32_t k = 0; k < cap && k < (int32_t)rec.size(); ++k) out[k] = rec[k];
   kt::clear_error();
   return KTILER_OK;
 }

@@ -77,6 +77,10 @@ class SubKernelInfo(ctypes.Structure):
                 ("n_rects", ctypes.c_int32), ("cluster", ctypes.c_int32), ("footprint_bytes", ctypes.c_int64)]
 
 
+class FootprintRec(ctypes.Structure):
+    _fields_ = [("buf_id", ctypes.c_int32), ("mode", ctypes.c_int32), ("first", ctypes.c_int64), ("last", ctypes.c_int64)]
+
+
 class PlanStats(ctypes.Structure):
     _fields_ = [("n_subkernels", ctypes.c_int64), ("n_fragments", ctypes.c_int64), ("n_launches", ctypes.c_int64),
                 ("n_discard_lines", ctypes.c_int64), ("budget_bytes", ctypes.c_int64),
@@ -100,7 +104,7 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
            "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
            "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest", "ktiler_plan_num_clusters",
-           "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate"]
+           "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint"]
 
 _LIB = None
 
@@ -142,6 +146,7 @@ def lib() -> ctypes.CDLL:
         "ktiler_plan_get_cluster": ([vp, i32, P(i32), i32, P(i32), P(ctypes.c_double)], st),
         "ktiler_set_perf_table": ([vp, i32, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double)], st),
         "ktiler_calibrate": ([vp, i32, i32, P(i64), i32, P(ctypes.c_double), P(ctypes.c_double)], st),
+        "ktiler_discover_footprint": ([vp, i32, i32, i32, i32, i32, ctypes.c_uint64, P(FootprintRec), i32, P(i32)], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -231,6 +236,15 @@ class Graph:
         n = len(nblocks)
         _check(lib().ktiler_set_perf_table(self._h, node, n, (ctypes.c_int64 * n)(*nblocks),
                                            (ctypes.c_double * n)(*ms_cold), (ctypes.c_double * n)(*ms_hot)))
+
+    def discover_footprint(self, node: int, bx: int, by: int, bz: int = 0, trials: int = 3, seed: int = 1):
+        """Dependency footprint of one block by differential execution (include/ktiler.h,
+        SURVEY §8(f) f3) -> list of (buf_id, mode, first_byte, last_byte_exclusive)."""
+        n = ctypes.c_int32()
+        _check(lib().ktiler_discover_footprint(self._h, node, bx, by, bz, trials, seed, None, 0, ctypes.byref(n)))
+        arr = (FootprintRec * max(1, n.value))()
+        _check(lib().ktiler_discover_footprint(self._h, node, bx, by, bz, trials, seed, arr, n.value, ctypes.byref(n)))
+        return [(r.buf_id, r.mode, r.first, r.last) for r in arr[:n.value]]
 
     def calibrate(self, node: int, nblocks, reps: int = 5):
         """Measure a node's performance table on the current device -> (cold, hot) lists (ms)."""

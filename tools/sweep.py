@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--F", type=int, default=64)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--configs", default="default", help="default | json list of plan kwargs")
+    ap.add_argument("--geom", default="", help='json {op: [tile_w, tile_h, threads]} overriding B200_GEOMETRY')
     args = ap.parse_args()
     import torch
 
@@ -28,7 +29,12 @@ def main():
     from inputs import gpu as G
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
     ge.build()
-    p = Pipeline(args.W, args.H, args.F, internal=True)
+    geom = None
+    if args.geom:
+        from paper_conf_date_maghazeh0ep19_b200.pipeline import B200_GEOMETRY
+        geom = dict(B200_GEOMETRY)
+        geom.update({k: tuple(v) for k, v in json.loads(args.geom).items()})
+    p = Pipeline(args.W, args.H, args.F, internal=True, geometry=geom)
     s = torch.cuda.current_stream()
     G.fill("scene", 1234, p.view("rgb").data_ptr(), args.W * 3, args.W * 3 * args.H, args.W, args.H, F=args.F,
            stream=s.cuda_stream)
@@ -58,7 +64,7 @@ def main():
                 ts.append(e0.elapsed_time(e1))
             ms = statistics.median(ts)
             st = pl.stats()
-            print(json.dumps({"cfg": c, "minb": os.environ.get("KTILER_PERSIST_MINB", "default"), "ms": round(ms, 4),
+            print(json.dumps({"cfg": c, "geom": args.geom or "default", "minb": os.environ.get("KTILER_PERSIST_MINB", "default"), "ms": round(ms, 4),
                               "Mpix/s": round(pix / ms / 1e3, 1), "fragments": st["n_fragments"],
                               "launches": st["n_launches"]}), flush=True)
             del pl
