@@ -2026,7 +2026,8 @@ ktiler_status ktiler_discover_footprint(ktiler_graph_t gh, int32_t node, int32_t
   std::vector<int64_t> loff(nb + 1, 0);
   for (int b = 0; b < nb; ++b) loff[b + 1] = loff[b] + (off[b + 1] - off[b]) / 128;
   uint64_t probe_salt = seed ^ 0xD1B54A32D192ED03ull;
-  auto probe = [&](int64_t la, int64_t lb) -> bool {
+  // one perturbation of lines [la, lb): does any written byte change?
+  auto probe1 = [&](int64_t la, int64_t lb) -> bool {
     copy_all(snap, true);
     for (int b = 0; b < nb; ++b) {
       const int64_t a = std::max(la, loff[b]), c = std::min(lb, loff[b + 1]);
@@ -2043,6 +2044,14 @@ ktiler_status ktiler_discover_footprint(ktiler_graph_t gh, int32_t node, int32_t
     cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
     return h != 0;
+  };
+  // a set is independent only if `trials` independent random perturbations all leave the
+  // written bytes unchanged (a single one can cancel out through the kernel's arithmetic,
+  // e.g. opposite changes of two taps of a filter)
+  auto probe = [&](int64_t la, int64_t lb) -> bool {
+    for (int t = 0; t < std::max(2, trials); ++t)
+      if (probe1(la, lb)) return true;
+    return false;
   };
   std::vector<int64_t> read_lines;
   std::vector<std::pair<int64_t, int64_t>> stack{{0, loff[nb]}};

@@ -300,9 +300,12 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
     Access want;
     builtin_read_map(d->op, w, want);
     const Access& r = n.acc[n.racc];
-    if (r.ax != want.ax || r.ay != want.ay || r.ox != want.ox || r.oy != want.oy || r.hl != want.hl ||
-        r.hr != want.hr || r.ht != want.ht || r.hb != want.hb)
-      return fail(KTILER_E_INVALID, "declared READ footprint is not the op's true stencil for its output tile");
+    // the declared footprint must cover the true stencil (same scale and offset, halos at
+    // least the stencil's): a larger one only adds dependencies (e.g. the line-quantized
+    // maps fitted from ktiler_discover_footprint), a smaller one could produce a wrong plan
+    if (r.ax != want.ax || r.ay != want.ay || r.ox != want.ox || r.oy != want.oy || r.hl < want.hl ||
+        r.hr < want.hr || r.ht < want.ht || r.hb < want.hb)
+      return fail(KTILER_E_INVALID, "declared READ footprint does not cover the op's true stencil for its output tile");
     const Buffer& ib = g->g.bufs[r.buf];
     if (ib.d.elem_bytes != builtin_in_elem(d->op) || ob.d.elem_bytes != builtin_out_elem(d->op))
       return fail(KTILER_E_INVALID, "buffer element sizes do not match the op");

@@ -169,9 +169,17 @@ def test_error_paths(K):
     b = g.add_buffer(0x200000, 64, 64, 1)
     c = g.add_buffer(0x300000, 32, 32, 1)
     acc = lambda buf, mode, ax, ay, h=0: dict(buf=buf, mode=mode, ax=ax, ay=ay, hl=h, hr=h, ht=h, hb=h)
-    # wrong declared footprint for a built-in -> rejected
+    # declared footprint smaller than a built-in's stencil (halo 1 < 2) -> rejected
     with pytest.raises(K.KtilerError):
         g.add_kernel(K.OP_BLUR5, (4, 4, 1), (64, 1, 1), [acc(b, K.READ, 16, 16, 1), acc(c, K.WRITE, 16, 16)])
+    # wrong scale -> rejected; a covering (larger-halo) footprint is accepted: it only adds
+    # dependencies (the line-quantized maps fitted from ktiler_discover_footprint)
+    with pytest.raises(K.KtilerError):
+        g.add_kernel(K.OP_BLUR5, (4, 4, 1), (64, 1, 1), [acc(b, K.READ, 32, 16, 2), acc(c, K.WRITE, 16, 16)])
+    gc = K.Graph()
+    bb = gc.add_buffer(0x200000, 64, 64, 1)
+    cc = gc.add_buffer(0x300000, 64, 64, 1)
+    gc.add_kernel(K.OP_BLUR5, (4, 4, 1), (64, 1, 1), [acc(bb, K.READ, 16, 16, 16), acc(cc, K.WRITE, 16, 16)])
     n0 = g.add_kernel(K.OP_GRAY, (4, 8, 1), (64, 1, 1), [acc(a, K.READ, 16, 8), acc(b, K.WRITE, 16, 8)])
     with pytest.raises(K.KtilerError):
         g.add_edge(n0, n0, b)

@@ -116,7 +116,7 @@ def test_fitted_maps_replan_to_oracle(setup):
     q.view("rgb").copy_(torch.from_numpy(rgb))
     for n in BUFS[1:]:
         q.b.store.tensors[n].fill_(0xA5)
-    plan = g2.plan(64 * 1024, kind="budget", exec_mode="graph")
+    plan = g2.plan(1 << 20, kind="rows", rows=1, exec_mode="graph")
     assert plan.num_fragments() > 1
     plan.execute(0)
     torch.cuda.synchronize()
