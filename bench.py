@@ -201,8 +201,14 @@ def run_reference(args):
         "e2e": {"value": v, "unit": "Mpix/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
 
 
+# algorithmic bytes per OUTPUT pixel of each kernel (input bytes it must read + output bytes)
+NODE_BYTES = {"gray": 3 + 1, "blur": 1 + 1, "down": 4 + 1, "sobel": 1 + 4, "thresh": 4 + 1}
+
+
 def trace_shares(pipe, pol):
-    """Per-kernel share of CTA time in one traced execute of a fresh plan of ``pol``."""
+    """Per-kernel share of CTA time in one traced execute of a fresh plan of ``pol``, and
+    per kernel the mean device span of its launches (first CTA start -> last CTA end) with
+    the algorithmic bytes those launches move."""
     import numpy as np
     pl = pipe.b.g.plan(0, **pol)
     pl.trace_enable(1 << 22)
@@ -218,8 +224,21 @@ def trace_shares(pipe, pol):
     tot = dur.sum()
     out = {names[v] if v >= 0 else "discard": round(float(dur[node == v].sum() / tot), 3) for v in sorted(set(node.tolist()))}
     span = int(k0["t1"].max() - k0["t0"].min())
+    per = {}
+    ids = k0["id"].astype(np.int64)
+    for lid in np.unique(ids):
+        v = launches[int(lid)][1]
+        if v < 0:
+            continue
+        m = ids == lid
+        sp = float(k0["t1"][m].max() - k0["t0"][m].min())
+        tw, th = pipe.geometry[names[v]][:2]
+        d = per.setdefault(names[v], {"launches": 0, "span_ns": 0.0, "bytes": 0.0})
+        d["launches"] += 1
+        d["span_ns"] += sp
+        d["bytes"] += launches[int(lid)][2] * tw * th * NODE_BYTES[names[v]]
     del pl
-    return out, span / 1e6
+    return out, span / 1e6, per
 
 
 def main():
@@ -353,10 +372,22 @@ def main():
         del un
     if not args.no_trace and rank == 0:
         try:
-            tiled_sh, tiled_span = trace_shares(p, pol) if args.mode != "persistent" else (None, None)
-            un_sh, un_span = trace_shares(p, dict(kind="none", exec_mode="graph"))
+            tiled_sh, tiled_span, per_node = trace_shares(p, pol) if args.mode != "persistent" else (None, None, None)
+            un_sh, un_span, _ = trace_shares(p, dict(kind="none", exec_mode="graph"))
             line["trace"] = {"tiled_cta_share": tiled_sh, "tiled_span_ms": tiled_span, "untiled_cta_share": un_sh,
                              "untiled_span_ms": un_span}
+            if per_node:
+                # the dominant kernel of the tiled step (largest CTA-time share): its
+                # algorithmic bytes per launch / its mean launch span (device-side tracer)
+                dom = max(tiled_sh, key=lambda k: tiled_sh[k] if k in per_node else -1)
+                d = per_node[dom]
+                ach = d["bytes"] / d["launches"] / (d["span_ns"] / d["launches"])  # B/ns = GB/s
+                line["roofline"]["dominant_kernel"] = {
+                    "kernel": dom, "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                    "launches_per_step": d["launches"], "mean_launch_us": d["span_ns"] / d["launches"] / 1e3,
+                    "algorithmic_bytes": f"{NODE_BYTES[dom]} B per output pixel x output pixels per launch",
+                    "timing": "device-side tracer (%globaltimer, first CTA start -> last CTA end per launch); "
+                              "launches of the DAG overlap, so this is a per-launch rate, not a share of the step"}
         except Exception as e:  # diagnostics only
             line["trace"] = {"error": str(e)}
     if not args.no_e2e:
