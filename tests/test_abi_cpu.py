@@ -217,3 +217,12 @@ def test_plan_without_device_requires_cache_bytes(K):
     with pytest.raises(K.KtilerError) as e:
         p.plan(0, kind="budget", exec_mode="graph")
     assert e.value.status == K.E_CUDA
+
+
+def test_smoke_configuration_is_tileable(K):
+    """__graft_entry__.smoke()'s plans split the graph into several fragments (B200
+    geometry; a budget below one leaf block's closure would be KTILER_E_UNTILEABLE)."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    p = Pipeline(520, 198, 2, T=60.0, internal=True, device=None)
+    assert p.b.g.plan(800 * 1024, kind="budget", exec_mode="graph", discard=True, pdl=True).num_fragments() > 1
+    assert p.b.g.plan(1 << 20, kind="rows", rows=1, exec_mode="persistent", discard=True).num_fragments() > 1
