@@ -433,13 +433,17 @@ __device__ void blur_compute(const DBuf& out, const Tile& t, const uint8_t* sm, 
 // ---------------------------------------------------------------------------------
 // down2: 2x2 mean, round half up.  16 output pixels from 2 staged rows x 32 bytes.
 // ---------------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t hsum2(uint32_t w) {  // (b0+b1, b2+b3) as u16x2
-  return (w & 0x00FF00FFu) + ((w >> 8) & 0x00FF00FFu);
+// (sum of the 2x2 block + 2) >> 2 for output pixels 2j, 2j+1 from one word of each input
+// row: per word, bytes (0, 2) and (1, 3) as u16x2 lanes (E, O), so E + O holds the two
+// horizontal pair sums; two 3-input adds take both rows and the rounding constant.  The
+// lanes are < 2^10, so the >> 2 of the packed word moves only garbage into bits 14-15 and
+// 30-31: bytes 0 and 2 are the results.
+__device__ __forceinline__ uint32_t down2px(uint32_t a, uint32_t b) {
+  const uint32_t s = (a & 0x00FF00FFu) + prmt(a, 0, 0x4341) + (b & 0x00FF00FFu) + prmt(b, 0, 0x4341) + 0x00020002u;
+  return s >> 2;
 }
 __device__ __forceinline__ uint32_t down4(uint32_t a0, uint32_t a1, uint32_t b0, uint32_t b1) {
-  uint32_t lo = ((hsum2(a0) + hsum2(b0) + 0x00020002u) >> 2) & 0x00FF00FFu;
-  uint32_t hi = ((hsum2(a1) + hsum2(b1) + 0x00020002u) >> 2) & 0x00FF00FFu;
-  return prmt(lo, hi, 0x6420);
+  return prmt(down2px(a0, b0), down2px(a1, b1), 0x6420);
 }
 
 __device__ void down_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
@@ -575,10 +579,17 @@ __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm,
 // ---------------------------------------------------------------------------------
 // thresh: f32 -> u8 {0,255}, strict >
 // ---------------------------------------------------------------------------------
+// four f32 pixels -> four bytes {0, 255}: set.gt.u32.f32 gives 0xFFFFFFFF / 0 per pixel
+// (IEEE compare: NaN > T is false), byte 0 of each mask packed with three PRMTs
+__device__ __forceinline__ uint32_t fset_gt(uint32_t v, float T) {
+  uint32_t m;
+  asm("set.gt.u32.f32 %0, %1, %2;" : "=r"(m) : "f"(__uint_as_float(v)), "f"(T));
+  return m;
+}
 __device__ __forceinline__ uint32_t gt4(uint4 v, float T) {
-  uint32_t a = __uint_as_float(v.x) > T ? 0xFFu : 0u, b = __uint_as_float(v.y) > T ? 0xFFu : 0u;
-  uint32_t c = __uint_as_float(v.z) > T ? 0xFFu : 0u, d = __uint_as_float(v.w) > T ? 0xFFu : 0u;
-  return a | (b << 8) | (c << 16) | (d << 24);
+  const uint32_t lo = prmt(fset_gt(v.x, T), fset_gt(v.y, T), 0x0040);
+  const uint32_t hi = prmt(fset_gt(v.z, T), fset_gt(v.w, T), 0x0040);
+  return prmt(lo, hi, 0x5410);
 }
 
 __device__ void thresh_compute(const DBuf& out, const Tile& t, const uint8_t* sm, float T, int nt, int tid) {
