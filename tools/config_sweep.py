@@ -54,8 +54,9 @@ def main():
     only = {int(x) for x in args.only.split(",")}
 
     def run(tag, obj, W, H, F, cfg, flush_l2):
+        cfg = dict(cfg)
         try:
-            pl = obj.b.g.plan(cfg.pop("cache_bytes", 0), **cfg)
+            pl = obj.b.g.plan(cfg.get("cache_bytes", 0), **{k: v for k, v in cfg.items() if k != "cache_bytes"})
             ms = timeit(torch, s, lambda: pl.execute(s.cuda_stream), args.reps, flush if flush_l2 else None)
             st = pl.stats()
             print(json.dumps({"config": tag, "cfg": cfg, "ms": round(ms, 4), "Mpix/s": round(W * H * F / ms / 1e3, 1),
