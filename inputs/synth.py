@@ -125,3 +125,27 @@ def make(kind: str, seed: int, W: int, H: int, F: int = 1) -> np.ndarray:
     if kind == "scene":
         return scene(seed, W, H, F)
     raise ValueError(kind)
+
+
+def hs_fields(seed: int, W: int, H: int, F: int = 1):
+    """Horn-Schunck JI inputs, seeded and synthetic: brightness
+    derivatives Ix, Iy, It in [-1, 1) on a 1/64 grid, smooth-ish (a hashed value per 4x4
+    cell plus a hashed per-pixel perturbation), and an initial flow (u, v) in [-2, 2) on a
+    1/64 grid.  Returns (coef [F, H, W, 4] f32 with channel 3 = 0, s0 [F, H, W, 2] f32).
+    Plain data generation: no part of the method's arithmetic."""
+    z = np.arange(F * H * W, dtype=np.uint64).reshape(F, H, W)
+    f = np.arange(F, dtype=np.uint64)[:, None, None]
+    y = np.arange(H, dtype=np.uint64)[None, :, None]
+    x = np.arange(W, dtype=np.uint64)[None, None, :]
+    cell = (f * np.uint64(1 << 40)) + ((y >> np.uint64(2)) << np.uint64(20)) + (x >> np.uint64(2))
+    base = np.uint64((seed * 0xD1B54A32D192ED03) & M64)
+    out = []
+    for ch in range(5):
+        salt = np.uint64((ch + 1) * 0x9E3779B97F4A7C15 & M64)
+        c = splitmix64_np(cell ^ base ^ salt)
+        p = splitmix64_np(z ^ base ^ salt ^ np.uint64(0x5851F42D4C957F2D))
+        v = ((c & np.uint64(0x7F)).astype(np.int32) - 64) + ((p & np.uint64(0xF)).astype(np.int32) - 8)
+        out.append(np.clip(v, -64, 63).astype(np.float32) / np.float32(64.0))
+    coef = np.stack([out[0], out[1], out[2], np.zeros_like(out[0])], axis=-1)
+    s0 = np.stack([out[3] * np.float32(2.0), out[4] * np.float32(2.0)], axis=-1)
+    return coef, s0

@@ -23,6 +23,9 @@ Contents (ids O-n):
   (PAPER.md:171, 271), cache constraint.
 * O-12 ``lru_dram_bytes``: fully-associative LRU line model (expectation only,
   not a parity target — "parity unpinned" for anything it predicts).
+* O-13 ``application_tiling``: Alg. 1 with performance tables.
+* O-14 ``hs_jacobi``: K Horn–Schunck Jacobi iterations, the paper's JI nodes
+  (SURVEY §8(f) f2), in f32 (the GPU's exact operation order) or f64.
 """
 from __future__ import annotations
 
@@ -728,3 +731,36 @@ def lru_dram_bytes(g: OGraph, tr: Trace, schedule, cache_bytes: int, discard_dea
             cache.pop(ln, None)
     wr_tail = sum(LINE for d in cache.values() if d)
     return {"read": rd, "write": wr, "write_incl_tail": wr + wr_tail}
+
+
+# ---------------------------------------------------------------------------------------
+# O-14: Horn–Schunck Jacobi iterations (the JI nodes of Fig. 4)
+# ---------------------------------------------------------------------------------------
+def hs_jacobi(coef: np.ndarray, s0: np.ndarray, a2: float, iters: int, dtype=np.float32) -> np.ndarray:
+    """K Jacobi iterations of the Horn–Schunck equations (Horn & Schunck 1981, the method
+    HSOpticalFlow implements): with ub, vb the mean of the 4 neighbours
+    (replicate border, reading A39),
+        t  = (Ix*ub + Iy*vb + It) / (alpha^2 + Ix^2 + Iy^2)
+        u' = ub - Ix*t,   v' = vb - Iy*t.
+    coef [F, H, W, 4] = (Ix, Iy, It, -); s0 [F, H, W, 2] = (u, v); a2 = alpha^2.  Every
+    operation is evaluated in the order written in include/ktiler.h (KTILER_OP_JACOBI),
+    one numpy op at a time in ``dtype`` (float32: each op IEEE-rounded, no contraction)."""
+    c = coef.astype(dtype)
+    Ix, Iy, It = c[..., 0], c[..., 1], c[..., 2]
+    a2 = dtype(a2)
+    quarter = dtype(0.25)
+    den = (a2 + Ix * Ix) + Iy * Iy
+    s = s0.astype(dtype).copy()
+    for _ in range(iters):
+        u, v = s[..., 0], s[..., 1]
+
+        def mean4(a):
+            left = np.concatenate([a[:, :, :1], a[:, :, :-1]], axis=2)
+            right = np.concatenate([a[:, :, 1:], a[:, :, -1:]], axis=2)
+            up = np.concatenate([a[:, :1], a[:, :-1]], axis=1)
+            down = np.concatenate([a[:, 1:], a[:, -1:]], axis=1)
+            return ((left + right) + (up + down)) * quarter
+        ub, vb = mean4(u), mean4(v)
+        t = ((Ix * ub + Iy * vb) + It) / den
+        s = np.stack([ub - Ix * t, vb - Iy * t], axis=-1)
+    return s

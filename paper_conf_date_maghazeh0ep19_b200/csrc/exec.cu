@@ -74,6 +74,7 @@ struct KParams {
   int32_t use_tmap;
   int32_t in_stream;    // input is a graph input: load it evict-first
   DBuf in, out;
+  DBuf aux;             // KTILER_OP_JACOBI: the coefficient buffer (second READ access)
   int32_t tw, th;
   float T;
   int32_t nrect, ndisc, pdl;
@@ -186,7 +187,7 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
 }
 
 template <int OP, bool SCALAR>
-__global__ void __launch_bounds__(256, (OP == 1 || OP == 3) ? 3 : 4) op_kernel(const __grid_constant__ KParams p) {
+__global__ void __launch_bounds__(256, (OP == 1 || OP == 3 || OP == 6) ? 3 : 4) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
@@ -262,11 +263,11 @@ __global__ void __launch_bounds__(256, (OP == 1 || OP == 3) ? 3 : 4) op_kernel(c
       ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
       ph ^= 1u << b;
       const ktd::Tile t = s_tile[b];
-      if ((OP == 1 || OP == 3) && ktd::needs_fix(OP, p.in, t)) {
+      if ((OP == 1 || OP == 3 || OP == 6) && ktd::needs_fix(OP, p.in, t)) {
         ktd::stage_fix(OP, p.in, t, buf, nt, tid);
         __syncthreads();
       }
-      ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid);
+      ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid, &p.aux);
       const int64_t nx = i + 2 * (int64_t)gridDim.x;
       if (p.chain) {
         __syncthreads();  // tile written (and buffer b consumed)
@@ -720,6 +721,7 @@ kfn_t vec_kernel(int op) {
     case 1: return op_kernel<1, false>;
     case 2: return op_kernel<2, false>;
     case 3: return op_kernel<3, false>;
+    case 6: return op_kernel<6, false>;
     default: return op_kernel<4, false>;
   }
 }
@@ -858,6 +860,7 @@ void build_launches(ktiler_plan_s* P) {
         L.n = const_cast<kt::Node*>(&n);
         L.kp.in = dbuf(g.bufs[r.buf]);
         L.kp.out = dbuf(g.bufs[w.buf]);
+        if (n.racc2 >= 0) L.kp.aux = dbuf(g.bufs[n.acc[n.racc2].buf]);
         L.kp.in_stream = !g.written_by_node(r.buf);
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
@@ -1044,6 +1047,7 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
     case KTILER_OP_BLUR5: bw = 16 * (nseg + 2); bh = th + 4; break;
     case KTILER_OP_DOWN2: bw = 32 * nseg; bh = 2 * th; break;
     case KTILER_OP_SOBEL3: bw = 16 * (nseg + 2); bh = th + 2; break;
+    case KTILER_OP_JACOBI: bw = 4 * (tw + 4); bh = th + 2; break;
     default: bw = 64 * nseg; bh = th; break;
   }
   if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != ktd::stage_bytes(n.op, tw, th)) return false;
@@ -1330,7 +1334,8 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   const int nn = (int)g.nodes.size();
   const int nsub = (int)S.subs.size();
   for (auto& n : g.nodes)
-    if (n.op == KTILER_OP_CUSTOM) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode runs built-in ops only");
+    if (n.op == KTILER_OP_CUSTOM || n.op == KTILER_OP_JACOBI)
+      return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode runs the image-pipeline built-ins (GRAY..THRESH) only");
   if (nn > PMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: at most 8 nodes");
   std::vector<PNode> pn(nn);
   for (int v = 0; v < nn; ++v) {

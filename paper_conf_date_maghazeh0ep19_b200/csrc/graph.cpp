@@ -92,12 +92,15 @@ static bool builtin_read_map(int op, const Access& w, Access& r) {
     case KTILER_OP_DOWN2:
       r.ax = 2 * w.ax; r.ay = 2 * w.ay; r.ox = 2 * w.ox; r.oy = 2 * w.oy;
       return true;
+    case KTILER_OP_JACOBI: r.hl = r.hr = 2; r.ht = r.hb = 1; return true;  // (u, v) of the 4 neighbours
     default: return false;
   }
 }
 
-static int builtin_in_elem(int op) { return op == KTILER_OP_GRAY ? 3 : (op == KTILER_OP_THRESH ? 4 : 1); }
-static int builtin_out_elem(int op) { return op == KTILER_OP_SOBEL3 ? 4 : 1; }
+static int builtin_in_elem(int op) {
+  return op == KTILER_OP_GRAY ? 3 : ((op == KTILER_OP_THRESH || op == KTILER_OP_JACOBI) ? 4 : 1);
+}
+static int builtin_out_elem(int op) { return (op == KTILER_OP_SOBEL3 || op == KTILER_OP_JACOBI) ? 4 : 1; }
 
 ktiler_status Graph::finalize() {
   if (finalized) return KTILER_OK;
@@ -249,7 +252,7 @@ ktiler_status ktiler_add_buffer(ktiler_graph_t g, const ktiler_buffer_desc* d, i
 ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, int32_t* node_id) {
   if (!g || !d || !node_id) return fail(KTILER_E_INVALID, "NULL argument");
   if (g->g.finalized) return fail(KTILER_E_STATE, "graph already planned; create a new graph");
-  if (d->op < KTILER_OP_GRAY || d->op > KTILER_OP_CUSTOM) return fail(KTILER_E_INVALID, "unknown op");
+  if (d->op < KTILER_OP_GRAY || d->op > KTILER_OP_JACOBI) return fail(KTILER_E_INVALID, "unknown op");
   if (d->n_access <= 0 || !d->access) return fail(KTILER_E_INVALID, "a kernel needs at least one access");
   Node n;
   n.op = d->op;
@@ -275,8 +278,13 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
       if (n.wacc >= 0 && d->op != KTILER_OP_CUSTOM) return fail(KTILER_E_INVALID, "built-in kernels have exactly one WRITE access");
       n.wacc = i;
     } else {
-      if (n.racc >= 0 && d->op != KTILER_OP_CUSTOM) return fail(KTILER_E_INVALID, "built-in kernels have exactly one READ access");
-      n.racc = i;
+      if (d->op == KTILER_OP_JACOBI && n.racc >= 0) {
+        if (n.racc2 >= 0) return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI has exactly two READ accesses");
+        n.racc2 = i;
+      } else {
+        if (n.racc >= 0 && d->op != KTILER_OP_CUSTOM) return fail(KTILER_E_INVALID, "built-in kernels have exactly one READ access");
+        n.racc = i;
+      }
     }
     n.acc.push_back(x);
   }
@@ -309,6 +317,17 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
     const Buffer& ib = g->g.bufs[r.buf];
     if (ib.d.elem_bytes != builtin_in_elem(d->op) || ob.d.elem_bytes != builtin_out_elem(d->op))
       return fail(KTILER_E_INVALID, "buffer element sizes do not match the op");
+    if (d->op == KTILER_OP_JACOBI) {
+      if (n.racc2 < 0) return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI has exactly two READ accesses");
+      const Access& c = n.acc[n.racc2];
+      const Buffer& cb = g->g.bufs[c.buf];
+      if (c.ax != 2 * w.ax || c.ay != w.ay || c.ox != 2 * w.ox || c.oy != w.oy)
+        return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI coefficient footprint must be (2*ax, ay) of the output's");
+      if (cb.d.elem_bytes != 4 || cb.d.width != 2 * ob.d.width || cb.d.height != ob.d.height)
+        return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI coefficients are f32 [H][4W] (Ix, Iy, It, - per pixel)");
+      if ((ob.d.width & 3) || (w.ax & 3)) return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI needs an even image width and tile width");
+      if (c.buf == r.buf || c.buf == w.buf) return fail(KTILER_E_INVALID, "KTILER_OP_JACOBI buffers must be distinct");
+    }
     if (d->op == KTILER_OP_DOWN2) {
       if ((ib.d.width & 1) || (ib.d.height & 1)) return fail(KTILER_E_INVALID, "DOWN2 needs even input sizes (SURVEY A3)");
       if (ob.d.width != ib.d.width / 2 || ob.d.height != ib.d.height / 2)
@@ -316,13 +335,14 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
     } else if (ob.d.width != ib.d.width || ob.d.height != ib.d.height) {
       return fail(KTILER_E_INVALID, "input and output sizes differ");
     }
-    if (d->op == KTILER_OP_THRESH) {
-      if (n.params.size() != sizeof(float)) return fail(KTILER_E_INVALID, "THRESH params must be one float T");
+    if (d->op == KTILER_OP_THRESH || d->op == KTILER_OP_JACOBI) {
+      if (n.params.size() != sizeof(float))
+        return fail(KTILER_E_INVALID, "THRESH / JACOBI params must be one float (T / alpha^2)");
       std::memcpy(&n.T, n.params.data(), sizeof(float));
     }
     int64_t nt = n.nthreads();
     if (nt > 1024) return fail(KTILER_E_INVALID, "more than 1024 threads per block");
-    n.scalar = (nt == w.ax * w.ay);
+    n.scalar = (nt == w.ax * w.ay) && d->op != KTILER_OP_JACOBI;
     if (!n.scalar) {
       if (w.ax % 16) return fail(KTILER_E_INVALID, "vector variant needs tile width % 16 == 0 (else use one thread per pixel)");
       if (nt % 32) return fail(KTILER_E_INVALID, "vector variant needs a multiple of 32 threads per block");

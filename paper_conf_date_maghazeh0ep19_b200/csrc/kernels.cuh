@@ -165,6 +165,7 @@ __device__ __forceinline__ StageGeo stage_geo(int op, const DBuf& in, const Tile
     case 1: return {t.y0 - 2, t.x0 - 16, up16(in.W), rows + 4, 16 * (nseg + 2), true};
     case 2: return {2 * t.y0, 2 * t.x0, up16(in.W), 2 * rows, 32 * nseg, false};
     case 3: return {t.y0 - 1, t.x0 - 16, up16(in.W), rows + 2, 16 * (nseg + 2), true};
+    case 6: return {t.y0 - 1, 4 * (t.x0 - 2), up16(4 * in.W), rows + 2, 4 * (t.fw + 4), true};  // f32, 1 px = 2 floats
     default: return {t.y0, 4 * t.x0, up16(4 * in.W), rows, 64 * nseg, false};
   }
 }
@@ -178,6 +179,7 @@ __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
     case 2: return 2 * th * 32 * nseg;           // 2 blur rows per output row
     case 3: return (th + 2) * 16 * (nseg + 2);   // down rows y-1..y+1
     case 4: return th * 64 * nseg;               // f32 rows
+    case 6: return (th + 2) * 4 * (tw + 4);      // (u, v) rows y-1..y+th, one pixel of halo per side
   }
   return 0;
 }
@@ -230,20 +232,22 @@ __device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map,
 // the caller synchronizes afterwards.  Returns quickly for interior tiles.
 __device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid,
                                           int bar_id = 4) {
-  if (op != 1 && op != 3) return;
+  if (op != 1 && op != 3 && op != 6) return;
   const StageGeo g = stage_geo(op, in, t);
-  const int left = g.xb0 < 0 ? (int)(-g.xb0) : 0;                                       // columns < 0
-  const int rfrom = (int)(in.W - g.xb0) < g.stride ? (int)(in.W - g.xb0) : g.stride;      // columns >= W
+  const int pe = op == 6 ? 8 : 1;                                                          // bytes per pixel
+  const int ew = op == 6 ? 4 : 1;                                                          // bytes per element
+  const int left = g.xb0 < 0 ? (int)(-g.xb0) : 0;                                          // bytes < 0
+  const int rfrom = (int)(ew * in.W - g.xb0) < g.stride ? (int)(ew * in.W - g.xb0) : g.stride;  // bytes >= row end
   const int right = g.stride - rfrom;
-  const int top = g.ry0 < 0 ? (int)(-g.ry0) : 0;                                         // rows < 0
-  const int bfrom = (int)(in.H - g.ry0) < g.nr ? (int)(in.H - g.ry0) : g.nr;              // rows >= H
+  const int top = g.ry0 < 0 ? (int)(-g.ry0) : 0;                                           // rows < 0
+  const int bfrom = (int)(in.H - g.ry0) < g.nr ? (int)(in.H - g.ry0) : g.nr;                // rows >= H
   const int per = left + right;
   if (per) {
     for (int i = tid; i < (bfrom - top) * per; i += nt) {
       const int r = top + i / per, k = i % per;
       uint8_t* row = sm + r * g.stride;
-      if (k < left) row[k] = row[left];                 // pixel 0
-      else row[rfrom + (k - left)] = row[rfrom - 1];    // pixel W-1
+      if (k < left) row[k] = row[left + k % pe];                   // pixel 0
+      else row[rfrom + (k - left)] = row[rfrom - pe + (k - left) % pe];  // last pixel
     }
   }
   if (top || bfrom < g.nr) {
@@ -260,9 +264,10 @@ __device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t,
 
 // Does tile t of a stencil op need stage_fix?  (CTA-uniform)
 __device__ __forceinline__ bool needs_fix(int op, const DBuf& in, const Tile& t) {
-  if (op != 1 && op != 3) return false;
+  if (op != 1 && op != 3 && op != 6) return false;
   const StageGeo g = stage_geo(op, in, t);
-  return g.xb0 < 0 || g.xb0 + g.stride > in.W || g.ry0 < 0 || g.ry0 + g.nr > in.H;
+  const int64_t rowb = op == 6 ? 4 * in.W : in.W;
+  return g.xb0 < 0 || g.xb0 + g.stride > rowb || g.ry0 < 0 || g.ry0 + g.nr > in.H;
 }
 
 __device__ __forceinline__ void store_u8_16(uint8_t* d, int64_t x, int64_t W, uint4 o) {
@@ -606,15 +611,59 @@ __device__ void thresh_compute(const DBuf& out, const Tile& t, const uint8_t* sm
   });
 }
 
+// ---------------------------------------------------------------------------------
+// jacobi: one Horn-Schunck Jacobi iteration (KTILER_OP_JACOBI, the paper's JI node).  The
+// staged window holds (u, v) of rows y0-1 .. y1 with one pixel of halo per side
+// (replicate-fixed at image edges); an item = 2 pixels of one row.  Coefficients
+// (Ix, Iy, It, -) come straight from global memory (read once, 1:1, 128-bit loads).
+// Every operation is an explicitly rounded f32 op in the order of include/ktiler.h, so
+// the result is bit-identical to any IEEE evaluation in that order (DESIGN A39).
+// ---------------------------------------------------------------------------------
+__device__ __forceinline__ float2 jacobi_px(float2 l, float2 r, float2 u, float2 d, float4 c, float a2) {
+  const float ub = __fmul_rn(__fadd_rn(__fadd_rn(l.x, r.x), __fadd_rn(u.x, d.x)), 0.25f);
+  const float vb = __fmul_rn(__fadd_rn(__fadd_rn(l.y, r.y), __fadd_rn(u.y, d.y)), 0.25f);
+  const float num = __fadd_rn(__fadd_rn(__fmul_rn(c.x, ub), __fmul_rn(c.y, vb)), c.z);
+  const float den = __fadd_rn(__fadd_rn(a2, __fmul_rn(c.x, c.x)), __fmul_rn(c.y, c.y));
+  const float tt = __fdiv_rn(num, den);
+  return make_float2(__fsub_rn(ub, __fmul_rn(c.x, tt)), __fsub_rn(vb, __fmul_rn(c.y, tt)));
+}
+
+__device__ void jacobi_compute(const DBuf& out, const DBuf& coef, const Tile& t, const uint8_t* sm, float a2, int nt,
+                               int tid) {
+  const int stride = 4 * (t.fw + 4);           // bytes per staged row
+  const int npair = (int)((t.x1 - t.x0) >> 2);  // pixel pairs per row (x in floats, 4 floats per pair)
+  const int rows = t.rows();
+  const int64_t px0 = t.x0 >> 1;               // first output pixel
+  for (int it = tid; it < npair * rows; it += nt) {
+    const int r = it / npair, q = it - r * npair;
+    // staged pixel k of a row sits at byte 8 * (k + 1); pixels 2q-1 .. 2q+2 of the centre row
+    const uint8_t* cen = sm + (r + 1) * stride + 16 * q;
+    const float4 a = *reinterpret_cast<const float4*>(cen);       // pixels 2q-1, 2q
+    const float4 b = *reinterpret_cast<const float4*>(cen + 16);  // pixels 2q+1, 2q+2
+    const float2 u0 = *reinterpret_cast<const float2*>(cen - stride + 8);   // up row, pixel 2q
+    const float2 u1 = *reinterpret_cast<const float2*>(cen - stride + 16);  // up row, pixel 2q+1
+    const float2 d0 = *reinterpret_cast<const float2*>(cen + stride + 8);
+    const float2 d1 = *reinterpret_cast<const float2*>(cen + stride + 16);
+    const int64_t y = t.y0 + r, x = px0 + 2 * q;
+    const float4* cp = reinterpret_cast<const float4*>(coef.p + t.z * coef.fstride + y * coef.pitch) + x;
+    const float4 c0 = __ldcg(cp), c1 = __ldcg(cp + 1);  // every iteration re-reads them: keep in L2
+    const float2 o0 = jacobi_px(make_float2(a.x, a.y), make_float2(b.x, b.y), u0, d0, c0, a2);
+    const float2 o1 = jacobi_px(make_float2(a.z, a.w), make_float2(b.z, b.w), u1, d1, c1, a2);
+    float4* dst = reinterpret_cast<float4*>(out.p + t.z * out.fstride + y * out.pitch) + (x >> 1);
+    *dst = make_float4(o0.x, o0.y, o1.x, o1.y);
+  }
+}
+
 // Compute op's output tile from its staged input (after the staging is complete).
 __device__ __forceinline__ void compute_tile(int op, const DBuf& out, const Tile& t, const uint8_t* sm, float T,
-                                             int nt, int tid) {
+                                             int nt, int tid, const DBuf* aux = nullptr) {
   switch (op) {
     case 0: gray_compute(out, t, sm, nt, tid); break;
     case 1: blur_compute<BLUR_R>(out, t, sm, nt, tid); break;
     case 2: down_compute(out, t, sm, nt, tid); break;
     case 3: sobel_compute<SOBEL_R>(out, t, sm, nt, tid); break;
     case 4: thresh_compute(out, t, sm, T, nt, tid); break;
+    case 6: jacobi_compute(out, *aux, t, sm, T, nt, tid); break;  // T = a2 (alpha^2)
   }
 }
 

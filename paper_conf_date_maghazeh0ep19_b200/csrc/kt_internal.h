@@ -43,7 +43,8 @@ struct Node {
   ktiler_launch_fn launch = nullptr;
   void* user = nullptr;
   int wacc = -1;     // index of the (single) WRITE access for built-ins
-  int racc = -1;     // index of the (single) READ access for built-ins
+  int racc = -1;     // index of the (first) READ access for built-ins
+  int racc2 = -1;    // KTILER_OP_JACOBI: its second READ access (the coefficients)
   int64_t nblocks = 0;
   int64_t gid0 = 0;  // first global block id
   float T = 200.f;

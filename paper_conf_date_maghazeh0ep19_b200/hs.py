@@ -1,0 +1,69 @@
+"""The paper's own workload: the Jacobi-iteration chain of Horn–Schunck
+optical flow, HSOpticalFlow's JI nodes (Fig. 4: 500 JI nodes per step,
+98.5% of the application's time, the nodes KTILER tiles).
+
+``HSJacobi`` declares K chained KTILER_OP_JACOBI nodes through the C ABI:
+
+    s_0 --JI_1--> s_1 --JI_2--> ... --JI_K--> s_K        every JI_k also reads `coef`
+
+  s_k   f32 [frames][H][2W]: (u, v) per pixel, the flow after k iterations;
+  coef  f32 [frames][H][4W]: (Ix, Iy, It, unused) per pixel; alpha^2 = a2 is the op's parameter.
+
+Each iterate is its own buffer (the paper's DFG has one vector per JI node; KTILER's
+hazard model is RAW only), so s_1..s_{K-1} are internal (discardable) and the
+whole chain is one KTILER cluster: Alg. 2 tiles across iterations with the halo growing
+by one pixel per iteration, exactly as for the image pipeline.  Device buffers are torch
+tensors (allocator only); every step of the chain runs in libktiler's sm_100a kernel."""
+from __future__ import annotations
+
+import struct
+
+from . import ktiler as K
+from .pipeline import _GraphBuilder
+
+
+class HSJacobi:
+    def __init__(self, W: int, H: int, iters: int, frames: int = 1, a2: float = 1.0, tile=(64, 16),
+                 threads: int = 128, device="cuda", internal: bool = True):
+        if W % 2 or tile[0] % 8:
+            raise ValueError("HSJacobi needs an even width and a tile width that is a multiple of 8 pixels")
+        self.W, self.H, self.K, self.F = W, H, iters, frames
+        b = _GraphBuilder(device, 128)
+        self.b = b
+        b.buffer("coef", 4 * W, H, frames, 4, internal=False)
+        for k in range(iters + 1):
+            b.buffer(f"s{k}", 2 * W, H, frames, 4, internal=internal and 0 < k < iters)
+        tw, th = tile
+        grid = (-(-W // tw), -(-H // th), frames)
+        cid = b.bufs["coef"][0]
+        self.nodes = []
+        for k in range(1, iters + 1):
+            src, dst = b.bufs[f"s{k - 1}"][0], b.bufs[f"s{k}"][0]
+            acc = [dict(buf=src, mode=K.READ, ax=2 * tw, ay=th, hl=2, hr=2, ht=1, hb=1),
+                   dict(buf=cid, mode=K.READ, ax=4 * tw, ay=th),
+                   dict(buf=dst, mode=K.WRITE, ax=2 * tw, ay=th)]
+            nid = b.g.add_kernel(K.OP_JACOBI, grid, (threads, 1, 1), acc, struct.pack("f", a2))
+            self.nodes.append(nid)
+            if k > 1:
+                b.g.add_edge(self.nodes[-2], nid, src, -1.0)
+        self.grid = grid
+        self.plan_obj = None
+
+    @property
+    def graph(self) -> K.Graph:
+        return self.b.g
+
+    def view(self, name: str):
+        """torch view of a buffer: coef -> [F, H, W, 4], s_k -> [F, H, W, 2] (float32)."""
+        import torch
+        bid, Wf, H, F, elem, pitch = self.b.bufs[name]
+        t = self.b.store.tensors[name].view(F, H, pitch)[:, :, :Wf * 4].contiguous().view(torch.float32) \
+            if pitch != Wf * 4 else self.b.store.tensors[name].view(torch.float32).view(F, H, Wf)
+        return t.view(F, H, Wf // (4 if name == "coef" else 2), 4 if name == "coef" else 2)
+
+    def plan(self, cache_bytes: int = 0, **policy) -> K.Plan:
+        self.plan_obj = self.b.g.plan(cache_bytes, **policy)
+        return self.plan_obj
+
+    def run(self, stream: int = 0) -> None:
+        self.plan_obj.execute(stream)

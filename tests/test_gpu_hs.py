@@ -1,0 +1,61 @@
+"""§8(f) f2 on the GPU: chains of KTILER_OP_JACOBI nodes (the paper's JI nodes,
+PAPER.md:381–399) through libktiler vs the f32 oracle O-14, bit for bit, untiled and tiled
+across iterations (Alg. 2 closures growing one pixel per iteration), in several executors."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+from inputs import synth  # noqa: E402
+from oracle import oracle as O  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import __graft_entry__ as ge
+    ge.build()
+
+
+def _run(W, H, F, K, a2, seed, internal, **pol):
+    from paper_conf_date_maghazeh0ep19_b200.hs import HSJacobi
+    h = HSJacobi(W, H, K, frames=F, a2=a2, internal=internal)
+    coef, s0 = synth.hs_fields(seed, W, H, F)
+    for k in range(1, K + 1):
+        h.b.store.tensors[f"s{k}"].fill_(0xFF)  # NaN poison: a skipped block cannot pass
+    h.b.store.tensors["coef"].copy_(torch.from_numpy(coef.reshape(-1).view(np.uint8)))
+    h.b.store.tensors["s0"].copy_(torch.from_numpy(s0.reshape(-1).view(np.uint8)))
+    cb = pol.pop("cache_bytes", 1 << 20)
+    plan = h.plan(cb, **pol)
+    h.run()
+    torch.cuda.synchronize()
+    got = h.b.store.tensors[f"s{K}"].cpu().numpy().view(np.float32).reshape(F, H, W, 2)
+    return got, plan, coef, s0, h
+
+
+CASES = [(128, 64, 1, 1), (256, 160, 1, 5), (512, 256, 2, 8), (200, 120, 1, 3)]
+
+
+@pytest.mark.parametrize("W,H,F,K", CASES)
+@pytest.mark.parametrize("pol", [dict(kind="none", exec_mode="graph"),
+                                 dict(kind="rows", rows=1, exec_mode="graph", discard=True),
+                                 dict(kind="rows", rows=2, exec_mode="dag", discard=True),
+                                 dict(kind="budget", cache_bytes=4 << 20, exec_mode="stream"),
+                                 dict(kind="rows", rows=1, exec_mode="wave", discard=True)],
+                         ids=lambda d: "-".join(f"{k}={v}" for k, v in d.items()))
+def test_jacobi_chain_bit_exact(W, H, F, K, pol):
+    got, plan, coef, s0, _ = _run(W, H, F, K, 0.5, W + K, internal=bool(pol.get("discard")), **dict(pol))
+    ref = O.hs_jacobi(coef, s0, 0.5, K)
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+    if pol["kind"] == "rows" and K > 1:
+        assert plan.num_fragments() > 1
+
+
+def test_every_iterate_bit_exact():
+    """Intermediates too (not discarded): s_k == k oracle iterations for every k."""
+    W, H, K = 192, 96, 4
+    _, plan, coef, s0, h = _run(W, H, 1, K, 2.0, 3, internal=False, kind="rows", rows=1, exec_mode="graph")
+    for k in range(1, K + 1):
+        got = h.b.store.tensors[f"s{k}"].cpu().numpy().view(np.float32).reshape(1, H, W, 2)
+        assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 2.0, k).view(np.uint32)), k
