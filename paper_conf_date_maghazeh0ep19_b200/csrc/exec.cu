@@ -1047,7 +1047,7 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
     case KTILER_OP_BLUR5: bw = 16 * (nseg + 2); bh = th + 4; break;
     case KTILER_OP_DOWN2: bw = 32 * nseg; bh = 2 * th; break;
     case KTILER_OP_SOBEL3: bw = 16 * (nseg + 2); bh = th + 2; break;
-    case KTILER_OP_JACOBI: bw = 4 * (tw + 4); bh = th + 2; break;
+    case KTILER_OP_JACOBI: bw = 4 * (tw + 8); bh = th + 2; break;
     default: bw = 64 * nseg; bh = th; break;
   }
   if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != ktd::stage_bytes(n.op, tw, th)) return false;

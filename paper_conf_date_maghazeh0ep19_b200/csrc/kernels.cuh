@@ -165,7 +165,7 @@ __device__ __forceinline__ StageGeo stage_geo(int op, const DBuf& in, const Tile
     case 1: return {t.y0 - 2, t.x0 - 16, up16(in.W), rows + 4, 16 * (nseg + 2), true};
     case 2: return {2 * t.y0, 2 * t.x0, up16(in.W), 2 * rows, 32 * nseg, false};
     case 3: return {t.y0 - 1, t.x0 - 16, up16(in.W), rows + 2, 16 * (nseg + 2), true};
-    case 6: return {t.y0 - 1, 4 * (t.x0 - 2), up16(4 * in.W), rows + 2, 4 * (t.fw + 4), true};  // f32, 1 px = 2 floats
+    case 6: return {t.y0 - 1, 4 * (t.x0 - 4), up16(4 * in.W), rows + 2, 4 * (t.fw + 8), true};  // f32, 2 px halo (16-B aligned)
     default: return {t.y0, 4 * t.x0, up16(4 * in.W), rows, 64 * nseg, false};
   }
 }
@@ -179,7 +179,7 @@ __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
     case 2: return 2 * th * 32 * nseg;           // 2 blur rows per output row
     case 3: return (th + 2) * 16 * (nseg + 2);   // down rows y-1..y+1
     case 4: return th * 64 * nseg;               // f32 rows
-    case 6: return (th + 2) * 4 * (tw + 4);      // (u, v) rows y-1..y+th, one pixel of halo per side
+    case 6: return (th + 2) * 4 * (tw + 8);      // (u, v) rows y-1..y+th, two pixels of halo per side
   }
   return 0;
 }
@@ -630,25 +630,27 @@ __device__ __forceinline__ float2 jacobi_px(float2 l, float2 r, float2 u, float2
 
 __device__ void jacobi_compute(const DBuf& out, const DBuf& coef, const Tile& t, const uint8_t* sm, float a2, int nt,
                                int tid) {
-  const int stride = 4 * (t.fw + 4);           // bytes per staged row
+  const int stride = 4 * (t.fw + 8);           // bytes per staged row (2 px of halo per side)
   const int npair = (int)((t.x1 - t.x0) >> 2);  // pixel pairs per row (x in floats, 4 floats per pair)
   const int rows = t.rows();
   const int64_t px0 = t.x0 >> 1;               // first output pixel
   for (int it = tid; it < npair * rows; it += nt) {
     const int r = it / npair, q = it - r * npair;
-    // staged pixel k of a row sits at byte 8 * (k + 1); pixels 2q-1 .. 2q+2 of the centre row
+    // staged pixel k of a row sits at byte 8 * (k + 2): pixels 2q-2 .. 2q+3 of the centre row
     const uint8_t* cen = sm + (r + 1) * stride + 16 * q;
-    const float4 a = *reinterpret_cast<const float4*>(cen);       // pixels 2q-1, 2q
-    const float4 b = *reinterpret_cast<const float4*>(cen + 16);  // pixels 2q+1, 2q+2
-    const float2 u0 = *reinterpret_cast<const float2*>(cen - stride + 8);   // up row, pixel 2q
-    const float2 u1 = *reinterpret_cast<const float2*>(cen - stride + 16);  // up row, pixel 2q+1
-    const float2 d0 = *reinterpret_cast<const float2*>(cen + stride + 8);
-    const float2 d1 = *reinterpret_cast<const float2*>(cen + stride + 16);
+    const float4 a = *reinterpret_cast<const float4*>(cen);        // pixels 2q-2, 2q-1
+    const float4 b = *reinterpret_cast<const float4*>(cen + 16);   // pixels 2q, 2q+1 (unused centre)
+    const float4 c = *reinterpret_cast<const float4*>(cen + 32);   // pixels 2q+2, 2q+3
+    const float4 up = *reinterpret_cast<const float4*>(cen - stride + 16);  // row above: 2q, 2q+1
+    const float4 dn = *reinterpret_cast<const float4*>(cen + stride + 16);  // row below
     const int64_t y = t.y0 + r, x = px0 + 2 * q;
     const float4* cp = reinterpret_cast<const float4*>(coef.p + t.z * coef.fstride + y * coef.pitch) + x;
     const float4 c0 = __ldcg(cp), c1 = __ldcg(cp + 1);  // every iteration re-reads them: keep in L2
-    const float2 o0 = jacobi_px(make_float2(a.x, a.y), make_float2(b.x, b.y), u0, d0, c0, a2);
-    const float2 o1 = jacobi_px(make_float2(a.z, a.w), make_float2(b.z, b.w), u1, d1, c1, a2);
+    // pixel 2q: left 2q-1, right 2q+1;  pixel 2q+1: left 2q, right 2q+2
+    const float2 o0 = jacobi_px(make_float2(a.z, a.w), make_float2(b.z, b.w), make_float2(up.x, up.y),
+                                make_float2(dn.x, dn.y), c0, a2);
+    const float2 o1 = jacobi_px(make_float2(b.x, b.y), make_float2(c.x, c.y), make_float2(up.z, up.w),
+                                make_float2(dn.z, dn.w), c1, a2);
     float4* dst = reinterpret_cast<float4*>(out.p + t.z * out.fstride + y * out.pitch) + (x >> 1);
     *dst = make_float4(o0.x, o0.y, o1.x, o1.y);
   }

@@ -53,13 +53,24 @@ class HSJacobi:
     def graph(self) -> K.Graph:
         return self.b.g
 
-    def view(self, name: str):
-        """torch view of a buffer: coef -> [F, H, W, 4], s_k -> [F, H, W, 2] (float32)."""
-        import torch
+    def _rows(self, name: str):
+        """uint8 view [F, H, row bytes] of a buffer (pitch padding excluded)."""
         bid, Wf, H, F, elem, pitch = self.b.bufs[name]
-        t = self.b.store.tensors[name].view(F, H, pitch)[:, :, :Wf * 4].contiguous().view(torch.float32) \
-            if pitch != Wf * 4 else self.b.store.tensors[name].view(torch.float32).view(F, H, Wf)
-        return t.view(F, H, Wf // (4 if name == "coef" else 2), 4 if name == "coef" else 2)
+        return self.b.store.tensors[name].view(F, H, pitch)[:, :, :Wf * elem]
+
+    def set(self, name: str, arr) -> None:
+        """Copy a host float32 array ([F, H, W, 4] for coef, [F, H, W, 2] for s_k) in."""
+        import numpy as np
+        import torch
+        r = self._rows(name)
+        r.copy_(torch.from_numpy(np.ascontiguousarray(arr, dtype=np.float32).view(np.uint8).reshape(r.shape)))
+
+    def get(self, name: str):
+        """Host float32 copy of a buffer: [F, H, W, 4] for coef, [F, H, W, 2] for s_k."""
+        import numpy as np
+        r = self._rows(name).cpu().numpy()
+        ch = 4 if name == "coef" else 2
+        return np.ascontiguousarray(r).view(np.float32).reshape(self.F, self.H, self.W, ch)
 
     def plan(self, cache_bytes: int = 0, **policy) -> K.Plan:
         self.plan_obj = self.b.g.plan(cache_bytes, **policy)

@@ -24,14 +24,13 @@ def _run(W, H, F, K, a2, seed, internal, **pol):
     coef, s0 = synth.hs_fields(seed, W, H, F)
     for k in range(1, K + 1):
         h.b.store.tensors[f"s{k}"].fill_(0xFF)  # NaN poison: a skipped block cannot pass
-    h.b.store.tensors["coef"].copy_(torch.from_numpy(coef.reshape(-1).view(np.uint8)))
-    h.b.store.tensors["s0"].copy_(torch.from_numpy(s0.reshape(-1).view(np.uint8)))
+    h.set("coef", coef)
+    h.set("s0", s0)
     cb = pol.pop("cache_bytes", 1 << 20)
     plan = h.plan(cb, **pol)
     h.run()
     torch.cuda.synchronize()
-    got = h.b.store.tensors[f"s{K}"].cpu().numpy().view(np.float32).reshape(F, H, W, 2)
-    return got, plan, coef, s0, h
+    return h.get(f"s{K}"), plan, coef, s0, h
 
 
 CASES = [(128, 64, 1, 1), (256, 160, 1, 5), (512, 256, 2, 8), (200, 120, 1, 3)]
@@ -57,5 +56,5 @@ def test_every_iterate_bit_exact():
     W, H, K = 192, 96, 4
     _, plan, coef, s0, h = _run(W, H, 1, K, 2.0, 3, internal=False, kind="rows", rows=1, exec_mode="graph")
     for k in range(1, K + 1):
-        got = h.b.store.tensors[f"s{k}"].cpu().numpy().view(np.float32).reshape(1, H, W, 2)
+        got = h.get(f"s{k}")
         assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 2.0, k).view(np.uint32)), k
