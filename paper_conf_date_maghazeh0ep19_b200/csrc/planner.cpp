@@ -544,12 +544,31 @@ ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragmen
   out.budget = (int64_t)std::floor((double)cache_bytes * frac);
   bool force = (pol.flags & KTILER_PF_FORCE_MINIMAL) != 0;
   const bool resident = (pol.flags & KTILER_PF_RESIDENT_BUDGET) != 0;
-  if (pol.kind != KTILER_FRAG_ALG1) {
+  if (pol.kind != KTILER_FRAG_ALG1 && pol.kind != KTILER_FRAG_CHAIN) {
     std::vector<int> all(g.topo.begin(), g.topo.end());
     out.clusters.push_back(all);
     out.cluster_cost.push_back(0.0);
   }
   switch (pol.kind) {
+    case KTILER_FRAG_CHAIN: {  // fixed partition: `rows` consecutive nodes per cluster
+      if (pol.rows < 1) return fail(KTILER_E_INVALID, "CHAIN policy needs rows >= 1 (nodes per cluster)");
+      const int nn = (int)g.topo.size();
+      for (int a = 0; a < nn; a += (int)pol.rows) {
+        std::vector<int> mem(g.topo.begin() + a, g.topo.begin() + std::min<int64_t>(nn, a + pol.rows));
+        Partitioner p(g, out, resident);
+        std::fill(p.in_c.begin(), p.in_c.end(), (uint8_t)0);
+        for (int v : mem) p.in_c[v] = 1;
+        p.budget_lines = out.budget / 128;
+        p.rows_cap = 0;
+        p.force_minimal = force;
+        p.cluster_id = (int32_t)out.clusters.size();
+        ktiler_status st = p.run();
+        if (st) return st;
+        out.clusters.push_back(mem);
+        out.cluster_cost.push_back(0.0);
+      }
+      return KTILER_OK;
+    }
     case KTILER_FRAG_ALG1: return alg1(g, out.budget / 128, pol.alg1_thld, resident, out);
     case KTILER_FRAG_NONE: untiled(g, out); return KTILER_OK;
     case KTILER_FRAG_BUDGET: {

@@ -18,7 +18,7 @@ OK, E_INVALID, E_CYCLE, E_UNTILEABLE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = 
 BUF_INTERNAL = 1
 READ, WRITE = 1, 2
 OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM, OP_JACOBI = range(7)
-FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1 = range(5)
+FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1, FRAG_CHAIN = range(6)
 EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE = range(7)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL, PF_RESIDENT_BUDGET = 1, 2, 4, 8
 
@@ -26,7 +26,7 @@ EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRA
               "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG, "chain": EXEC_GRAPH_CHAIN,
               "wave": EXEC_GRAPH_WAVE}
 FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE,
-              "alg1": FRAG_ALG1}
+              "alg1": FRAG_ALG1, "chain": FRAG_CHAIN}
 
 
 SELFTEST_SQRT = 0
