@@ -187,7 +187,7 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
 }
 
 template <int OP, bool SCALAR>
-__global__ void __launch_bounds__(256, (OP == 1 || OP == 3 || OP == 6) ? 3 : 4) op_kernel(const __grid_constant__ KParams p) {
+__global__ void __launch_bounds__(256, (OP == 1 || OP == 3 || OP == 6) ? 2 : 4) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
@@ -1017,6 +1017,15 @@ void fold_dag_discards(ktiler_plan_s* P) {
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+// L2 sector promotion of the TMA requests (KTILER_TMA_PROMOTION = 0 / 64 / 128 / 256 bytes;
+// default 256).
+CUtensorMapL2promotion l2_promotion() {
+  static const int v = getenv("KTILER_TMA_PROMOTION") ? atoi(getenv("KTILER_TMA_PROMOTION")) : 256;
+  return v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+                : (v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                           : (v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B));
+}
+
 EncodeTiledFn get_encode() {
   static EncodeTiledFn fn = nullptr;
   static bool tried = false;
@@ -1057,7 +1066,7 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
   cuuint64_t strides[2] = {(cuuint64_t)B.d.pitch_bytes, (cuuint64_t)B.d.frame_stride_bytes};
   cuuint32_t box[3] = {(cuuint32_t)(bw / 4), (cuuint32_t)bh, 1}, es[3] = {1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, B.d.base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   CU_TENSOR_MAP_SWIZZLE_NONE, l2_promotion(), CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return false;
   *box_bytes = (uint32_t)(bw * bh);
   return true;

@@ -48,6 +48,12 @@ __device__ __forceinline__ void st16_stream(void* p, uint4 v, uint64_t pol) {
                "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol)
                : "memory");
 }
+// 32 bytes (8 words, 32-B aligned) in one 256-bit store (sm_100: STG.E.256)
+__device__ __forceinline__ void st32(void* p, const uint32_t* v) {
+  asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]),
+               "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
+}
 __device__ __forceinline__ void discard_line(const void* p) {
   asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
 }
@@ -122,8 +128,6 @@ __device__ void scalar_tile(int op, const DBuf& in, const DBuf& out, const Tile&
 // ---------------------------------------------------------------------------------
 // staging
 // ---------------------------------------------------------------------------------
-constexpr int BLUR_R = 8;
-constexpr int SOBEL_R = 4;
 
 // ---- TMA bulk copies completing on an mbarrier (the Blackwell async proxy) ----
 __device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
@@ -282,25 +286,26 @@ __device__ __forceinline__ void store_u8_16(uint8_t* d, int64_t x, int64_t W, ui
 }
 
 // ---------------------------------------------------------------------------------
-// gray: rgb8 -> u8.  Y = (19595R + 38470G + 7471B + 32768) >> 16 computed as
-// 256*dp4a(px, [76,150,29,0]) + dp4a(px, [139,70,47,0]) + 32768, whose byte 2 is Y
-// (19595 = 76*256+139, 38470 = 150*256+70, 7471 = 29*256+47; the sum is < 2^24).
+// gray: rgb8 -> u8.  Y = (19595R + 38470G + 7471B + 32768) >> 16.  The weights are u16,
+// the channels u8: dp2a (two u16 x u8 products + accumulator, lower or upper byte pair of
+// the pixel word) takes them straight from the interleaved words, two dp2a per pixel and
+// no unpacking.  Pixels 4j..4j+3 live in words (w0, w1, w2) = [R0 G0 B0 R1] [G1 B1 R2 G2]
+// [B2 R3 G3 B3]; the weight pairs follow the byte pairs each dp2a sees.  The sum is
+// < 2^24, so byte 2 of it is Y.
 // ---------------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t luma_sum(uint32_t px) {
-  uint32_t hi = __dp4a(px, 0x001D964Cu, 0u);
-  uint32_t lo = __dp4a(px, 0x002F468Bu, 32768u);
-  return hi * 256u + lo;
+constexpr uint32_t WR = 19595u, WG = 38470u, WB = 7471u;
+__device__ __forceinline__ uint32_t pk16(uint32_t lo, uint32_t hi) { return lo | (hi << 16); }
+__device__ __forceinline__ void luma4(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t s[4]) {
+  s[0] = __dp2a_hi(pk16(WB, 0), w0, __dp2a_lo(pk16(WR, WG), w0, 32768u));   // R0 G0 | B0 (R1)
+  s[1] = __dp2a_lo(pk16(WG, WB), w1, __dp2a_hi(pk16(0, WR), w0, 32768u));   // (B0) R1 | G1 B1
+  s[2] = __dp2a_lo(pk16(WB, 0), w2, __dp2a_hi(pk16(WR, WG), w1, 32768u));   // R2 G2 | B2 (R3)
+  s[3] = __dp2a_hi(pk16(WG, WB), w2, __dp2a_lo(pk16(0, WR), w2, 32768u));   // (B2) R3 | G3 B3
 }
 
 __device__ __forceinline__ uint4 gray16(const uint32_t w[12]) {
   uint32_t s[16];
 #pragma unroll
-  for (int k = 0; k < 16; ++k) {
-    const int b = 3 * k, q = b >> 2, sh = b & 3;
-    // bytes 3k..3k+2 into bytes 0..2 (byte 3 has weight 0 in both dot products)
-    uint32_t px = sh == 0 ? w[q] : (sh == 1 ? (w[q] >> 8) : prmt(w[q], w[q + 1], 0x3210 + 0x1111 * sh));
-    s[k] = luma_sum(px);
-  }
+  for (int j = 0; j < 4; ++j) luma4(w[3 * j], w[3 * j + 1], w[3 * j + 2], s + 4 * j);
   uint4 o;
   uint32_t* ow = &o.x;
 #pragma unroll
@@ -314,16 +319,25 @@ __device__ __forceinline__ uint4 gray16(const uint32_t w[12]) {
 
 // Items of a tile = (row group g, 16-px column segment s), item it = g * nseg + s, dealt
 // round-robin to the CTA's threads.  One loop, so each op's (fully unrolled) item body is
-// instantiated once — several copies overflow the instruction cache.  The B200 geometry
-// (256-px tiles, nseg = 16) takes the shift path for the index split.
+// instantiated once — several copies overflow the instruction cache.  Power-of-two
+// segment counts (the B200 geometry) take the shift path for the index split.
 template <class F>
 __device__ __forceinline__ void for_items(int nseg, int ngrp, int nt, int tid, F&& f) {
   const int total = nseg * ngrp;
-  const bool n16 = nseg == 16;
+  const bool pow2 = (nseg & (nseg - 1)) == 0;
+  const int sh = __ffs(nseg) - 1;
   for (int it = tid; it < total; it += nt) {
-    const int g = n16 ? (it >> 4) : it / nseg;
+    const int g = pow2 ? (it >> sh) : it / nseg;
     f(g, it - g * nseg);
   }
+}
+
+// Rows per item of the sliding-window stencils: as few row groups as still give every
+// thread an item, so the halo rows each item re-reads (4 for blur5, 2 for sobel3) are
+// amortised over as many output rows as the CTA's thread count allows.
+__device__ __forceinline__ int rows_per_item(int rows, int nseg, int nt) {
+  const int ngrp = max(1, nt / nseg);
+  return (rows + ngrp - 1) / ngrp;
 }
 
 // Output base of a tile (pixel (x0, y0) of frame z) and its "all segments full" flag.
@@ -407,14 +421,17 @@ __device__ __forceinline__ uint4 vblur_pack(const uint32_t* h0, const uint32_t* 
                     prmt(v[6], v[7], 0x7531));
 }
 
-template <int R>
+// One item = a 16-px column strip of rpi output rows.  The 5-row window of horizontal
+// partials h[] rotates through five register arrays; the row loop is unrolled by 5 so
+// every slot index is a compile-time constant (no register moves), whatever rpi is.
 __device__ void blur_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
   const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (t.fseg() + 2);
   const bool full = (t.x1 - t.x0) == 16 * nseg;
   uint8_t* const ob = tile_out(out, t, 1);
   const int pitch = (int)out.pitch;
-  for_items(nseg, (rows + R - 1) / R, nt, tid, [&](int g, int s) {
-    const int ra = g * R, rb = min(ra + R, rows);
+  const int rpi = rows_per_item(rows, nseg, nt);
+  for_items(nseg, (rows + rpi - 1) / rpi, nt, tid, [&](int g, int s) {
+    const int ra = g * rpi, n = min(rpi, rows - ra);
     const uint8_t* col = sm + 16 * (s + 1) + ra * stride;  // staged row r holds image row y0 - 2 + r
     uint8_t* d = ob + ra * pitch + 16 * s;
     uint32_t h[5][8];
@@ -424,13 +441,16 @@ __device__ void blur_compute(const DBuf& out, const Tile& t, const uint8_t* sm, 
       smem_window(col + i * stride, w);
       hblur16(w, h[i]);
     }
+    for (int r0 = 0; r0 < n; r0 += 5) {
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (ra + r >= rb) break;
-      smem_window(col + (r + 4) * stride, w);
-      hblur16(w, h[(r + 4) % 5]);
-      const uint4 o = vblur_pack(h[r % 5], h[(r + 1) % 5], h[(r + 2) % 5], h[(r + 3) % 5], h[(r + 4) % 5]);
-      if (full) st16(d + r * pitch, o); else store_u8_16(d + r * pitch, t.x0 + 16 * s, out.W, o);
+      for (int k = 0; k < 5; ++k) {
+        const int r = r0 + k;
+        if (r >= n) break;
+        smem_window(col + (r + 4) * stride, w);
+        hblur16(w, h[(k + 4) % 5]);
+        const uint4 o = vblur_pack(h[k % 5], h[(k + 1) % 5], h[(k + 2) % 5], h[(k + 3) % 5], h[(k + 4) % 5]);
+        if (full) st16(d + r * pitch, o); else store_u8_16(d + r * pitch, t.x0 + 16 * s, out.W, o);
+      }
     }
   });
 }
@@ -518,64 +538,76 @@ __device__ __forceinline__ float2 mag2(uint32_t gx, uint32_t gy) {
   return sqrt2_int(__ffma2_rn(X, X, __fmul2_rn(Y, Y)));
 }
 
-template <int R>
+// One item = a 16-px column strip of rpi output rows; the 3-row window rotates through
+// three register sets, the row loop unrolled by 3 (static slot indices).
+__device__ __forceinline__ void sobel_row(const SobelRow& T, const SobelRow& M, const SobelRow& B, uint8_t* drow,
+                                          bool seg_full, int64_t x0, int64_t W) {
+  // column smoothing S = top + 2 mid + bot, difference D = bot - top + 255 (per lane)
+  uint32_t SE[6], SO[6], DE[6], DO[6];
+#pragma unroll
+  for (int q = 0; q < 6; ++q) {
+    if (q >= 1) {
+      SE[q] = T.e[q] + B.e[q] + 2u * M.e[q];
+      DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
+    }
+    if (q <= 4) {
+      SO[q] = T.o[q] + B.o[q] + 2u * M.o[q];
+      DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
+    }
+  }
+  float* dst = reinterpret_cast<float*>(drow);
+  uint32_t o[16];  // columns x .. x+15
+#pragma unroll
+  for (int q = 1; q <= 4; ++q) {
+    const uint32_t gxe = SO[q] + 0x03FC03FCu - prmt(SO[q - 1], SO[q], 0x5432);
+    const uint32_t gye = prmt(DO[q - 1], DO[q], 0x5432) + 2u * DE[q] + DO[q];
+    const uint32_t gxo = prmt(SE[q], SE[q + 1], 0x5432) + 0x03FC03FCu - SE[q];
+    const uint32_t gyo = DE[q] + 2u * DO[q] + prmt(DE[q], DE[q + 1], 0x5432);
+    const float2 ev = mag2(gxe, gye);  // columns c, c+2 (c = x + 4q - 4)
+    const float2 od = mag2(gxo, gyo);  // columns c+1, c+3
+    o[4 * q - 4] = __float_as_uint(ev.x);
+    o[4 * q - 3] = __float_as_uint(od.x);
+    o[4 * q - 2] = __float_as_uint(ev.y);
+    o[4 * q - 1] = __float_as_uint(od.y);
+  }
+  if (seg_full) {
+    // two 256-bit stores: each covers whole 32-B sectors (16-B stores at a 64-B lane stride
+    // would write every sector in two halves, doubling the L2 write requests)
+    st32(dst, o);
+    st32(dst + 8, o + 8);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 16; ++k)
+      if (x0 + k < W) dst[k] = __uint_as_float(o[k]);
+  }
+}
+
 __device__ void sobel_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
   const int nseg = t.nseg(), rows = t.rows(), stride = 16 * (t.fseg() + 2);
   const bool full = (t.x1 - t.x0) == 16 * nseg;
   uint8_t* const ob = tile_out(out, t, 4);
   const int pitch = (int)out.pitch;
-  for_items(nseg, (rows + R - 1) / R, nt, tid, [&](int g, int s) {
-    const int ra = g * R, rb = min(ra + R, rows);
+  const int rpi = rows_per_item(rows, nseg, nt);
+  for_items(nseg, (rows + rpi - 1) / rpi, nt, tid, [&](int g, int s) {
+    const int ra = g * rpi, n = min(rpi, rows - ra);
     const uint8_t* col = sm + 16 * (s + 1) + ra * stride;  // staged row r holds image row y0 - 1 + r
     uint8_t* drow = ob + ra * pitch + 64 * s;
     const bool seg_full = full || t.x0 + 16 * s + 16 <= out.W;
+    const int64_t x0 = t.x0 + 16 * s;
     SobelRow w[3];
     uint32_t tw[6];
     smem_window(col, tw);
     sobel_split(tw, w[0]);
     smem_window(col + stride, tw);
     sobel_split(tw, w[1]);
+    for (int r0 = 0; r0 < n; r0 += 3) {
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (ra + r >= rb) break;
-      smem_window(col + (r + 2) * stride, tw);
-      sobel_split(tw, w[(r + 2) % 3]);
-      const SobelRow& T = w[r % 3];
-      const SobelRow& M = w[(r + 1) % 3];
-      const SobelRow& B = w[(r + 2) % 3];
-      // column smoothing S = top + 2 mid + bot, difference D = bot - top + 255 (per lane)
-      uint32_t SE[6], SO[6], DE[6], DO[6];
-#pragma unroll
-      for (int q = 0; q < 6; ++q) {
-        if (q >= 1) {
-          SE[q] = T.e[q] + B.e[q] + 2u * M.e[q];
-          DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
-        }
-        if (q <= 4) {
-          SO[q] = T.o[q] + B.o[q] + 2u * M.o[q];
-          DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
-        }
-      }
-      float* dst = reinterpret_cast<float*>(drow + r * pitch);
-#pragma unroll
-      for (int q = 1; q <= 4; ++q) {
-        const uint32_t gxe = SO[q] + 0x03FC03FCu - prmt(SO[q - 1], SO[q], 0x5432);
-        const uint32_t gye = prmt(DO[q - 1], DO[q], 0x5432) + 2u * DE[q] + DO[q];
-        const uint32_t gxo = prmt(SE[q], SE[q + 1], 0x5432) + 0x03FC03FCu - SE[q];
-        const uint32_t gyo = DE[q] + 2u * DO[q] + prmt(DE[q], DE[q + 1], 0x5432);
-        const float2 ev = mag2(gxe, gye);  // columns c, c+2 (c = x + 4q - 4)
-        const float2 od = mag2(gxo, gyo);  // columns c+1, c+3
-        if (seg_full) {
-          st16(dst + 4 * (q - 1), make_uint4(__float_as_uint(ev.x), __float_as_uint(od.x), __float_as_uint(ev.y),
-                                             __float_as_uint(od.y)));
-        } else {
-          const int64_t x = t.x0 + 16 * s + 4 * (q - 1);
-          float* d = dst + 4 * (q - 1);
-          if (x < out.W) d[0] = ev.x;
-          if (x + 1 < out.W) d[1] = od.x;
-          if (x + 2 < out.W) d[2] = ev.y;
-          if (x + 3 < out.W) d[3] = od.y;
-        }
+      for (int k = 0; k < 3; ++k) {
+        const int r = r0 + k;
+        if (r >= n) break;
+        smem_window(col + (r + 2) * stride, tw);
+        sobel_split(tw, w[(k + 2) % 3]);
+        sobel_row(w[k % 3], w[(k + 1) % 3], w[(k + 2) % 3], drow + r * pitch, seg_full, x0, out.W);
       }
     }
   });
@@ -661,9 +693,9 @@ __device__ __forceinline__ void compute_tile(int op, const DBuf& out, const Tile
                                              int nt, int tid, const DBuf* aux = nullptr) {
   switch (op) {
     case 0: gray_compute(out, t, sm, nt, tid); break;
-    case 1: blur_compute<BLUR_R>(out, t, sm, nt, tid); break;
+    case 1: blur_compute(out, t, sm, nt, tid); break;
     case 2: down_compute(out, t, sm, nt, tid); break;
-    case 3: sobel_compute<SOBEL_R>(out, t, sm, nt, tid); break;
+    case 3: sobel_compute(out, t, sm, nt, tid); break;
     case 4: thresh_compute(out, t, sm, T, nt, tid); break;
     case 6: jacobi_compute(out, *aux, t, sm, T, nt, tid); break;  // T = a2 (alpha^2)
   }

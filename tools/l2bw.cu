@@ -1,0 +1,87 @@
+// L2 (LTS) throughput microbenchmark — the secondary ceiling of SURVEY §8(d): every byte
+// of the tiled schedule (hits and misses alike) passes through the L2 slices, so their
+// throughput, not HBM, bounds a schedule whose intermediates stay resident.
+//
+// Modes, each over a buffer of `mb` MiB touched once beforehand (resident when mb << L2):
+//   read   : every thread streams 16-B ld.global.cg loads over the buffer, XOR-reduced
+//   write  : 16-B st.global over the buffer
+//   copy   : read half A, write half B (the op kernels' pattern)
+// Grid = 148 x 8 CTAs x 256 threads, grid-stride, 20 passes per launch (resident sizes);
+// CUDA events around `iters` launches;
+// prints one JSON line per mode with bytes / time.  Diagnostic tool, not product code.
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/l2bw tools/l2bw.cu
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+
+__global__ void rd(const uint4* __restrict__ p, size_t n, unsigned* sink, int reps) {
+  uint32_t acc = 0;
+  for (int k = 0; k < reps; ++k)
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint4 v;
+    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p + i));
+    acc ^= v.x ^ v.y ^ v.z ^ v.w;
+  }
+  if (acc == 0x12345678u) *sink = acc;
+}
+__global__ void wr(uint4* __restrict__ p, size_t n, unsigned salt, int reps) {
+  for (int k = 0; k < reps; ++k)
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    p[i] = make_uint4(salt + k, (unsigned)i, salt, (unsigned)i);
+}
+__global__ void cp(const uint4* __restrict__ a, uint4* __restrict__ b, size_t n, int reps) {
+  for (int k = 0; k < reps; ++k)
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint4 v;
+    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(a + i));
+    b[i] = v;
+  }
+}
+
+int main(int argc, char** argv) {
+  const int iters = 50;
+  const size_t sizes_mb[] = {16, 32, 48, 64, 96, 4096};
+  int nsm = 0;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+  uint4* buf;
+  unsigned* sink;
+  cudaMalloc(&buf, (size_t)4096 << 20);
+  cudaMalloc(&sink, 4);
+  cudaMemset(buf, 1, (size_t)4096 << 20);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  const int grid = nsm * 8, block = 256;
+  for (size_t mb : sizes_mb) {
+    const size_t n = (mb << 20) / 16;
+    const int it = mb > 1024 ? 5 : iters;
+    const int reps = mb > 1024 ? 1 : 20;  // passes per launch (no launch gaps in the resident cases)
+    for (int mode = 0; mode < 3; ++mode) {
+      auto run = [&]() {
+        if (mode == 0) rd<<<grid, block>>>(buf, n, sink, reps);
+        else if (mode == 1) wr<<<grid, block>>>(buf, n, 7u, reps);
+        else cp<<<grid, block>>>(buf, buf + n / 2, n / 2, reps);
+      };
+      run();
+      run();
+      cudaEventRecord(e0);
+      for (int i = 0; i < it; ++i) run();
+      cudaEventRecord(e1);
+      cudaEventSynchronize(e1);
+      float ms = 0;
+      cudaEventElapsedTime(&ms, e0, e1);
+      const double bytes = (double)(mb << 20) * it * reps;  // copy: n/2 read + n/2 written = mb
+      printf("{\"tool\": \"l2bw\", \"mode\": \"%s\", \"mb\": %zu, \"GBps\": %.1f, \"us_per_pass\": %.2f}\n",
+             mode == 0 ? "read" : (mode == 1 ? "write" : "copy"), mb, bytes / (ms * 1e-3) / 1e9, ms * 1e3 / (it * reps));
+    }
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    fprintf(stderr, "%s\n", cudaGetErrorString(e));
+    return 1;
+  }
+  return 0;
+}
