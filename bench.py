@@ -61,13 +61,15 @@ def parse():
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=0.5)
+    ap.add_argument("--l2-fraction", type=float, default=0.75)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="frames: weak = every rank runs the whole batch (per-GPU work fixed), strong = split it")
     ap.add_argument("--window", type=int, default=2)
-    ap.add_argument("--no-discard", action="store_true")
+    ap.add_argument("--discard", action="store_true",
+                    help="discard dead intermediate lines (DRAM -55%% but slower on B200: DESIGN.md §6)")
+    ap.add_argument("--no-discard", action="store_true", help="(default) keep dead lines")
     ap.add_argument("--pdl", action="store_true")
     ap.add_argument("--ctas", type=int, default=0)
     ap.add_argument("--skew", type=int, default=0)
@@ -137,6 +139,17 @@ def peaks():
         return float(d["hbm_gbs"]), "measured: MEASURED_PEAKS.json hbm_gbs (torch copy, read+write)"
     except Exception:
         return 6650.0, "fallback: B200_PROFILING.md"
+
+
+def l2_ceiling():
+    """Measured L2 read / write-to-resident throughput (tools/l2bw.cu, 64 MiB resident
+    buffer) from profiles/, or None."""
+    try:
+        rows = [json.loads(l) for l in open(os.path.join(ROOT, "profiles", "r01_l2bw.jsonl"))]
+        r = {d["mode"]: d["GBps"] for d in rows if d["mb"] == 64}
+        return {"read": r["read"], "write": r["write"], "source": "profiles/r01_l2bw.jsonl (tools/l2bw, 64 MiB resident)"}
+    except Exception:
+        return None
 
 
 def traffic_for(cfg: dict):
@@ -282,7 +295,7 @@ def main():
         G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
         pix_rank = W * H * per
     torch.cuda.synchronize()
-    discard = not args.no_discard
+    discard = args.discard and not args.no_discard
     resident = not args.no_resident
     pol = dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode, discard=discard,
                pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew, window=args.window, resident_budget=resident)
@@ -360,6 +373,16 @@ def main():
                      "peak_source": peak_src},
         "clocks": clk.summary(),
     }
+    l2 = l2_ceiling()
+    if l2:
+        # secondary ceiling: every byte the kernels read or write passes the L2 slices;
+        # writes into L2 are capped near the HBM write rate on B200 (dirty lines are written
+        # back within microseconds), reads of resident lines at ~2.6x HBM
+        rd, wr = 6.25 * pix, 3.5 * pix
+        floor_ms = (rd / (l2["read"] * 1e9) + wr / (l2["write"] * 1e9)) * 1e3
+        line["roofline"]["l2"] = {"bound": "l2", "read_peak": l2["read"], "write_peak": l2["write"], "unit": "GB/s",
+                                  "algorithmic_bytes": "6.25 B/px read + 3.5 B/px written (all five kernels)",
+                                  "floor_ms": floor_ms, "frac": floor_ms / ms, "source": l2["source"]}
     if not args.no_untiled:
         un = p.b.g.plan(0, kind="none", exec_mode="graph", discard=False)
         ms_un = timed(lambda: (sp.exchange() if sp is not None and world > 1 else None, un.execute(s)),
