@@ -51,7 +51,7 @@ WORKLOADS = {
 }
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
@@ -81,7 +81,7 @@ def parse():
     ap.add_argument("--no-trace", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
-    return ap.parse_args()
+    return ap.parse_args(argv)
 
 
 class Clocks:
@@ -254,6 +254,13 @@ def trace_shares(pipe, pol):
     return out, span / 1e6, per
 
 
+def policy(args) -> dict:
+    """The fragment policy of the timed step (also used by tests/test_gpu_fullsize.py)."""
+    return dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode,
+                discard=args.discard and not args.no_discard, pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew,
+                window=args.window, resident_budget=not args.no_resident)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -295,10 +302,8 @@ def main():
         G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
         pix_rank = W * H * per
     torch.cuda.synchronize()
-    discard = args.discard and not args.no_discard
-    resident = not args.no_resident
-    pol = dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode, discard=discard,
-               pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew, window=args.window, resident_budget=resident)
+    pol = policy(args)
+    discard, resident = pol["discard"], pol["resident_budget"]
     plan = p.plan(0, **pol)
     st = plan.stats()
 

@@ -50,11 +50,20 @@ def splitmix64_np(z: np.ndarray) -> np.ndarray:
 
 def uniform(seed: int, W: int, H: int, F: int = 1) -> np.ndarray:
     """uint8 array [F, H, W, 3] of hashed bytes."""
-    n = F * H * W * 3
-    i = np.arange(n, dtype=np.uint64)
-    with np.errstate(over="ignore"):
-        i += np.uint64((seed * K_SEED) & M64)
-    return (splitmix64_np(i) & np.uint64(0xFF)).astype(np.uint8).reshape(F, H, W, 3)
+    return uniform_rows(seed, W, H, 0, H, F)
+
+
+def uniform_rows(seed: int, W: int, H: int, y0: int, y1: int, F: int = 1, f0: int = 0) -> np.ndarray:
+    """Rows [y0, y1) of frames [f0, f0+F) of ``uniform(seed)`` (global size W x H): uint8
+    [F, y1-y0, W, 3], byte for byte the same as the slice of the whole image."""
+    out = np.empty((F, y1 - y0, W, 3), dtype=np.uint8)
+    for k in range(F):
+        base = (((f0 + k) * H + y0) * W) * 3
+        i = np.arange(base, base + (y1 - y0) * W * 3, dtype=np.uint64)
+        with np.errstate(over="ignore"):
+            i += np.uint64((seed * K_SEED) & M64)
+        out[k] = (splitmix64_np(i) & np.uint64(0xFF)).astype(np.uint8).reshape(y1 - y0, W, 3)
+    return out
 
 
 def scene_rects(s: int, W: int, H: int):
@@ -72,18 +81,27 @@ def scene_rects(s: int, W: int, H: int):
 
 
 def scene_frame(s: int, W: int, H: int) -> np.ndarray:
-    img = np.empty((H, W, 3), dtype=np.int32)
+    return scene_rows(s, W, H, 0, H)
+
+
+def scene_rows(s: int, W: int, H: int, y0: int, y1: int) -> np.ndarray:
+    """Rows [y0, y1) of frame seed ``s`` of the scene (global size W x H): uint8
+    [y1-y0, W, 3], byte for byte the same as the slice of the whole frame."""
+    n = y1 - y0
+    img = np.empty((n, W, 3), dtype=np.int32)
     img[:, :, 0] = (np.arange(W, dtype=np.int64) * 255 // W)[None, :]
-    img[:, :, 1] = (np.arange(H, dtype=np.int64) * 255 // H)[:, None]
+    img[:, :, 1] = (np.arange(y0, y1, dtype=np.int64) * 255 // H)[:, None]
     img[:, :, 2] = 128
-    for (x0, y0, x1, y1, r, g, b) in scene_rects(s, W, H):
-        img[y0:y1, x0:x1, 0] = r
-        img[y0:y1, x0:x1, 1] = g
-        img[y0:y1, x0:x1, 2] = b
-    i = np.arange(H * W * 3, dtype=np.uint64)
+    for (x0, ry0, x1, ry1, r, g, b) in scene_rects(s, W, H):
+        a, c = max(ry0, y0), min(ry1, y1)
+        if a < c:
+            img[a - y0:c - y0, x0:x1, 0] = r
+            img[a - y0:c - y0, x0:x1, 1] = g
+            img[a - y0:c - y0, x0:x1, 2] = b
+    i = np.arange(y0 * W * 3, y1 * W * 3, dtype=np.uint64)
     with np.errstate(over="ignore"):
         i += np.uint64((s * K_NOISE) & M64)
-    noise = (splitmix64_np(i) & np.uint64(15)).astype(np.int32).reshape(H, W, 3) - 8
+    noise = (splitmix64_np(i) & np.uint64(15)).astype(np.int32).reshape(n, W, 3) - 8
     return np.clip(img + noise, 0, 255).astype(np.uint8)
 
 
