@@ -6,6 +6,8 @@
 //   read   : every thread streams 16-B ld.global.cg loads over the buffer, XOR-reduced
 //   write  : 16-B st.global over the buffer
 //   copy   : read half A, write half B (the op kernels' pattern)
+//   write_evict_last / write_evict_unchanged : the write with an L2 createpolicy hint
+//   write256 / read256 : 32 B per thread per instruction (STG.E.256 / LDG.E.256)
 // Grid = 148 x 8 CTAs x 256 threads, grid-stride, 20 passes per launch (resident sizes);
 // CUDA events around `iters` launches;
 // prints one JSON line per mode with bytes / time.  Diagnostic tool, not product code.
@@ -32,6 +34,38 @@ __global__ void wr(uint4* __restrict__ p, size_t n, unsigned salt, int reps) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
     p[i] = make_uint4(salt + k, (unsigned)i, salt, (unsigned)i);
 }
+// resident writes with an L2 eviction-priority hint (createpolicy): evict_last / evict_unchanged
+__global__ void wr_hint(uint4* __restrict__ p, size_t n, unsigned salt, int reps, int hint) {
+  uint64_t pol;
+  if (hint == 0) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  else asm volatile("createpolicy.fractional.L2::evict_unchanged.b64 %0, 1.0;" : "=l"(pol));
+  for (int k = 0; k < reps; ++k)
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+      asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;" ::"l"(p + i), "r"(salt + k), "r"((unsigned)i),
+                   "r"(salt), "r"((unsigned)i), "l"(pol)
+                   : "memory");
+}
+// resident writes, 32 B per thread per instruction (st.global.v8.b32 = STG.E.256)
+__global__ void wr256(uint4* __restrict__ p, size_t n, unsigned salt, int reps) {
+  for (int k = 0; k < reps; ++k)
+    for (size_t i = 2 * (blockIdx.x * (size_t)blockDim.x + threadIdx.x); i + 1 < n; i += 2 * (size_t)gridDim.x * blockDim.x)
+      asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p + i), "r"(salt + k), "r"((unsigned)i),
+                   "r"(salt), "r"((unsigned)i), "r"(salt), "r"(salt), "r"(salt), "r"(salt)
+                   : "memory");
+}
+// resident reads, 32 B per thread per instruction (ld.global.cg.v8.b32)
+__global__ void rd256(const uint4* __restrict__ p, size_t n, unsigned* sink, int reps) {
+  uint32_t acc = 0;
+  for (int k = 0; k < reps; ++k)
+    for (size_t i = 2 * (blockIdx.x * (size_t)blockDim.x + threadIdx.x); i + 1 < n; i += 2 * (size_t)gridDim.x * blockDim.x) {
+      uint32_t v[8];
+      asm volatile("ld.global.cg.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                   : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+                   : "l"(p + i));
+      acc ^= v[0] ^ v[1] ^ v[2] ^ v[3] ^ v[4] ^ v[5] ^ v[6] ^ v[7];
+    }
+  if (acc == 0x12345678u) *sink = acc;
+}
 __global__ void cp(const uint4* __restrict__ a, uint4* __restrict__ b, size_t n, int reps) {
   for (int k = 0; k < reps; ++k)
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
@@ -43,7 +77,7 @@ __global__ void cp(const uint4* __restrict__ a, uint4* __restrict__ b, size_t n,
 
 int main(int argc, char** argv) {
   const int iters = 50;
-  const size_t sizes_mb[] = {16, 32, 48, 64, 96, 4096};
+  const size_t sizes_mb[] = {4, 8, 16, 32, 64, 96, 4096};
   int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
   uint4* buf;
@@ -59,11 +93,14 @@ int main(int argc, char** argv) {
     const size_t n = (mb << 20) / 16;
     const int it = mb > 1024 ? 5 : iters;
     const int reps = mb > 1024 ? 1 : 20;  // passes per launch (no launch gaps in the resident cases)
-    for (int mode = 0; mode < 3; ++mode) {
+    for (int mode = 0; mode < 7; ++mode) {
       auto run = [&]() {
         if (mode == 0) rd<<<grid, block>>>(buf, n, sink, reps);
         else if (mode == 1) wr<<<grid, block>>>(buf, n, 7u, reps);
-        else cp<<<grid, block>>>(buf, buf + n / 2, n / 2, reps);
+        else if (mode == 2) cp<<<grid, block>>>(buf, buf + n / 2, n / 2, reps);
+        else if (mode < 5) wr_hint<<<grid, block>>>(buf, n, 7u, reps, mode - 3);
+        else if (mode == 5) wr256<<<grid, block>>>(buf, n, 7u, reps);
+        else rd256<<<grid, block>>>(buf, n, sink, reps);
       };
       run();
       run();
@@ -75,7 +112,7 @@ int main(int argc, char** argv) {
       cudaEventElapsedTime(&ms, e0, e1);
       const double bytes = (double)(mb << 20) * it * reps;  // copy: n/2 read + n/2 written = mb
       printf("{\"tool\": \"l2bw\", \"mode\": \"%s\", \"mb\": %zu, \"GBps\": %.1f, \"us_per_pass\": %.2f}\n",
-             mode == 0 ? "read" : (mode == 1 ? "write" : "copy"), mb, bytes / (ms * 1e-3) / 1e9, ms * 1e3 / (it * reps));
+             mode == 0 ? "read" : (mode == 1 ? "write" : (mode == 2 ? "copy" : (mode == 3 ? "write_evict_last" : (mode == 4 ? "write_evict_unchanged" : (mode == 5 ? "write256" : "read256"))))), mb, bytes / (ms * 1e-3) / 1e9, ms * 1e3 / (it * reps));
     }
   }
   cudaError_t e = cudaGetLastError();
