@@ -1145,7 +1145,14 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   if (e != cudaSuccess) return cuda_fail(e, "cudaGraphCreate");
   std::vector<std::vector<cudaGraphNode_t>> nodes_of(nsub);
   const std::vector<std::vector<int>> edges = dag_edges(P);
-  auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, cudaGraphNode_t* node) -> ktiler_status {
+  // PF_PDL: the edges from a sub-kernel's producers (Schedule::sub_deps; with
+  // KTILER_DAG_PDL_EDGES=all every kernel edge) are programmatic: the consumer's CTAs may
+  // become resident while the producer's last wave drains and wait in griddepcontrol.wait
+  // (full completion + memory flush of every programmatic producer) before reading.
+  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
+  static const bool pdl_all = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "all");
+  auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, const std::vector<uint8_t>& prog,
+                      cudaGraphNode_t* node) -> ktiler_status {
     kfn_t fn = launch_fn(L);
     int64_t grid = 0;
     ktiler_status ps = prep_launch(P, L, fn, &grid);
@@ -1157,19 +1164,47 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     kp.blockDim = L.block;
     kp.sharedMemBytes = (unsigned)L.smem;
     kp.kernelParams = args;
-    cudaError_t ee = cudaGraphAddKernelNode(node, gr, deps.data(), deps.size(), &kp);
+    if (!pdl) {
+      cudaError_t ee = cudaGraphAddKernelNode(node, gr, deps.data(), deps.size(), &kp);
+      if (ee != cudaSuccess) return cuda_fail(ee, "cudaGraphAddKernelNode");
+      return KTILER_OK;
+    }
+    cudaError_t ee = cudaGraphAddKernelNode(node, gr, nullptr, 0, &kp);
     if (ee != cudaSuccess) return cuda_fail(ee, "cudaGraphAddKernelNode");
+    std::vector<cudaGraphEdgeData> ed(deps.size());
+    for (size_t j = 0; j < deps.size(); ++j) {
+      std::memset(&ed[j], 0, sizeof(ed[j]));
+      if (!prog.empty() && prog[j]) {
+        ed[j].from_port = cudaGraphKernelNodePortProgrammatic;
+        ed[j].type = cudaGraphDependencyTypeProgrammatic;
+      }
+    }
+    std::vector<cudaGraphNode_t> to(deps.size(), *node);
+    if (!deps.empty() && (ee = cudaGraphAddDependencies_v2(gr, deps.data(), to.data(), ed.data(), deps.size())) != cudaSuccess)
+      return cuda_fail(ee, "cudaGraphAddDependencies_v2");
     return KTILER_OK;
   };
   size_t li = 0;
   for (int i = 0; i < nsub; ++i) {
+    std::vector<std::pair<cudaGraphNode_t, uint8_t>> dp;
+    for (int d : edges[i]) {
+      const bool prod = pdl_all || std::find(S.sub_deps[i].begin(), S.sub_deps[i].end(), d) != S.sub_deps[i].end();
+      for (cudaGraphNode_t n : nodes_of[d]) dp.push_back({n, (uint8_t)(pdl && prod)});
+    }
+    std::sort(dp.begin(), dp.end());
     std::vector<cudaGraphNode_t> deps;
-    for (int d : edges[i]) deps.insert(deps.end(), nodes_of[d].begin(), nodes_of[d].end());
-    std::sort(deps.begin(), deps.end());
-    deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
+    std::vector<uint8_t> prog;
+    for (size_t j = 0; j < dp.size(); ++j) {
+      if (!deps.empty() && deps.back() == dp[j].first) {
+        prog.back() &= dp[j].second;  // a node reached both ways: full completion wins
+        continue;
+      }
+      deps.push_back(dp[j].first);
+      prog.push_back(dp[j].second);
+    }
     for (; li < P->launches.size() && P->launches[li].sub == i; ++li) {
       cudaGraphNode_t nd;
-      ktiler_status st = add_node(P->launches[li], deps, &nd);
+      ktiler_status st = add_node(P->launches[li], deps, prog, &nd);
       if (st) {
         cudaGraphDestroy(gr);
         return st;
@@ -1183,7 +1218,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     std::sort(deps.begin(), deps.end());
     deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
     cudaGraphNode_t nd;
-    ktiler_status st = add_node(D, deps, &nd);
+    ktiler_status st = add_node(D, deps, {}, &nd);
     if (st) {
       cudaGraphDestroy(gr);
       return st;
