@@ -10,5 +10,5 @@ for l in sys.stdin:
     except Exception:
         print("?", l[:100]); continue
     c = d.get("cfg", {})
-    print(f"  {c.get('exec_mode','?'):10s} {c.get('kind','?'):7s} f={c.get('l2_fraction','-')} w={c.get('window','-')} "
+    print(f"  {c.get('exec_mode','?'):10s} {c.get('kind','?'):7s} r={c.get('rows','-')} f={c.get('l2_fraction','-')} w={c.get('window','-')} "
           f"ms={d.get('ms','-')} frags={d.get('fragments','-')} {d.get('error','')[:80]}")
