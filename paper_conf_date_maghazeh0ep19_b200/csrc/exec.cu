@@ -187,7 +187,7 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
 }
 
 template <int OP, bool SCALAR>
-__global__ void __launch_bounds__(256, (OP == 1 || OP == 3 || OP == 6) ? 2 : 4) op_kernel(const __grid_constant__ KParams p) {
+__global__ void __launch_bounds__(256, (OP == 3 || OP == 6) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
@@ -1109,7 +1109,19 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
   // sub-kernels tile by tile (64 x 8K, 0.5 x L2 resident budget: 4.03 ms vs 4.23 ms
   // grid-stride).  Measured on 64 x 8K; KTILER_TILES_PER_CTA overrides.
   const bool concurrent = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE;
-  const int tpc = tpc_env >= 0 ? tpc_env : (L.blocks > 8 * L.resident ? 2 : ((chain || concurrent) ? 1 : 0));
+  int tpc = tpc_env >= 0 ? tpc_env : (L.blocks > 8 * L.resident ? 2 : ((chain || concurrent) ? 1 : 0));
+  if (tpc_env < 0 && tpc == 2 && L.node >= 0 && !L.n->scalar && L.kp.stage_bytes && L.smem == (int)(2 * L.kp.stage_bytes)) {
+    // double buffering halves the CTAs that fit by shared memory; when registers would
+    // allow >= 1.5x as many single-buffer CTAs, the extra warps hide more latency than the
+    // second buffer does (blur5: 0.97 -> 0.87 ms on 64 x 8K)
+    int occ1 = 0, occ2 = 0;
+    const int thr = (int)(L.block.x * L.block.y * L.block.z);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ1, fn, thr, (int)L.kp.stage_bytes);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, fn, thr, L.smem);
+    if (2 * occ1 >= 3 * occ2) tpc = 1;
+  }
+  // a single staging buffer holds one tile: such a launch must not grid-stride
+  if (L.node >= 0 && !L.n->scalar && L.kp.stage_bytes && L.smem < (int)(2 * L.kp.stage_bytes) && tpc != 1) tpc = 1;
   if (L.node >= 0 && !L.n->scalar) {
     if (tpc > 0) grid = (grid + tpc - 1) / tpc;
     else grid = std::min<int64_t>(grid, L.resident);
