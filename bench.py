@@ -61,7 +61,7 @@ def parse(argv=None):
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=0.75)
+    ap.add_argument("--l2-fraction", type=float, default=1.25)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],

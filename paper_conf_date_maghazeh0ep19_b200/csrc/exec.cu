@@ -72,7 +72,7 @@ struct KParams {
   int64_t lid;          // launch index (trace id)
   uint32_t box_bytes;   // bytes one tensor-TMA box delivers
   int32_t use_tmap;
-  int32_t in_stream;    // input is a graph input: load it evict-first
+  int32_t in_stream;    // load the input evict-first (graph input; consumed intermediate of a tiled plan)
   DBuf in, out;
   DBuf aux;             // KTILER_OP_JACOBI: the coefficient buffer (second READ access)
   int32_t tw, th;
@@ -365,7 +365,7 @@ struct PNode {
   CUtensorMap tmap;  // input tile map (tensor TMA), valid if use_tmap
   uint32_t box_bytes;
   int32_t use_tmap;
-  int32_t in_stream;  // input is a graph input: load it evict-first
+  int32_t in_stream;  // load the input evict-first (graph input; consumed intermediate of a tiled plan)
   DBuf in, out;
   int32_t op, scalar, tw, th;
   float T;
@@ -861,7 +861,15 @@ void build_launches(ktiler_plan_s* P) {
         L.kp.in = dbuf(g.bufs[r.buf]);
         L.kp.out = dbuf(g.bufs[w.buf]);
         if (n.racc2 >= 0) L.kp.aux = dbuf(g.bufs[n.acc[n.racc2].buf]);
-        L.kp.in_stream = !g.written_by_node(r.buf);
+        // Staged reads with an L2 evict-first hint: graph inputs always (read once); in a
+        // tiled plan also the intermediates, whose consumer is their last reader — a
+        // consumed line becomes the first eviction candidate, so the dead lines of earlier
+        // fragments stop crowding out the live ones (64 x 8K: 3.43 -> 3.28 ms, DESIGN.md
+        // §6, A42).  Untiled plans keep the default policy (halo rows are re-read by the
+        // next tile row much later).  KTILER_EVICT_READS=0/1 forces it off/on.
+        static const int evict_env = getenv("KTILER_EVICT_READS") ? atoi(getenv("KTILER_EVICT_READS")) : -1;
+        const bool evict_reads = evict_env >= 0 ? evict_env != 0 : P->s.nfrag > 1;
+        L.kp.in_stream = evict_reads || !g.written_by_node(r.buf);
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
         L.kp.T = n.T;
@@ -1411,7 +1419,8 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     q.T = n.T;
     q.use_tmap = !n.scalar && make_tmap(g, n, &q.tmap, &q.box_bytes);
     if (!n.scalar && !q.use_tmap) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: input tile map unavailable");
-    q.in_stream = !g.written_by_node(r.buf);
+    static const int evict_env = getenv("KTILER_EVICT_READS") ? atoi(getenv("KTILER_EVICT_READS")) : -1;
+    q.in_stream = (evict_env >= 0 ? evict_env != 0 : S.nfrag > 1) || !g.written_by_node(r.buf);  // as for launches
   }
   int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
