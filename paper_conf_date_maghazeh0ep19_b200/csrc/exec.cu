@@ -862,13 +862,13 @@ void build_launches(ktiler_plan_s* P) {
         L.kp.out = dbuf(g.bufs[w.buf]);
         if (n.racc2 >= 0) L.kp.aux = dbuf(g.bufs[n.acc[n.racc2].buf]);
         // Staged reads with an L2 evict-first hint: graph inputs always (read once); in a
-        // tiled plan also the intermediates, whose consumer is their last reader — a
-        // consumed line becomes the first eviction candidate, so the dead lines of earlier
-        // fragments stop crowding out the live ones (64 x 8K: 3.43 -> 3.28 ms, DESIGN.md
-        // §6, A42).  Untiled plans keep the default policy (halo rows are re-read by the
-        // next tile row much later).  KTILER_EVICT_READS=0/1 forces it off/on.
+        // tiled plan also the intermediates read by one node only (that node is their last
+        // reader), so a consumed line becomes the first eviction candidate and the dead
+        // lines of earlier fragments stop crowding out the live ones (64 x 8K: 3.43 ->
+        // 3.28 ms, A42).  Untiled plans keep the default policy (halo rows are
+        // re-read by the next tile row much later).  KTILER_EVICT_READS=0/1 forces it.
         static const int evict_env = getenv("KTILER_EVICT_READS") ? atoi(getenv("KTILER_EVICT_READS")) : -1;
-        const bool evict_reads = evict_env >= 0 ? evict_env != 0 : P->s.nfrag > 1;
+        const bool evict_reads = evict_env >= 0 ? evict_env != 0 : (P->s.nfrag > 1 && g.bufs[r.buf].readers.size() == 1);
         L.kp.in_stream = evict_reads || !g.written_by_node(r.buf);
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
@@ -1420,7 +1420,8 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     q.use_tmap = !n.scalar && make_tmap(g, n, &q.tmap, &q.box_bytes);
     if (!n.scalar && !q.use_tmap) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: input tile map unavailable");
     static const int evict_env = getenv("KTILER_EVICT_READS") ? atoi(getenv("KTILER_EVICT_READS")) : -1;
-    q.in_stream = (evict_env >= 0 ? evict_env != 0 : S.nfrag > 1) || !g.written_by_node(r.buf);  // as for launches
+    q.in_stream = (evict_env >= 0 ? evict_env != 0 : (S.nfrag > 1 && g.bufs[r.buf].readers.size() == 1)) ||
+                  !g.written_by_node(r.buf);  // as for launches
   }
   int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
