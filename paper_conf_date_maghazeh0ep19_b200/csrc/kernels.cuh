@@ -4,21 +4,23 @@
 // threads (thread tid); the rect is exactly the block's declared WRITE footprint, so the
 // planner's dependency analysis and the kernels can never disagree.
 //
-// Vector variant (B200 geometry) = two phases, so the persistent executor can overlap
-// the memory of one tile with the arithmetic of another:
-//   stage_tile    the block's input footprint (+ halo, replicate-clamped at image edges)
-//                 into shared memory with cp.async.cg: every 16-B chunk of the tile in
-//                 flight at once, L2-only (so data other CTAs produced in the same
-//                 persistent launch is never read from a stale L1); no wait;
+// Vector variant (B200 geometry) = two phases, so the executors can overlap the memory of
+// one tile with the arithmetic of another:
+//   staging       the block's input footprint (+ halo) lands in shared memory by ONE
+//                 tensor-map TMA (cp.async.bulk.tensor.3d, completion on an mbarrier); a
+//                 replicate fix-up (stage_fix) reproduces the image-edge clamp that TMA's
+//                 zero fill does not;
 //   compute_tile  one work item = 16 output pixels of one row (gray, down2, thresh) or a
-//                 16-pixel column strip of R rows with a sliding row window in registers
-//                 (blur5, sobel3); packed 2x16-bit SIMD arithmetic in 32-bit registers,
-//                 byte permutes (PRMT) to unpack/pack, dp4a for the luma dot product,
-//                 128-bit stores.
+//                 16-pixel column strip of rows_per_item rows with a sliding row window in
+//                 registers (blur5, sobel3); packed 2x16-bit SIMD arithmetic in 32-bit
+//                 registers, byte permutes (PRMT) to unpack/pack, dp2a for the luma dot
+//                 product, 128-bit stores (256-bit for the f32 Sobel rows).
 // Scalar variant: the paper's Fig. 1 geometry, one thread per pixel.
-// Cache policy: the graph input (rgb) is read once -> L2 evict_first; the graph output
-// (mask) is never re-read -> L2 evict_first stores; intermediates keep the default policy
-// so they stay resident for their consumer sub-kernel (the point of KTILER).
+// Cache policy: the graph input (rgb) is read once -> L2 evict_first; in a tiled plan so
+// is every intermediate with a single reader node (its consumer is its last reader,
+// DESIGN.md A42); the graph output (mask) is never re-read -> L2 evict_first stores;
+// intermediate stores keep the default policy so they stay resident for their consumer
+// sub-kernel (the point of KTILER).
 // Border: replicate (clamp-to-edge) at image edges only.
 #pragma once
 
