@@ -414,9 +414,19 @@ def main():
                 dom = max(tiled_sh, key=lambda k: tiled_sh[k] if k in per_node else -1)
                 d = per_node[dom]
                 ach = d["bytes"] / d["launches"] / (d["span_ns"] / d["launches"])  # B/ns = GB/s
+                dtraffic = None
+                try:
+                    dt = json.load(open(os.path.join(ROOT, "profiles", "r01_dominant_traffic.json")))
+                    if dt["kernel"] == dom and all(line["config"].get(k) == v for k, v in dt["config"].items()
+                                                   if k not in ("workload",)) and dt["config"]["workload"] == args.workload:
+                        dtraffic = {"bytes": dt["dram_bytes_per_launch_mean"], "source": dt["source"]}
+                except Exception:
+                    pass
                 line["roofline"]["dominant_kernel"] = {
                     "kernel": dom, "bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                     "launches_per_step": d["launches"], "mean_launch_us": d["span_ns"] / d["launches"] / 1e3,
+                    "traffic": dtraffic["bytes"] if dtraffic else None,
+                    "traffic_source": dtraffic["source"] if dtraffic else None,
                     "algorithmic_bytes": f"{NODE_BYTES[dom]} B per output pixel x output pixels per launch",
                     "timing": "device-side tracer (%globaltimer, first CTA start -> last CTA end per launch); "
                               "launches of the DAG overlap, so this is a per-launch rate, not a share of the step"}

