@@ -26,6 +26,9 @@ Contents (ids O-n):
 * O-13 ``application_tiling``: Alg. 1 with performance tables.
 * O-14 ``hs_jacobi``: K Horn–Schunck Jacobi iterations, the paper's JI nodes
   (SURVEY §8(f) f2), in f32 (the GPU's exact operation order) or f64.
+* O-7  ``gauss_taps`` / ``gauss_f32``: the float variant of the blur (SURVEY §8(c) O-7,
+  reading A43): separable Gaussian with f64-normalised taps rounded to f32, evaluated in
+  f64 with replicate border, as the plain definition.
 """
 from __future__ import annotations
 
@@ -764,3 +767,35 @@ def hs_jacobi(coef: np.ndarray, s0: np.ndarray, a2: float, iters: int, dtype=np.
         t = ((Ix * ub + Iy * vb) + It) / den
         s = np.stack([ub - Ix * t, vb - Iy * t], axis=-1)
     return s
+
+
+def gauss_taps(sigma: float) -> np.ndarray:
+    """O-7 weights (reading A43): radius r = ceil(3 sigma); w_k = exp(-k^2 / (2 sigma^2))
+    for k = -r..r, normalised to sum 1 in f64, then rounded to f32 (the values both sides
+    use).  Returned as float32 [2r+1]."""
+    r = int(np.ceil(3.0 * np.float64(np.float32(sigma))))
+    s = np.float64(np.float32(sigma))
+    k = np.arange(-r, r + 1, dtype=np.float64)
+    w = np.exp(-k * k / (2.0 * s * s))
+    return (w / w.sum()).astype(np.float32)
+
+
+def gauss_f32(x: np.ndarray, sigma: float, passes: int = 1) -> np.ndarray:
+    """O-7: ``passes`` applications of the separable Gaussian to f32 images x [F, H, W],
+    out[y][x] = sum_i w_i sum_j w_j in[clamp(y+i)][clamp(x+j)] (replicate border), written
+    out in f64 (the definition; the GPU computes it in f32 FMA chains, tolerance 1e-5 on
+    data in [0, 1], BJ:5).  Returns float64 [F, H, W]."""
+    w = gauss_taps(sigma).astype(np.float64)
+    r = (len(w) - 1) // 2
+    a = x.astype(np.float64)
+    for _ in range(passes):
+        F, H, W = a.shape
+        p = np.pad(a, ((0, 0), (0, 0), (r, r)), mode="edge")
+        h = np.zeros_like(a)
+        for j in range(2 * r + 1):
+            h += w[j] * p[:, :, j:j + W]
+        p = np.pad(h, ((0, 0), (r, r), (0, 0)), mode="edge")
+        a = np.zeros_like(h)
+        for i in range(2 * r + 1):
+            a += w[i] * p[:, i:i + H, :]
+    return a

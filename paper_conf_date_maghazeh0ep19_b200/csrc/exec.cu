@@ -77,6 +77,8 @@ struct KParams {
   DBuf aux;             // KTILER_OP_JACOBI: the coefficient buffer (second READ access)
   int32_t tw, th;
   float T;
+  float taps[2 * ktd::GAUSS_H + 1];  // KTILER_OP_GAUSS_F32: f32 weights, taps[k + radius]
+  int32_t radius;
   int32_t nrect, ndisc, pdl;
   int64_t stage_bytes;  // one of the two staging buffers
   LRect r[MAXR];
@@ -187,7 +189,7 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
 }
 
 template <int OP, bool SCALAR>
-__global__ void __launch_bounds__(256, (OP == 3 || OP == 6) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
+__global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
@@ -263,11 +265,11 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6) ? 2 : (OP == 1 ? 3 :
       ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
       ph ^= 1u << b;
       const ktd::Tile t = s_tile[b];
-      if ((OP == 1 || OP == 3 || OP == 6) && ktd::needs_fix(OP, p.in, t)) {
+      if ((OP == 1 || OP == 3 || OP == 6 || OP == 7) && ktd::needs_fix(OP, p.in, t)) {
         ktd::stage_fix(OP, p.in, t, buf, nt, tid);
         __syncthreads();
       }
-      ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid, &p.aux);
+      ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid, &p.aux, p.taps, p.radius);
       const int64_t nx = i + 2 * (int64_t)gridDim.x;
       if (p.chain) {
         __syncthreads();  // tile written (and buffer b consumed)
@@ -722,6 +724,7 @@ kfn_t vec_kernel(int op) {
     case 2: return op_kernel<2, false>;
     case 3: return op_kernel<3, false>;
     case 6: return op_kernel<6, false>;
+    case 7: return op_kernel<7, false>;
     default: return op_kernel<4, false>;
   }
 }
@@ -873,6 +876,8 @@ void build_launches(ktiler_plan_s* P) {
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
         L.kp.T = n.T;
+        L.kp.radius = n.radius;
+        for (int k = 0; k <= 2 * n.radius && k < 2 * ktd::GAUSS_H + 1; ++k) L.kp.taps[k] = n.taps[k];
         L.kp.pdl = pdl;
         size_t m = std::min<size_t>(MAXR, sk.rects.size() - c);
         L.kp.nrect = (int32_t)m;
@@ -1065,9 +1070,11 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
     case KTILER_OP_DOWN2: bw = 32 * nseg; bh = 2 * th; break;
     case KTILER_OP_SOBEL3: bw = 16 * (nseg + 2); bh = th + 2; break;
     case KTILER_OP_JACOBI: bw = 4 * (tw + 8); bh = th + 2; break;
+    case KTILER_OP_GAUSS_F32: bw = 4 * (tw + 2 * ktd::GAUSS_H); bh = th + 2 * ktd::GAUSS_H; break;
     default: bw = 64 * nseg; bh = th; break;
   }
-  if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != ktd::stage_bytes(n.op, tw, th)) return false;
+  const int window = n.op == KTILER_OP_GAUSS_F32 ? bw * bh : ktd::stage_bytes(n.op, tw, th);  // gauss: + its pass buffer
+  if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != window) return false;
   if (B.d.pitch_bytes % 16 || B.d.frame_stride_bytes % 16) return false;
   const int64_t rowbytes = B.d.width * B.d.elem_bytes;
   cuuint64_t dims[3] = {(cuuint64_t)((rowbytes + 3) / 4), (cuuint64_t)B.d.height, (cuuint64_t)B.d.frames};
@@ -1398,7 +1405,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   const int nn = (int)g.nodes.size();
   const int nsub = (int)S.subs.size();
   for (auto& n : g.nodes)
-    if (n.op == KTILER_OP_CUSTOM || n.op == KTILER_OP_JACOBI)
+    if (n.op == KTILER_OP_CUSTOM || n.op == KTILER_OP_JACOBI || n.op == KTILER_OP_GAUSS_F32)
       return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode runs the image-pipeline built-ins (GRAY..THRESH) only");
   if (nn > PMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: at most 8 nodes");
   std::vector<PNode> pn(nn);

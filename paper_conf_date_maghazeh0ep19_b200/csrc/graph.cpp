@@ -8,6 +8,7 @@
 //     is an index interval per axis (Graph::producers / Graph::consumers);
 //   - memory lines: the 128-B lines of each access's clipped rect.
 #include <algorithm>
+#include <cmath>
 #include <cstring>
 #include <mutex>
 
@@ -77,7 +78,7 @@ BRange Graph::consumers(const Chan& c, int64_t px, int64_t py) const {
 // True stencil of each built-in, for the declared output tile (tw, th) of the WRITE
 // access: read map (ax, ay, ox, oy, halos).  A declared read footprint must match it
 // exactly, so a mis-declared footprint can never yield an invalid schedule.
-static bool builtin_read_map(int op, const Access& w, Access& r) {
+static bool builtin_read_map(int op, const Access& w, Access& r, int radius = 0) {
   r.mode = KTILER_READ;
   r.ox = w.ox;
   r.oy = w.oy;
@@ -93,14 +94,17 @@ static bool builtin_read_map(int op, const Access& w, Access& r) {
       r.ax = 2 * w.ax; r.ay = 2 * w.ay; r.ox = 2 * w.ox; r.oy = 2 * w.oy;
       return true;
     case KTILER_OP_JACOBI: r.hl = r.hr = 2; r.ht = r.hb = 1; return true;  // (u, v) of the 4 neighbours
+    case KTILER_OP_GAUSS_F32: r.hl = r.hr = r.ht = r.hb = radius; return true;
     default: return false;
   }
 }
 
 static int builtin_in_elem(int op) {
-  return op == KTILER_OP_GRAY ? 3 : ((op == KTILER_OP_THRESH || op == KTILER_OP_JACOBI) ? 4 : 1);
+  return op == KTILER_OP_GRAY ? 3 : ((op == KTILER_OP_THRESH || op == KTILER_OP_JACOBI || op == KTILER_OP_GAUSS_F32) ? 4 : 1);
 }
-static int builtin_out_elem(int op) { return (op == KTILER_OP_SOBEL3 || op == KTILER_OP_JACOBI) ? 4 : 1; }
+static int builtin_out_elem(int op) {
+  return (op == KTILER_OP_SOBEL3 || op == KTILER_OP_JACOBI || op == KTILER_OP_GAUSS_F32) ? 4 : 1;
+}
 
 ktiler_status Graph::finalize() {
   if (finalized) return KTILER_OK;
@@ -252,7 +256,7 @@ ktiler_status ktiler_add_buffer(ktiler_graph_t g, const ktiler_buffer_desc* d, i
 ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, int32_t* node_id) {
   if (!g || !d || !node_id) return fail(KTILER_E_INVALID, "NULL argument");
   if (g->g.finalized) return fail(KTILER_E_STATE, "graph already planned; create a new graph");
-  if (d->op < KTILER_OP_GRAY || d->op > KTILER_OP_JACOBI) return fail(KTILER_E_INVALID, "unknown op");
+  if (d->op < KTILER_OP_GRAY || d->op > KTILER_OP_GAUSS_F32) return fail(KTILER_E_INVALID, "unknown op");
   if (d->n_access <= 0 || !d->access) return fail(KTILER_E_INVALID, "a kernel needs at least one access");
   Node n;
   n.op = d->op;
@@ -305,8 +309,20 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
     if (n.racc < 0) return fail(KTILER_E_INVALID, "built-in kernels have exactly one READ access");
     if (w.hl || w.hr || w.ht || w.hb || w.ox || w.oy)
       return fail(KTILER_E_INVALID, "built-in WRITE access must have zero offsets and halos (output tile = ax x ay)");
+    if (d->op == KTILER_OP_GAUSS_F32) {  // sigma -> radius and f32 taps (f64-normalised, reading A43)
+      float sigma = 0.0f;
+      if (n.params.size() != sizeof(float)) return fail(KTILER_E_INVALID, "GAUSS_F32 params must be one float (sigma)");
+      std::memcpy(&sigma, n.params.data(), sizeof(float));
+      if (!(sigma > 0.0f) || std::ceil(3.0 * (double)sigma) > 4.0)
+        return fail(KTILER_E_INVALID, "GAUSS_F32 sigma must be > 0 with ceil(3 sigma) <= 4");
+      n.radius = (int)std::ceil(3.0 * (double)sigma);
+      double wk[9], sum = 0.0;
+      for (int k = -n.radius; k <= n.radius; ++k) sum += (wk[k + n.radius] = std::exp(-(double)k * k / (2.0 * sigma * sigma)));
+      for (int k = 0; k <= 2 * n.radius; ++k) n.taps[k] = (float)(wk[k] / sum);
+      n.T = sigma;
+    }
     Access want;
-    builtin_read_map(d->op, w, want);
+    builtin_read_map(d->op, w, want, n.radius);
     const Access& r = n.acc[n.racc];
     // the declared footprint must cover the true stencil (same scale and offset, halos at
     // least the stencil's): a larger one only adds dependencies (e.g. the line-quantized
@@ -342,7 +358,8 @@ ktiler_status ktiler_add_kernel(ktiler_graph_t g, const ktiler_kernel_desc* d, i
     }
     int64_t nt = n.nthreads();
     if (nt > 1024) return fail(KTILER_E_INVALID, "more than 1024 threads per block");
-    n.scalar = (nt == w.ax * w.ay) && d->op != KTILER_OP_JACOBI;
+    n.scalar = (nt == w.ax * w.ay) && d->op != KTILER_OP_JACOBI && d->op != KTILER_OP_GAUSS_F32;
+    if (d->op == KTILER_OP_GAUSS_F32 && w.ax > 248) return fail(KTILER_E_INVALID, "GAUSS_F32 tile width must be <= 248");
     if (!n.scalar) {
       if (w.ax % 16) return fail(KTILER_E_INVALID, "vector variant needs tile width % 16 == 0 (else use one thread per pixel)");
       if (nt % 32) return fail(KTILER_E_INVALID, "vector variant needs a multiple of 32 threads per block");

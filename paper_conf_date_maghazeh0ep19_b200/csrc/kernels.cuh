@@ -158,6 +158,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* m, unsigned parity) {
 // Staged window of op's input for tile t: rows [ry0, ry0+nr) (clamped to the image for the
 // stencils), byte columns [xb0, xb0 + stride) (negative / beyond-width columns of the
 // stencils are filled by stage_fix with the replicate rule).
+constexpr int GAUSS_H = 4;  // staged halo of KTILER_OP_GAUSS_F32 (radius <= 4; 16-B aligned boxes)
 struct StageGeo {
   int64_t ry0, xb0, limit;  // limit = roundup16(row bytes) <= pitch
   int nr, stride;
@@ -172,6 +173,7 @@ __device__ __forceinline__ StageGeo stage_geo(int op, const DBuf& in, const Tile
     case 2: return {2 * t.y0, 2 * t.x0, up16(in.W), 2 * rows, 32 * nseg, false};
     case 3: return {t.y0 - 1, t.x0 - 16, up16(in.W), rows + 2, 16 * (nseg + 2), true};
     case 6: return {t.y0 - 1, 4 * (t.x0 - 4), up16(4 * in.W), rows + 2, 4 * (t.fw + 8), true};  // f32, 2 px halo (16-B aligned)
+    case 7: return {t.y0 - GAUSS_H, 4 * (t.x0 - GAUSS_H), up16(4 * in.W), rows + 2 * GAUSS_H, 4 * (t.fw + 2 * GAUSS_H), true};
     default: return {t.y0, 4 * t.x0, up16(4 * in.W), rows, 64 * nseg, false};
   }
 }
@@ -186,6 +188,8 @@ __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
     case 3: return (th + 2) * 16 * (nseg + 2);   // down rows y-1..y+1
     case 4: return th * 64 * nseg;               // f32 rows
     case 6: return (th + 2) * 4 * (tw + 8);      // (u, v) rows y-1..y+th, two pixels of halo per side
+    case 7: return (th + 2 * GAUSS_H) * 4 * (tw + 2 * GAUSS_H)  // f32 window, GAUSS_H px of halo
+                   + (th + 2 * GAUSS_H) * 4 * tw;              // + the horizontal pass
   }
   return 0;
 }
@@ -238,10 +242,10 @@ __device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map,
 // the caller synchronizes afterwards.  Returns quickly for interior tiles.
 __device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t, uint8_t* sm, int nt, int tid,
                                           int bar_id = 4) {
-  if (op != 1 && op != 3 && op != 6) return;
+  if (op != 1 && op != 3 && op != 6 && op != 7) return;
   const StageGeo g = stage_geo(op, in, t);
-  const int pe = op == 6 ? 8 : 1;                                                          // bytes per pixel
-  const int ew = op == 6 ? 4 : 1;                                                          // bytes per element
+  const int pe = op == 6 ? 8 : (op == 7 ? 4 : 1);                                          // bytes per pixel
+  const int ew = op >= 6 ? 4 : 1;                                                          // bytes per element
   const int left = g.xb0 < 0 ? (int)(-g.xb0) : 0;                                          // bytes < 0
   const int rfrom = (int)(ew * in.W - g.xb0) < g.stride ? (int)(ew * in.W - g.xb0) : g.stride;  // bytes >= row end
   const int right = g.stride - rfrom;
@@ -270,9 +274,9 @@ __device__ __forceinline__ void stage_fix(int op, const DBuf& in, const Tile& t,
 
 // Does tile t of a stencil op need stage_fix?  (CTA-uniform)
 __device__ __forceinline__ bool needs_fix(int op, const DBuf& in, const Tile& t) {
-  if (op != 1 && op != 3 && op != 6) return false;
+  if (op != 1 && op != 3 && op != 6 && op != 7) return false;
   const StageGeo g = stage_geo(op, in, t);
-  const int64_t rowb = op == 6 ? 4 * in.W : in.W;
+  const int64_t rowb = op >= 6 ? 4 * in.W : in.W;
   return g.xb0 < 0 || g.xb0 + g.stride > rowb || g.ry0 < 0 || g.ry0 + g.nr > in.H;
 }
 
@@ -690,9 +694,97 @@ __device__ void jacobi_compute(const DBuf& out, const DBuf& coef, const Tile& t,
   }
 }
 
+// ---------------------------------------------------------------------------------
+// gauss_f32: separable Gaussian on f32 (KTILER_OP_GAUSS_F32, the float variant SURVEY
+// §8(c) O-7 describes).  taps[0..2r] are the host's f64-normalised weights rounded to f32
+// (r = ceil(3 sigma) <= GAUSS_H).  Horizontal pass over the staged window (rows y0-H ..
+// y1+H) into a second shared buffer, a CTA barrier, then the vertical pass; each output is
+// an f32 FMA chain in tap order k = -r..r.  Replicate border via stage_fix.
+// ---------------------------------------------------------------------------------
+// An item = 4 consecutive pixels of one row: float4 shared-memory loads and stores (the
+// window rows start 16-B aligned: GAUSS_H = 4 floats of halo), each output one FMA chain in
+// tap order.  Columns past a ragged tile's last multiple of 4 take the per-pixel path.
+template <int R>
+__device__ __forceinline__ void gauss_compute_r(const DBuf& out, const Tile& t, const uint8_t* sm, const float* taps,
+                                                int nt, int tid) {
+  static_assert(R >= 1 && R <= GAUSS_H, "radius");
+  const int tw = t.fw, rows = t.rows(), nr = rows + 2 * GAUSS_H;
+  const int w = (int)(t.x1 - t.x0), nq = (w + 3) >> 2;
+  const float* S = reinterpret_cast<const float*>(sm);           // [nr][tw + 2H]
+  float* Hs = const_cast<float*>(S) + nr * (tw + 2 * GAUSS_H);   // [nr][tw]
+  const int sw = tw + 2 * GAUSS_H;
+  float wk[2 * R + 1];
+#pragma unroll
+  for (int k = 0; k <= 2 * R; ++k) wk[k] = taps[k];
+  for (int i = tid; i < nr * nq; i += nt) {
+    const int row = i / nq, x = 4 * (i - row * nq);
+    const float* src = S + row * sw + GAUSS_H + x;  // 16-B aligned
+    if (x + 4 <= w) {
+      float v[12];  // window columns x-4 .. x+7
+#pragma unroll
+      for (int q = 0; q < 3; ++q) {
+        const float4 f = *reinterpret_cast<const float4*>(src - 4 + 4 * q);
+        v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
+      }
+      float o[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float a = 0.0f;
+#pragma unroll
+        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], v[4 + j + k], a);
+        o[j] = a;
+      }
+      *reinterpret_cast<float4*>(Hs + row * tw + x) = make_float4(o[0], o[1], o[2], o[3]);
+    } else {
+      for (int j = 0; x + j < w; ++j) {
+        float a = 0.0f;
+#pragma unroll
+        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], src[j + k], a);
+        Hs[row * tw + x + j] = a;
+      }
+    }
+  }
+  asm volatile("bar.sync 5, %0;" ::"r"(nt) : "memory");
+  float* const ob = reinterpret_cast<float*>(tile_out(out, t, 4));
+  const int pitch = (int)(out.pitch >> 2);
+  for (int i = tid; i < rows * nq; i += nt) {
+    const int y = i / nq, x = 4 * (i - y * nq);
+    const float* src = Hs + (y + GAUSS_H) * tw + x;
+    if (x + 4 <= w) {
+      float4 a = make_float4(0.0f, 0.0f, 0.0f, 0.0f);
+#pragma unroll
+      for (int k = -R; k <= R; ++k) {
+        const float4 h = *reinterpret_cast<const float4*>(src + k * tw);
+        a.x = __fmaf_rn(wk[k + R], h.x, a.x);
+        a.y = __fmaf_rn(wk[k + R], h.y, a.y);
+        a.z = __fmaf_rn(wk[k + R], h.z, a.z);
+        a.w = __fmaf_rn(wk[k + R], h.w, a.w);
+      }
+      *reinterpret_cast<float4*>(ob + y * pitch + x) = a;
+    } else {
+      for (int j = 0; x + j < w; ++j) {
+        float a = 0.0f;
+#pragma unroll
+        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], src[j + k * tw], a);
+        ob[y * pitch + x + j] = a;
+      }
+    }
+  }
+}
+__device__ void gauss_compute(const DBuf& out, const Tile& t, const uint8_t* sm, const float* taps, int r, int nt,
+                              int tid) {
+  switch (r) {
+    case 1: gauss_compute_r<1>(out, t, sm, taps, nt, tid); break;
+    case 2: gauss_compute_r<2>(out, t, sm, taps, nt, tid); break;
+    case 3: gauss_compute_r<3>(out, t, sm, taps, nt, tid); break;
+    default: gauss_compute_r<4>(out, t, sm, taps, nt, tid); break;
+  }
+}
+
 // Compute op's output tile from its staged input (after the staging is complete).
 __device__ __forceinline__ void compute_tile(int op, const DBuf& out, const Tile& t, const uint8_t* sm, float T,
-                                             int nt, int tid, const DBuf* aux = nullptr) {
+                                             int nt, int tid, const DBuf* aux = nullptr, const float* taps = nullptr,
+                                             int radius = 0) {
   switch (op) {
     case 0: gray_compute(out, t, sm, nt, tid); break;
     case 1: blur_compute(out, t, sm, nt, tid); break;
@@ -700,6 +792,7 @@ __device__ __forceinline__ void compute_tile(int op, const DBuf& out, const Tile
     case 3: sobel_compute(out, t, sm, nt, tid); break;
     case 4: thresh_compute(out, t, sm, T, nt, tid); break;
     case 6: jacobi_compute(out, *aux, t, sm, T, nt, tid); break;  // T = a2 (alpha^2)
+    case 7: gauss_compute(out, t, sm, taps, radius, nt, tid); break;
   }
 }
 

@@ -45,6 +45,8 @@ struct Node {
   int wacc = -1;     // index of the (single) WRITE access for built-ins
   int racc = -1;     // index of the (first) READ access for built-ins
   int racc2 = -1;    // KTILER_OP_JACOBI: its second READ access (the coefficients)
+  int radius = 0;    // KTILER_OP_GAUSS_F32: ceil(3 sigma)
+  float taps[9] = {};  // KTILER_OP_GAUSS_F32: f64-normalised Gaussian weights rounded to f32
   int64_t nblocks = 0;
   int64_t gid0 = 0;  // first global block id
   float T = 200.f;

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(_PKG, "libktiler.so")
 OK, E_INVALID, E_CYCLE, E_UNTILEABLE, E_NOMEM, E_CUDA, E_STATE, E_UNSUPPORTED = range(8)
 BUF_INTERNAL = 1
 READ, WRITE = 1, 2
-OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM, OP_JACOBI = range(7)
+OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM, OP_JACOBI, OP_GAUSS_F32 = range(8)
 FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1, FRAG_CHAIN = range(6)
 EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE = range(7)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL, PF_RESIDENT_BUDGET = 1, 2, 4, 8

@@ -226,3 +226,24 @@ def test_smoke_configuration_is_tileable(K):
     p = Pipeline(520, 198, 2, T=60.0, internal=True, device=None)
     assert p.b.g.plan(800 * 1024, kind="budget", exec_mode="graph", discard=True, pdl=True).num_fragments() > 1
     assert p.b.g.plan(1 << 20, kind="rows", rows=1, exec_mode="persistent", discard=True).num_fragments() > 1
+
+
+def test_gauss_f32_params(K):
+    """KTILER_OP_GAUSS_F32: sigma must be positive with ceil(3 sigma) <= 4, and the declared
+    read halo must cover the radius."""
+    import struct
+    g = K.Graph()
+    a = g.add_buffer(0x100000, 64, 32, 4)
+    b = g.add_buffer(0x200000, 64, 32, 4)
+
+    def acc(buf, mode, ax, ay, h=0):
+        return dict(buf=buf, mode=mode, ax=ax, ay=ay, hl=h, hr=h, ht=h, hb=h)
+    for sigma in (0.0, -1.0, 1.4):
+        with pytest.raises(K.KtilerError):
+            g.add_kernel(K.OP_GAUSS_F32, (1, 2, 1), (64, 1, 1), [acc(a, K.READ, 64, 16, 4), acc(b, K.WRITE, 64, 16)],
+                         struct.pack("f", sigma))
+    with pytest.raises(K.KtilerError):  # radius 3 > declared halo 2
+        g.add_kernel(K.OP_GAUSS_F32, (1, 2, 1), (64, 1, 1), [acc(a, K.READ, 64, 16, 2), acc(b, K.WRITE, 64, 16)],
+                     struct.pack("f", 1.0))
+    g.add_kernel(K.OP_GAUSS_F32, (1, 2, 1), (64, 1, 1), [acc(a, K.READ, 64, 16, 3), acc(b, K.WRITE, 64, 16)],
+                 struct.pack("f", 1.0))
