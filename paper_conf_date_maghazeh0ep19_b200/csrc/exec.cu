@@ -1073,7 +1073,7 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
     case KTILER_OP_GAUSS_F32: bw = 4 * (tw + 2 * ktd::GAUSS_H); bh = th + 2 * ktd::GAUSS_H; break;
     default: bw = 64 * nseg; bh = th; break;
   }
-  const int window = n.op == KTILER_OP_GAUSS_F32 ? bw * bh : ktd::stage_bytes(n.op, tw, th);  // gauss: + its pass buffer
+  const int window = ktd::stage_bytes(n.op, tw, th);
   if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != window) return false;
   if (B.d.pitch_bytes % 16 || B.d.frame_stride_bytes % 16) return false;
   const int64_t rowbytes = B.d.width * B.d.elem_bytes;

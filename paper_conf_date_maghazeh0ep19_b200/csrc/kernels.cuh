@@ -188,8 +188,7 @@ __host__ __device__ inline int stage_bytes(int op, int tw, int th) {
     case 3: return (th + 2) * 16 * (nseg + 2);   // down rows y-1..y+1
     case 4: return th * 64 * nseg;               // f32 rows
     case 6: return (th + 2) * 4 * (tw + 8);      // (u, v) rows y-1..y+th, two pixels of halo per side
-    case 7: return (th + 2 * GAUSS_H) * 4 * (tw + 2 * GAUSS_H)  // f32 window, GAUSS_H px of halo
-                   + (th + 2 * GAUSS_H) * 4 * tw;              // + the horizontal pass
+    case 7: return (th + 2 * GAUSS_H) * 4 * (tw + 2 * GAUSS_H);  // f32 window, GAUSS_H px of halo
   }
   return 0;
 }
@@ -701,72 +700,83 @@ __device__ void jacobi_compute(const DBuf& out, const DBuf& coef, const Tile& t,
 // y1+H) into a second shared buffer, a CTA barrier, then the vertical pass; each output is
 // an f32 FMA chain in tap order k = -r..r.  Replicate border via stage_fix.
 // ---------------------------------------------------------------------------------
-// An item = 4 consecutive pixels of one row: float4 shared-memory loads and stores (the
-// window rows start 16-B aligned: GAUSS_H = 4 floats of halo), each output one FMA chain in
-// tap order.  Columns past a ragged tile's last multiple of 4 take the per-pixel path.
+// One item = a column strip 4 pixels wide and rows_per_item rows tall.  Each staged row is
+// read once (three float4 loads: columns x-4 .. x+7), its horizontal pass kept in a
+// (2R+1)-row register window that the unroll-by-(2R+1) row loop rotates with static
+// indices, and every output row is one vertical FMA chain over the window — no second
+// shared buffer, no CTA barrier.  Tiles cut by the image's right edge (a last strip
+// narrower than 4) take the per-pixel path.
+template <int R>
+__device__ __forceinline__ float4 gauss_hrow(const float* src, const float* wk) {  // src: staged column x (16-B aligned)
+  float v[12];  // columns x-4 .. x+7
+#pragma unroll
+  for (int q = 0; q < 3; ++q) {
+    const float4 f = *reinterpret_cast<const float4*>(src - 4 + 4 * q);
+    v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
+  }
+  float o[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    float a = 0.0f;
+#pragma unroll
+    for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], v[4 + j + k], a);
+    o[j] = a;
+  }
+  return make_float4(o[0], o[1], o[2], o[3]);
+}
 template <int R>
 __device__ __forceinline__ void gauss_compute_r(const DBuf& out, const Tile& t, const uint8_t* sm, const float* taps,
                                                 int nt, int tid) {
   static_assert(R >= 1 && R <= GAUSS_H, "radius");
-  const int tw = t.fw, rows = t.rows(), nr = rows + 2 * GAUSS_H;
-  const int w = (int)(t.x1 - t.x0), nq = (w + 3) >> 2;
-  const float* S = reinterpret_cast<const float*>(sm);           // [nr][tw + 2H]
-  float* Hs = const_cast<float*>(S) + nr * (tw + 2 * GAUSS_H);   // [nr][tw]
-  const int sw = tw + 2 * GAUSS_H;
-  float wk[2 * R + 1];
+  constexpr int NW = 2 * R + 1;
+  const int tw = t.fw, rows = t.rows(), w = (int)(t.x1 - t.x0);
+  const int nq = (w + 3) >> 2, sw = tw + 2 * GAUSS_H;
+  const float* S = reinterpret_cast<const float*>(sm);  // [rows + 2H][tw + 2H], row r = image row y0 - H + r
+  float wk[NW];
 #pragma unroll
-  for (int k = 0; k <= 2 * R; ++k) wk[k] = taps[k];
-  for (int i = tid; i < nr * nq; i += nt) {
-    const int row = i / nq, x = 4 * (i - row * nq);
-    const float* src = S + row * sw + GAUSS_H + x;  // 16-B aligned
-    if (x + 4 <= w) {
-      float v[12];  // window columns x-4 .. x+7
-#pragma unroll
-      for (int q = 0; q < 3; ++q) {
-        const float4 f = *reinterpret_cast<const float4*>(src - 4 + 4 * q);
-        v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
-      }
-      float o[4];
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        float a = 0.0f;
-#pragma unroll
-        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], v[4 + j + k], a);
-        o[j] = a;
-      }
-      *reinterpret_cast<float4*>(Hs + row * tw + x) = make_float4(o[0], o[1], o[2], o[3]);
-    } else {
-      for (int j = 0; x + j < w; ++j) {
-        float a = 0.0f;
-#pragma unroll
-        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], src[j + k], a);
-        Hs[row * tw + x + j] = a;
-      }
-    }
-  }
-  asm volatile("bar.sync 5, %0;" ::"r"(nt) : "memory");
+  for (int k = 0; k < NW; ++k) wk[k] = taps[k];
   float* const ob = reinterpret_cast<float*>(tile_out(out, t, 4));
   const int pitch = (int)(out.pitch >> 2);
-  for (int i = tid; i < rows * nq; i += nt) {
-    const int y = i / nq, x = 4 * (i - y * nq);
-    const float* src = Hs + (y + GAUSS_H) * tw + x;
-    if (x + 4 <= w) {
-      float4 a = make_float4(0.0f, 0.0f, 0.0f, 0.0f);
+  const int ngrp0 = max(1, nt / max(nq, 1));
+  const int rpi = (rows + ngrp0 - 1) / ngrp0, ngrp = (rows + rpi - 1) / rpi;
+  for (int it = tid; it < nq * ngrp; it += nt) {
+    const int g = it / nq, x = 4 * (it - g * nq);
+    const int ra = g * rpi, n = min(rpi, rows - ra);
+    // output row ra + r needs staged rows ra + r + H - R .. ra + r + H + R
+    const float* col = S + (ra + GAUSS_H - R) * sw + GAUSS_H + x;
+    float* d = ob + ra * pitch + x;
+    if (x + 4 > w) {  // ragged strip: per pixel
+      for (int r = 0; r < n; ++r)
+        for (int j = 0; x + j < w; ++j) {
+          float a = 0.0f;
+          for (int i = -R; i <= R; ++i) {
+            float h = 0.0f;
+            for (int k = -R; k <= R; ++k) h = __fmaf_rn(wk[k + R], col[(r + R + i) * sw + j + k], h);
+            a = __fmaf_rn(wk[i + R], h, a);
+          }
+          d[r * pitch + j] = a;
+        }
+      continue;
+    }
+    float4 h[NW];
 #pragma unroll
-      for (int k = -R; k <= R; ++k) {
-        const float4 h = *reinterpret_cast<const float4*>(src + k * tw);
-        a.x = __fmaf_rn(wk[k + R], h.x, a.x);
-        a.y = __fmaf_rn(wk[k + R], h.y, a.y);
-        a.z = __fmaf_rn(wk[k + R], h.z, a.z);
-        a.w = __fmaf_rn(wk[k + R], h.w, a.w);
-      }
-      *reinterpret_cast<float4*>(ob + y * pitch + x) = a;
-    } else {
-      for (int j = 0; x + j < w; ++j) {
-        float a = 0.0f;
+    for (int i = 0; i < NW - 1; ++i) h[i] = gauss_hrow<R>(col + i * sw, wk);
+    for (int r0 = 0; r0 < n; r0 += NW) {
 #pragma unroll
-        for (int k = -R; k <= R; ++k) a = __fmaf_rn(wk[k + R], src[j + k * tw], a);
-        ob[y * pitch + x + j] = a;
+      for (int k = 0; k < NW; ++k) {
+        const int r = r0 + k;
+        if (r >= n) break;
+        h[(k + NW - 1) % NW] = gauss_hrow<R>(col + (r + NW - 1) * sw, wk);
+        float4 a = make_float4(0.0f, 0.0f, 0.0f, 0.0f);
+#pragma unroll
+        for (int i = 0; i < NW; ++i) {
+          const float4 v = h[(k + i) % NW];
+          a.x = __fmaf_rn(wk[i], v.x, a.x);
+          a.y = __fmaf_rn(wk[i], v.y, a.y);
+          a.z = __fmaf_rn(wk[i], v.z, a.z);
+          a.w = __fmaf_rn(wk[i], v.w, a.w);
+        }
+        *reinterpret_cast<float4*>(d + r * pitch) = a;
       }
     }
   }

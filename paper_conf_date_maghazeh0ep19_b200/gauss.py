@@ -17,7 +17,7 @@ from .pipeline import _GraphBuilder
 
 
 class GaussChain:
-    def __init__(self, W: int, H: int, nodes: int = 2, frames: int = 1, sigma: float = 1.0, tile=(64, 16),
+    def __init__(self, W: int, H: int, nodes: int = 2, frames: int = 1, sigma: float = 1.0, tile=(128, 64),
                  threads: int = 128, device="cuda", internal: bool = True):
         self.W, self.H, self.K, self.F, self.sigma = W, H, nodes, frames, sigma
         self.radius = math.ceil(3 * sigma)

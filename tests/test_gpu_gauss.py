@@ -21,7 +21,7 @@ def _lib():
 
 def _run(W, H, F, nodes, sigma, seed, cache_bytes=1 << 20, **pol):
     from paper_conf_date_maghazeh0ep19_b200.gauss import GaussChain
-    g = GaussChain(W, H, nodes=nodes, frames=F, sigma=sigma)
+    g = GaussChain(W, H, nodes=nodes, frames=F, sigma=sigma, tile=(64, 16))  # small tiles: many fragments
     x = np.random.default_rng(seed).random((F, H, W), dtype=np.float32)
     for k in range(1, nodes + 1):
         g.b.store.tensors[f"x{k}"].fill_(0xFF)  # NaN poison: a skipped block cannot pass

@@ -11,7 +11,7 @@ from oracle import oracle as O
 from paper_conf_date_maghazeh0ep19_b200.gauss import GaussChain
 ge.build()
 for (W, H, K, sig) in [(512, 256, 4, 1.0), (640, 200, 2, 1.3)]:
-    g = GaussChain(W, H, nodes=K, sigma=sig)
+    g = GaussChain(W, H, nodes=K, sigma=sig, tile=(64, 16))
     x = np.random.default_rng(1).random((1, H, W), dtype=np.float32)
     g.view("x0").copy_(torch.from_numpy(x))
     g.plan(256 * 1024, kind="budget", exec_mode="dag")
@@ -19,7 +19,7 @@ for (W, H, K, sig) in [(512, 256, 4, 1.0), (640, 200, 2, 1.3)]:
     err = float(np.abs(g.view(f"x{K}").cpu().numpy().astype(np.float64) - O.gauss_f32(x, sig, passes=K)).max())
     print(json.dumps({"check": f"{W}x{H} K={K} sigma={sig}", "max_abs_err": err}))
 W, H, K = 7680, 4320, 4
-g = GaussChain(W, H, nodes=K, sigma=1.0, tile=(128, 16))
+g = GaussChain(W, H, nodes=K, sigma=1.0)
 g.view("x0").copy_(torch.rand((1, H, W), device="cuda"))
 s = torch.cuda.current_stream()
 for cfg in [dict(kind="none", exec_mode="graph"), dict(kind="budget", l2_fraction=1.0, exec_mode="dag", resident_budget=True),
