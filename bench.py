@@ -63,7 +63,7 @@ def parse(argv=None):
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=1.25)
+    ap.add_argument("--l2-fraction", type=float, default=0.85)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
@@ -72,6 +72,8 @@ def parse(argv=None):
     ap.add_argument("--discard", action="store_true",
                     help="discard dead intermediate lines (DRAM -55%% but slower on B200: DESIGN.md §6)")
     ap.add_argument("--no-discard", action="store_true", help="(default) keep dead lines")
+    ap.add_argument("--no-consumer-discard", action="store_true",
+                    help="keep the lines down2 / thresh consume (default: drop them once staged, DESIGN A44)")
     ap.add_argument("--pdl", action="store_true")
     ap.add_argument("--ctas", type=int, default=0)
     ap.add_argument("--skew", type=int, default=0)
@@ -262,7 +264,7 @@ def policy(args) -> dict:
     """The fragment policy of the timed step (also used by tests/test_gpu_fullsize.py)."""
     return dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode,
                 discard=args.discard and not args.no_discard, pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew,
-                window=args.window, resident_budget=not args.no_resident)
+                window=args.window, resident_budget=not args.no_resident, consumer_discard=not args.no_consumer_discard)
 
 
 def main():
@@ -350,7 +352,8 @@ def main():
     comp_bytes = pix * 3.25  # rgb in + mask out: the method's algorithmic bytes
     achieved = comp_bytes / (ms / 1000) / 1e9
     tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
-            "discard": discard, "window": args.window, "resident_budget": resident}
+            "discard": discard, "window": args.window, "resident_budget": resident,
+            "consumer_discard": pol["consumer_discard"]}
     traffic, traffic_src = traffic_for(tcfg)
     line = {
         "metric": METRIC,
@@ -369,7 +372,8 @@ def main():
                    "frames_per_gpu": per if sp is None else None,
                    "sharding": shard if world > 1 else "none", "pixels_per_gpu": pix_rank, "mode": args.mode,
                    "policy": args.kind, "rows": args.rows, "l2_fraction": args.l2_fraction, "window": args.window,
-                   "resident_budget": resident, "discard": discard, "pdl": args.pdl,
+                   "resident_budget": resident, "discard": discard, "consumer_discard": pol["consumer_discard"],
+                   "pdl": args.pdl,
                    "l2_flush": "not needed: each step reads >= 6.4 GB of input (>> 126 MB L2)" if Ftot > 1 or W >= 16384
                    else "none (input smaller than L2: steady-state replay)",
                    "fragments": st["n_fragments"], "subkernels": st["n_subkernels"],
@@ -417,9 +421,9 @@ def main():
                 dtraffic = None
                 try:
                     dt = json.load(open(os.path.join(ROOT, "profiles", "r01_dominant_traffic.json")))
-                    if dt["kernel"] == dom and all(line["config"].get(k) == v for k, v in dt["config"].items()
-                                                   if k not in ("workload",)) and dt["config"]["workload"] == args.workload:
-                        dtraffic = {"bytes": dt["dram_bytes_per_launch_mean"], "source": dt["source"]}
+                    if dom in dt["kernels"] and all(line["config"].get(k) == v for k, v in dt["config"].items()):
+                        kd = dt["kernels"][dom]
+                        dtraffic = {"bytes": kd["dram_bytes_per_launch_mean"], "source": kd["source"]}
                 except Exception:
                     pass
                 line["roofline"]["dominant_kernel"] = {

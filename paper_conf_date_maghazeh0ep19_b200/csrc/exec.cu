@@ -79,6 +79,7 @@ struct KParams {
   float T;
   float taps[2 * ktd::GAUSS_H + 1];  // KTILER_OP_GAUSS_F32: f32 weights, taps[k + radius]
   int32_t radius;
+  int32_t cdisc;  // KTILER_PF_CONSUMER_DISCARD: drop this block's (exclusively read) input lines once staged
   int32_t nrect, ndisc, pdl;
   int64_t stage_bytes;  // one of the two staging buffers
   LRect r[MAXR];
@@ -188,6 +189,26 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
   }
 }
 
+// KTILER_PF_CONSUMER_DISCARD: the whole 128-B lines of this block's input rect (no halo,
+// the buffer's only reader) leave L2 unwritten once they are staged in shared memory.
+template <int OP>
+__device__ __forceinline__ void consumer_discard(const KParams& p, const ktd::Tile& t, int nt, int tid) {
+  constexpr int EB = OP == 2 ? 2 : 4;  // input bytes per output pixel along x (down2: 2 u8; thresh: 1 f32)
+  const int64_t y0 = OP == 2 ? 2 * t.y0 : t.y0, nrows = OP == 2 ? 2 * (t.y1 - t.y0) : t.y1 - t.y0;
+  const uint8_t* base = p.in.p + t.z * p.in.fstride;
+  const int64_t b0 = EB * t.x0, b1 = EB * t.x1;
+  for (int64_t i = tid;; i += nt) {
+    // lines of row r: [ceil(a / 128), floor(b / 128)) of absolute addresses a, b
+    const int64_t first = ((int64_t)(uintptr_t)(base + y0 * p.in.pitch + b0) + 127) >> 7;
+    const int64_t last = ((int64_t)(uintptr_t)(base + y0 * p.in.pitch + b1)) >> 7;
+    const int64_t per = last > first ? last - first : 0;  // same for every row (128-B pitch)
+    if (per == 0 || i >= per * nrows) break;
+    const int64_t r = i / per, l = i - r * per;
+    const uint8_t* row = base + (y0 + r) * p.in.pitch;
+    ktd::discard_line(reinterpret_cast<const void*>((((int64_t)(uintptr_t)(row + b0) + 127) >> 7 << 7) + 128 * l));
+  }
+}
+
 template <int OP, bool SCALAR>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
@@ -265,6 +286,9 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
       ph ^= 1u << b;
       const ktd::Tile t = s_tile[b];
+      if constexpr (OP == 2 || OP == 4) {
+        if (p.cdisc) consumer_discard<OP>(p, t, nt, tid);
+      }
       if ((OP == 1 || OP == 3 || OP == 6 || OP == 7) && ktd::needs_fix(OP, p.in, t)) {
         ktd::stage_fix(OP, p.in, t, buf, nt, tid);
         __syncthreads();
@@ -873,6 +897,13 @@ void build_launches(ktiler_plan_s* P) {
         static const int evict_env = getenv("KTILER_EVICT_READS") ? atoi(getenv("KTILER_EVICT_READS")) : -1;
         const bool evict_reads = evict_env >= 0 ? evict_env != 0 : (P->s.nfrag > 1 && g.bufs[r.buf].readers.size() == 1);
         L.kp.in_stream = evict_reads || !g.written_by_node(r.buf);
+        // consumer-side discard (PF_CONSUMER_DISCARD, A44): tiled plan, internal input with
+        // this node as its only reader, read without halo, line-aligned rows
+        const kt::Buffer& ib = g.bufs[r.buf];
+        L.kp.cdisc = (P->pol.flags & KTILER_PF_CONSUMER_DISCARD) && P->s.nfrag > 1 && !n.scalar &&
+                     (n.op == KTILER_OP_DOWN2 || n.op == KTILER_OP_THRESH) && (ib.d.flags & KTILER_BUF_INTERNAL) &&
+                     ib.readers.size() == 1 && !r.hl && !r.hr && !r.ht && !r.hb && discardable(ib) &&
+                     g.written_by_node(r.buf);
         L.kp.tw = (int32_t)w.ax;
         L.kp.th = (int32_t)w.ay;
         L.kp.T = n.T;

@@ -95,6 +95,8 @@ MODES = [
     dict(exec_mode="persistent", skew=3, persistent_ctas=7),
     dict(exec_mode="dag"),
     dict(exec_mode="dag", pdl=True),  # programmatic edges from each sub-kernel's producers
+    dict(exec_mode="dag", consumer_discard=True),  # down2 / thresh drop their consumed lines
+    dict(exec_mode="graph", consumer_discard=True),
     dict(exec_mode="dag", window=1),
     dict(exec_mode="dag", window=4),
     dict(exec_mode="chain"),
