@@ -72,6 +72,8 @@ def parse(argv=None):
     ap.add_argument("--discard", action="store_true",
                     help="discard dead intermediate lines (DRAM -55%% but slower on B200: DESIGN.md §6)")
     ap.add_argument("--no-discard", action="store_true", help="(default) keep dead lines")
+    ap.add_argument("--halo-discard", action="store_true",
+                    help="also drop gray / down lines via per-block reader counts (DRAM -62%%, ~15%% slower: A44)")
     ap.add_argument("--no-consumer-discard", action="store_true",
                     help="keep the lines down2 / thresh consume (default: drop them once staged, DESIGN A44)")
     ap.add_argument("--pdl", action="store_true")
@@ -264,7 +266,8 @@ def policy(args) -> dict:
     """The fragment policy of the timed step (also used by tests/test_gpu_fullsize.py)."""
     return dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode,
                 discard=args.discard and not args.no_discard, pdl=args.pdl, persistent_ctas=args.ctas, skew=args.skew,
-                window=args.window, resident_budget=not args.no_resident, consumer_discard=not args.no_consumer_discard)
+                window=args.window, resident_budget=not args.no_resident, consumer_discard=not args.no_consumer_discard,
+                halo_discard=args.halo_discard)
 
 
 def main():
@@ -353,7 +356,7 @@ def main():
     achieved = comp_bytes / (ms / 1000) / 1e9
     tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
             "discard": discard, "window": args.window, "resident_budget": resident,
-            "consumer_discard": pol["consumer_discard"]}
+            "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"]}
     traffic, traffic_src = traffic_for(tcfg)
     line = {
         "metric": METRIC,
@@ -373,6 +376,7 @@ def main():
                    "sharding": shard if world > 1 else "none", "pixels_per_gpu": pix_rank, "mode": args.mode,
                    "policy": args.kind, "rows": args.rows, "l2_fraction": args.l2_fraction, "window": args.window,
                    "resident_budget": resident, "discard": discard, "consumer_discard": pol["consumer_discard"],
+                   "halo_discard": pol["halo_discard"],
                    "pdl": args.pdl,
                    "l2_flush": "not needed: each step reads >= 6.4 GB of input (>> 126 MB L2)" if Ftot > 1 or W >= 16384
                    else "none (input smaller than L2: steady-state replay)",

@@ -80,6 +80,11 @@ struct KParams {
   float taps[2 * ktd::GAUSS_H + 1];  // KTILER_OP_GAUSS_F32: f32 weights, taps[k + radius]
   int32_t radius;
   int32_t cdisc;  // KTILER_PF_CONSUMER_DISCARD: drop this block's (exclusively read) input lines once staged
+  // KTILER_PF_HALO_DISCARD (blur5, sobel3 reads with halo): per producer block a reader
+  // count; the reader that completes it drops the producer block's lines (uses the chain map
+  // fields rax..way / pgx, pgy for the producer range)
+  unsigned int* hcnt;       // [frames][pgy][pgx] readers so far (reset to 0 by the last one)
+  const uint8_t* hneed;     // [pgy][pgx] consumer blocks reading each producer block
   int32_t nrect, ndisc, pdl;
   int64_t stage_bytes;  // one of the two staging buffers
   LRect r[MAXR];
@@ -209,6 +214,44 @@ __device__ __forceinline__ void consumer_discard(const KParams& p, const ktd::Ti
   }
 }
 
+// Halo reads (blur5 of gray, sobel3 of down): a producer block's lines are dead once every
+// consumer block whose declared footprint covers it has staged them.  Warp 0 counts this
+// block in for each producer block in its range (closed form of the affine maps, as
+// chain_wait); the reader that completes a count resets it and drops that block's lines.
+__device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& t, int lane) {
+  const int bx = (int)(t.x0 / p.tw), by = (int)(t.y0 / p.th), bz = (int)t.z;
+  const int rx0 = max(0, p.rax * bx + p.rox - p.rhl), rx1 = min((int)p.in.W, p.rax * (bx + 1) + p.rox + p.rhr);
+  const int ry0 = max(0, p.ray * by + p.roy - p.rht), ry1 = min((int)p.in.H, p.ray * (by + 1) + p.roy + p.rhb);
+  const int px0 = rx0 / p.wax, px1 = min(p.pgx, (rx1 + p.wax - 1) / p.wax);
+  const int py0 = ry0 / p.way, py1 = min(p.pgy, (ry1 + p.way - 1) / p.way);
+  const int pw = px1 - px0, n = pw * (py1 - py0);
+  const uint8_t* fb = p.in.p + (int64_t)bz * p.in.fstride;
+  for (int i0 = 0; i0 < n; i0 += 32) {
+    const int i = i0 + lane;
+    const int py = py0 + i / max(pw, 1), px = px0 + i % max(pw, 1);
+    bool last = false;
+    if (i < n) {
+      const int64_t idx = ((int64_t)bz * p.pgy + py) * p.pgx + px;
+      last = atomicAdd(p.hcnt + idx, 1u) + 1u == (unsigned)p.hneed[(int64_t)py * p.pgx + px];
+      if (last) p.hcnt[idx] = 0u;  // every reader of this execute has counted: ready for the next one
+    }
+    // the whole warp drops each completed producer block's lines (u8 input: bytes = pixels)
+    for (unsigned m = __ballot_sync(0xFFFFFFFFu, last); m; m &= m - 1) {
+      const int src = __ffs(m) - 1;
+      const int qy = __shfl_sync(0xFFFFFFFFu, py, src), qx = __shfl_sync(0xFFFFFFFFu, px, src);
+      const int64_t x0 = (int64_t)p.wax * qx, x1 = min((int64_t)p.in.W, x0 + p.wax);
+      const int64_t y0 = (int64_t)p.way * qy, y1 = min((int64_t)p.in.H, y0 + p.way);
+      const int64_t a0 = (int64_t)(uintptr_t)(fb + y0 * p.in.pitch + x0);
+      const int64_t l0 = (a0 + 127) >> 7, l1 = (a0 + (x1 - x0)) >> 7;  // whole lines of the first row
+      const int64_t per = l1 > l0 ? l1 - l0 : 0, tot = per * (y1 - y0);
+      for (int64_t k = lane; k < tot; k += 32) {
+        const int64_t r = k / per, l = k - r * per;
+        ktd::discard_line(reinterpret_cast<const void*>(((l0 + l) << 7) + r * p.in.pitch));
+      }
+    }
+  }
+}
+
 template <int OP, bool SCALAR>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
@@ -289,6 +332,10 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       if constexpr (OP == 2 || OP == 4) {
         if (p.cdisc) consumer_discard<OP>(p, t, nt, tid);
       }
+      if constexpr (OP == 1 || OP == 3) {  // as soon as staged: the earlier, the fewer write-backs
+        if (p.hcnt && tid < 32) halo_discard(p, t, tid);
+      }
+
       if ((OP == 1 || OP == 3 || OP == 6 || OP == 7) && ktd::needs_fix(OP, p.in, t)) {
         ktd::stage_fix(OP, p.in, t, buf, nt, tid);
         __syncthreads();
@@ -801,6 +848,7 @@ struct ktiler_plan_s {
   bool executed = false;
   // GRAPH_CHAIN state: one device block (epoch | flags | dcount | prefix) and the tail
   void* cmem = nullptr;
+  std::vector<void*> hmem;  // halo-reader counters of consumer discards
   unsigned int* epoch = nullptr;
   std::vector<Launch> chain_tail;
   ~ktiler_plan_s() {
@@ -809,6 +857,7 @@ struct ktiler_plan_s {
     if (dmem) cudaFree(dmem);
     if (tb.rec) cudaFree(tb.rec);
     if (cmem) cudaFree(cmem);
+    for (void* m : hmem) cudaFree(m);
   }
 };
 
@@ -1430,6 +1479,61 @@ ktiler_status setup_chain(ktiler_plan_s* P) {
   return KTILER_OK;
 }
 
+// KTILER_PF_HALO_DISCARD (A44): blur5 / sobel3 launches of a tiled plan
+// whose input is an internal buffer they alone read get a reader count per producer block
+// (consumer blocks whose declared read rect meets it: Graph::consumers) and zeroed counters.
+ktiler_status setup_halo_discard(ktiler_plan_s* P) {
+  const kt::Graph& g = P->g;
+  if (!(P->pol.flags & KTILER_PF_HALO_DISCARD) || P->s.nfrag <= 1) return KTILER_OK;
+  std::vector<std::pair<unsigned int*, const uint8_t*>> per_node(g.nodes.size(), {nullptr, nullptr});
+  for (auto& L : P->launches) {
+    if (L.node < 0 || L.n->scalar || (L.n->op != KTILER_OP_BLUR5 && L.n->op != KTILER_OP_SOBEL3)) continue;
+    const kt::Node& n = g.nodes[L.node];
+    const kt::Access& r = n.acc[n.racc];
+    const kt::Buffer& ib = g.bufs[r.buf];
+    if (!(ib.d.flags & KTILER_BUF_INTERNAL) || ib.readers.size() != 1 || !discardable(ib) || ib.writer < 0) continue;
+    const kt::Chan* ch = nullptr;
+    for (const kt::Chan& c : g.in_ch[L.node])
+      if (c.buf == r.buf) ch = &c;
+    if (!ch) continue;
+    const kt::Node& u = g.nodes[ch->u];
+    const kt::Access& uw = u.acc[ch->w];
+    if (g.nodes[ch->u].op == KTILER_OP_CUSTOM || u.gx() > (1 << 20) || u.gy() > (1 << 20)) continue;
+    auto& slot = per_node[L.node];
+    if (!slot.first) {
+      const int64_t gx = u.gx(), gy = u.gy(), gz = u.gz();
+      std::vector<uint8_t> need((size_t)(gx * gy));
+      for (int64_t py = 0; py < gy; ++py)
+        for (int64_t px = 0; px < gx; ++px) {
+          const kt::BRange c = g.consumers(*ch, px, py);
+          const int64_t k = c.empty() ? 0 : (c.x1 - c.x0) * (c.y1 - c.y0);
+          if (k > 255) return fail(KTILER_E_UNSUPPORTED, "consumer discard: more than 255 readers of one block");
+          need[(size_t)(py * gx + px)] = (uint8_t)k;
+        }
+      void* cnt = nullptr;
+      void* nd = nullptr;
+      cudaError_t e = cudaMalloc(&cnt, (size_t)(gx * gy * gz) * 4);
+      if (e == cudaSuccess) e = cudaMalloc(&nd, need.size());
+      if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (halo-reader counters)");
+      P->hmem.push_back(cnt);
+      P->hmem.push_back(nd);
+      if ((e = cudaMemset(cnt, 0, (size_t)(gx * gy * gz) * 4)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
+      if ((e = cudaMemcpy(nd, need.data(), need.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+        return cuda_fail(e, "cudaMemcpy");
+      slot = {(unsigned int*)cnt, (const uint8_t*)nd};
+    }
+    KParams& k = L.kp;
+    k.hcnt = slot.first;
+    k.hneed = slot.second;
+    k.pgx = (int32_t)u.gx();
+    k.pgy = (int32_t)u.gy();
+    k.rax = (int32_t)r.ax; k.ray = (int32_t)r.ay; k.rox = (int32_t)r.ox; k.roy = (int32_t)r.oy;
+    k.rhl = r.hl; k.rhr = r.hr; k.rht = r.ht; k.rhb = r.hb;
+    k.wax = (int32_t)uw.ax; k.way = (int32_t)uw.ay;
+  }
+  return KTILER_OK;
+}
+
 ktiler_status setup_persistent(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const kt::Schedule& S = P->s;
@@ -1792,6 +1896,10 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
       for (auto& L : p->launches)
         if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar && L.kp.stage_bytes)
           L.kp.use_tmap = make_tmap(p->g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
+      {
+        ktiler_status s = setup_halo_discard(p);
+        if (s) return s;
+      }
       if (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN) {
         ktiler_status s = setup_chain(p);
         if (s) return s;

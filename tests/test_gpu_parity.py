@@ -97,6 +97,7 @@ MODES = [
     dict(exec_mode="dag", pdl=True),  # programmatic edges from each sub-kernel's producers
     dict(exec_mode="dag", consumer_discard=True),  # down2 / thresh drop their consumed lines
     dict(exec_mode="graph", consumer_discard=True),
+    dict(exec_mode="dag", consumer_discard=True, halo_discard=True),  # + counted halo-reader discards
     dict(exec_mode="dag", window=1),
     dict(exec_mode="dag", window=4),
     dict(exec_mode="chain"),

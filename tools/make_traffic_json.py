@@ -19,7 +19,8 @@ for k in range(0, len(args), 3):
         cfg = {"workload": "batch64_8k", "mode": c.get("exec_mode", "graph"), "policy": c.get("kind", "budget"),
                "l2_fraction": c.get("l2_fraction", 1.0), "discard": bool(c.get("discard", False)),
                "window": c.get("window", 2), "resident_budget": bool(c.get("resident_budget", False)),
-               "consumer_discard": bool(c.get("consumer_discard", False))}
+               "consumer_discard": bool(c.get("consumer_discard", False)),
+               "halo_discard": bool(c.get("halo_discard", False))}
         if c.get("skew"):
             cfg["skew"] = c["skew"]
         entries.append({"config": cfg, "dram_bytes_per_step": r["dram_GB"] * 1e9, "dram_read": r["read_GB"] * 1e9,
