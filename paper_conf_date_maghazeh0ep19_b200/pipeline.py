@@ -26,7 +26,7 @@ from . import ktiler as K
 # op -> (tile w, tile h, threads per block) for the vector variant
 B200_GEOMETRY = {
     "gray": (256, 32, 128),    # 512 items of 16 px (4 per thread); 24.6 KB staged rgb
-    "blur": (256, 64, 64),     # 64 column strips x 16 rows; 19.6 KB staged halo tile
+    "blur": (512, 64, 128),    # 128 column strips x 16 rows; 37 KB staged halo tile
     "down": (256, 32, 128),    # 512 items (4 per thread); 32 KB staged blur rows
     "sobel": (256, 64, 128),   # 128 strips x 8 rows; 19 KB halo tile
     "thresh": (256, 32, 128),  # 512 items (4 per thread); 32 KB staged f32

@@ -1,0 +1,5 @@
+C='[{"kind":"none","exec_mode":"graph"},{"kind":"budget","l2_fraction":0.85,"exec_mode":"dag","discard":false,"window":2,"resident_budget":true,"consumer_discard":true}]'
+for i in 1 2 3; do
+for g in '{}' '{"blur":[512,64,128]}' '{"blur":[512,64,128],"sobel":[256,128,128]}'; do
+  echo "geom $g"; timeout 300 python tools/sweep.py --reps 9 --geom "$g" --configs "$C" 2>&1 | python tools/compact.py
+done; done
