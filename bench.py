@@ -190,7 +190,21 @@ def cpu_baseline(W, H, T, seed, target_s):
         dt += time.perf_counter() - t1
         n += 1
     return {"value": W * rows * n / dt / 1e6, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} x {W}x{rows} scene image(s) through the untiled oracle graph, 1 thread, {dt:.1f} s"}
+            "sample": f"{n} x {W}x{rows} scene image(s) through the untiled oracle graph, 1 thread, {dt:.1f} s",
+            "host": host_cpu()}
+
+
+def host_cpu() -> dict:
+    """The oracle's host: CPU model name (/proc/cpuinfo) and the cores the OS exposes."""
+    name = "unknown"
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                name = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"model": name, "nproc": os.cpu_count()}
 
 
 def run_reference(args):
@@ -218,7 +232,7 @@ def run_reference(args):
         "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic", "config": {"workload": args.workload, "W": W, "H": H, "frames": Ftot, "baseline_config": cfg},
         "impl": "reference",
-        "cpu_baseline": {"value": v, "unit": "Mpix/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": v, "unit": "Mpix/s", "cores": 1, "kind": "oracle", "sample": sample, "host": host_cpu()},
         "e2e": {"value": v, "unit": "Mpix/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
 
 
@@ -321,21 +335,28 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
-    def timed(fn, steps, warm, clocks=None):
+    step_ms = []  # per-step event times of the last timed() with per_step=True (this rank)
+
+    def timed(fn, steps, warm, clocks=None, per_step=False):
         for _ in range(warm):
             fn()
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        marks = [torch.cuda.Event(enable_timing=True) for _ in range(steps)] if per_step else []
         if clocks:
             clocks.__enter__()
         e0.record(stream)
-        for _ in range(steps):
+        for k in range(steps):
             fn()
+            if per_step:
+                marks[k].record(stream)
         e1.record(stream)
         barrier()
         if clocks:
             clocks.__exit__()
         ms = e0.elapsed_time(e1) / steps
+        if per_step:
+            step_ms[:] = [(e0 if k == 0 else marks[k - 1]).elapsed_time(marks[k]) for k in range(steps)]
         if world > 1:
             t = torch.tensor([ms], device="cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -348,7 +369,7 @@ def main():
         plan.execute(s)
 
     clk = Clocks(local)
-    ms = timed(step, args.steps, args.warmup, clocks=clk)
+    ms = timed(step, args.steps, args.warmup, clocks=clk, per_step=True)
     pix = pix_rank * world
     value = pix / (ms / 1000) / 1e6
     peak, peak_src = peaks()
@@ -366,6 +387,8 @@ def main():
         "steps": args.steps,
         "warmup": args.warmup,
         "ms_per_step": ms,
+        "step_ms": {q: round(statistics.quantiles(step_ms, n=10)[i] if len(step_ms) >= 2 else ms, 4)
+                    for q, i in (("p10", 0), ("p50", 4), ("p90", 8))},
         "higher_is_better": True,
         "scaling": "strong" if (shard == "strips" or (shard == "frames" and args.scaling == "strong")) else "weak",
         "vs_baseline": None,
