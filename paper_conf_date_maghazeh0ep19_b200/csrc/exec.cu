@@ -871,6 +871,19 @@ DBuf dbuf(const kt::Buffer& b) {
 
 bool discardable(const kt::Buffer& b) { return (b.d.pitch_bytes % 128 == 0) && (b.d.frame_stride_bytes % 128 == 0); }
 
+// With KTILER_PF_CONSUMER_DISCARD in a tiled plan, buffer b's lines are dropped by its only
+// reader as soon as they are staged (A44): no discard list is needed for it.
+bool consumer_drops(const ktiler_plan_s* P, int b) {
+  const kt::Graph& g = P->g;
+  if (!(P->pol.flags & KTILER_PF_CONSUMER_DISCARD) || P->s.nfrag <= 1) return false;
+  const kt::Buffer& B = g.bufs[b];
+  if (!(B.d.flags & KTILER_BUF_INTERNAL) || B.readers.size() != 1 || B.writer < 0) return false;
+  const kt::Node& n = g.nodes[B.readers[0]];
+  if (n.scalar || (n.op != KTILER_OP_DOWN2 && n.op != KTILER_OP_THRESH)) return false;
+  const kt::Access& r = n.acc[n.racc];
+  return r.buf == b && !r.hl && !r.hr && !r.ht && !r.hb;
+}
+
 DRect drect(const kt::Graph& g, const kt::Discard& d) {
   const kt::Buffer& b = g.bufs[d.buf];
   DRect r;
@@ -987,7 +1000,7 @@ void build_launches(ktiler_plan_s* P) {
     }
     if (disc)
       for (auto& d : P->s.discards[si]) {
-        if (!discardable(g.bufs[d.buf])) continue;
+        if (!discardable(g.bufs[d.buf]) || consumer_drops(P, d.buf)) continue;  // A44: its reader drops it
         DRect dr = drect(g, d);
         if (dr.lpr > 0) pending.push_back(dr);
       }
