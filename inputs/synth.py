@@ -4,7 +4,7 @@ This module holds NONE of KTILER's arithmetic: it only produces the graph
 input image (interleaved RGB8, dense pitch 3*W, frames contiguous) that both
 the CPU oracle and the CUDA path consume.  The same counter-based generator is
 implemented a second time in ``inputs/synth_gpu.cu`` so that multi-GB inputs
-can be produced on the device without an upload; ``tests/test_inputs_gpu.py``
+can be produced on the device without an upload; ``tests/test_gpu_parity.py::test_gpu_generator_matches_numpy``
 checks the two byte for byte.
 
 Generators (the recipe DESIGN.md §3 states):

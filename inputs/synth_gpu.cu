@@ -1,7 +1,7 @@
 // Device twin of inputs/synth.py (seeded synthetic RGB8 inputs).
 // Holds none of KTILER's arithmetic; it exists only so multi-GB benchmark inputs
 // can be generated in HBM instead of uploaded.  Same counter-based generator as
-// the numpy version; tests/test_inputs_gpu.py checks them byte for byte.
+// the numpy version; tests/test_gpu_parity.py::test_gpu_generator_matches_numpy checks them byte for byte.
 #include <cstdint>
 #include <cuda_runtime.h>
 

@@ -10,7 +10,7 @@ timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; ech
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 4000 --csv --log-file gpurun_out/launches.csv \
   python bench.py --steps 2 --warmup 1 --no-cpu --no-e2e --no-trace --no-untiled > gpurun_out/launches_bench.log 2>&1
 echo "launches rc=$?"
-CFG="$(cat tools/cfg_traffic_r01s3.json)"
+CFG="$(python tools/run_sweep.py --config cfg_traffic_r01s3)"
 timeout 900 ncu --graph-profiling graph --cache-control all --clock-control none \
   --metrics dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__time_duration.sum --csv \
   python tools/sweep.py --reps 1 --configs "$CFG" > gpurun_out/traffic_cfg.csv 2> gpurun_out/traffic_cfg.err
