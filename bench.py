@@ -4,9 +4,10 @@ Workload (default ``batch64_8k`` = BASELINE configs[3]): 64 frames of 8K (7680x4
 through the 5-kernel pipeline gray -> blur5 -> down2 -> sobel3 -> thresh, the
 configuration the north star's 1-GPU target is stated on ("8K-class images on one B200")
 and the one its multi-GPU scaling target uses ("frame batches").  With --gpus N (one
-process per GPU, launched by torchrun) every rank runs its own 64-frame batch — frame
-sharding with no data-path collective, per-GPU work fixed ("scaling": "weak"; --scaling
-strong splits one 64-frame batch across the ranks instead).  Workload
+process per GPU, launched by torchrun) the batch is sharded by frames — frame
+sharding with no data-path collective: by default the one 64-frame batch is split into
+contiguous frame ranges (64/N frames per GPU, "scaling": "strong"; frames.frame_range);
+--scaling weak gives every rank a whole batch of its own instead.  Workload
 ``strip_65536`` (configs[4]) splits one 65536x65536 image into row strips whose 4 halo
 rows per side move over NCCL send/recv before each step.
 
@@ -66,8 +67,9 @@ def parse(argv=None):
     ap.add_argument("--l2-fraction", type=float, default=0.85)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
-                    help="frames: weak = every rank runs the whole batch (per-GPU work fixed), strong = split it")
+    ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
+                    help="frames: strong (default) = the one batch split into contiguous frame ranges "
+                         "(BASELINE configs[3]); weak = every rank runs a whole batch of its own")
     ap.add_argument("--window", type=int, default=2)
     ap.add_argument("--discard", action="store_true",
                     help="discard dead intermediate lines (DRAM -55%% but slower on B200: DESIGN.md §6)")
@@ -299,6 +301,7 @@ def main():
 
     from inputs import gpu as G
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    from paper_conf_date_maghazeh0ep19_b200 import frames as FR
     from paper_conf_date_maghazeh0ep19_b200.strips import StripPipeline
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -321,11 +324,16 @@ def main():
         G.fill("scene", args.seed, sp.rgb_ext()[sp.own_offset:].data_ptr(), W * 3, 0, W, H, y0=sp.o0,
                rows=sp.o1 - sp.o0, F=1, stream=s)
         pix_rank = W * (sp.o1 - sp.o0)
+        pix_ranks = [pix_rank] * world
         per = 1
     else:
-        strong = shard == "frames" and args.scaling == "strong" and Ftot >= world
-        per = Ftot // world if strong else Ftot
-        f0 = rank * per if shard == "frames" else 0
+        strong = shard == "frames" and args.scaling == "strong"
+        if strong:  # contiguous frame ranges, the first Ftot % world ranks one frame more
+            f0, per = FR.frame_range(Ftot, world, rank)
+            pix_ranks = [W * H * FR.frame_range(Ftot, world, r)[1] for r in range(world)]
+        else:  # weak: every rank its own whole batch (frames Ftot*rank ...)
+            f0, per = (rank * Ftot if shard == "frames" else 0), Ftot
+            pix_ranks = [W * H * Ftot] * world
         p = Pipeline(W, H, per, T=args.T, internal=True)
         G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
         pix_rank = W * H * per
@@ -362,11 +370,7 @@ def main():
         ms = e0.elapsed_time(e1) / steps
         if per_step:
             step_ms[:] = [(e0 if k == 0 else marks[k - 1]).elapsed_time(marks[k]) for k in range(steps)]
-        if world > 1:
-            t = torch.tensor([ms], device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = float(t.item())
-        return ms
+        return FR.max_over_ranks(ms, world, device="cuda")
 
     def step():
         if sp is not None and world > 1:
@@ -375,11 +379,11 @@ def main():
 
     clk = Clocks(local)
     ms = timed(step, args.steps, args.warmup, clocks=clk, per_step=True)
-    pix = pix_rank * world
-    value = pix / (ms / 1000) / 1e6
+    pix = sum(pix_ranks)
+    value = FR.job_mpix_per_s(pix_ranks, ms)
     peak, peak_src = peaks()
     comp_bytes = pix * 3.25  # rgb in + mask out: the method's algorithmic bytes
-    achieved = comp_bytes / (ms / 1000) / 1e9
+    achieved = comp_bytes / world / (ms / 1000) / 1e9  # per GPU, against one GPU's peak
     tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
             "discard": discard, "window": args.window, "resident_budget": resident,
             "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"]}

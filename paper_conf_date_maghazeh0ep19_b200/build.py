@@ -11,7 +11,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libktiler.so")
 SOURCES = ["graph.cpp", "planner.cpp", "exec.cu"]
-HEADERS = ["kt_internal.h", "kernels.cuh"]
+HEADERS = ["kt_internal.h", "kernels.cuh", "flow.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3,-Wall", "-Xptxas", "-v",

@@ -21,6 +21,7 @@
 #include <cstdlib>
 #include <cstring>
 
+#include "flow.cuh"
 #include "kernels.cuh"
 #include "kt_internal.h"
 
@@ -846,6 +847,13 @@ struct ktiler_plan_s {
   bool has_custom = false;
   TraceBuf tb{nullptr, nullptr, 0};
   bool executed = false;
+  ktiler_status sticky = KTILER_OK;  // a failed first-execute setup: the plan stays unusable
+  // FLOW state (KTILER_EXEC_FLOW): roles (ktiler_plan_set_flow_roles; empty = automatic)
+  std::vector<int32_t> flow_node_role, flow_slot_role;
+  ktflow::FParams fp{};
+  void (*ffn)(ktflow::FParams) = nullptr;
+  int fctas = 0, fthreads = 0, fsmem = 0;
+  void* fmem = nullptr;
   // GRAPH_CHAIN state: one device block (epoch | flags | dcount | prefix) and the tail
   void* cmem = nullptr;
   std::vector<void*> hmem;  // halo-reader counters of consumer discards
@@ -855,6 +863,7 @@ struct ktiler_plan_s {
     if (exec) cudaGraphExecDestroy(exec);
     if (graph) cudaGraphDestroy(graph);
     if (dmem) cudaFree(dmem);
+    if (fmem) cudaFree(fmem);
     if (tb.rec) cudaFree(tb.rec);
     if (cmem) cudaFree(cmem);
     for (void* m : hmem) cudaFree(m);
@@ -881,7 +890,13 @@ bool consumer_drops(const ktiler_plan_s* P, int b) {
   const kt::Node& n = g.nodes[B.readers[0]];
   if (n.scalar || (n.op != KTILER_OP_DOWN2 && n.op != KTILER_OP_THRESH)) return false;
   const kt::Access& r = n.acc[n.racc];
-  return r.buf == b && !r.hl && !r.hr && !r.ht && !r.hb;
+  if (r.buf != b || r.hl || r.hr || r.ht || r.hb) return false;
+  // consumer_discard drops only the lines wholly inside one block's input rect: the
+  // reader's blocks cover every line only when a block's input row is a whole number of
+  // lines (down2 reads 2 bytes, thresh 4 bytes per output pixel); otherwise the lines that
+  // straddle two blocks still need the scheduled list
+  const int64_t eb = n.op == KTILER_OP_DOWN2 ? 2 : 4;
+  return (eb * n.acc[n.wacc].ax) % 128 == 0;
 }
 
 DRect drect(const kt::Graph& g, const kt::Discard& d) {
@@ -1611,7 +1626,7 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   P->psmem = std::max(slot, 128) * nslots;
   if (P->psmem + (int)fa.sharedSizeBytes > smem_blk)
     return fail(KTILER_E_UNSUPPORTED, "PERSISTENT mode: staging slots exceed shared memory");
-  if (P->psmem > 48 * 1024) {
+  if (P->psmem + (int)fa.sharedSizeBytes > 48 * 1024) {
     cudaError_t ea = cudaFuncSetAttribute((const void*)P->pfn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->psmem);
     if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (persistent smem)");
   }
@@ -1796,6 +1811,277 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   return KTILER_OK;
 }
 
+
+// ------------------------------------------------------------------------------------
+// KTILER_EXEC_FLOW setup (flow.cuh): node table, global pipelined order, role ticket
+// lists, run-ahead window, slot -> role map, kernel variant and ring depth.
+// ------------------------------------------------------------------------------------
+typedef void (*ffn_t)(ktflow::FParams);
+ffn_t flow_variant(int k) {
+  switch (k) {
+    case 2: return ktflow::flow_kernel<4, 2>;
+    case 3: return ktflow::flow_kernel<4, 3>;
+    case 5: return ktflow::flow_kernel<3, 5>;
+    default: return ktflow::flow_kernel<4, 4>;
+  }
+}
+int flow_threads(int k) { return k == 5 ? 128 : 160; }
+
+// Automatic roles: every node its own role when the slots allow, the slots shared out in
+// proportion to each node's staged + written bytes (at least one each); otherwise
+// consecutive nodes (topological order) grouped into K roles of balanced bytes.
+void flow_auto_roles(const kt::Graph& g, int K, std::vector<int32_t>& node_role, std::vector<int32_t>& slot_role) {
+  const int nn = (int)g.nodes.size();
+  std::vector<double> wt(nn, 0.0);
+  for (int v = 0; v < nn; ++v) {
+    const kt::Node& n = g.nodes[v];
+    const kt::Access& w = n.acc[n.wacc];
+    const double per = ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) +
+                       (double)w.ax * w.ay * g.bufs[w.buf].d.elem_bytes;
+    wt[v] = per * (double)n.nblocks;
+  }
+  node_role.assign(nn, 0);
+  slot_role.clear();
+  if (nn <= K) {
+    for (int i = 0; i < nn; ++i) node_role[g.topo[i]] = i;
+    std::vector<int> cnt(nn, 1);
+    double tot = 0;
+    for (double x : wt) tot += x;
+    for (int extra = K - nn; extra > 0; --extra) {  // largest weight per slot gets the next slot
+      int best = 0;
+      double bv = -1;
+      for (int i = 0; i < nn; ++i) {
+        const double r = wt[g.topo[i]] / cnt[i];
+        if (r > bv) { bv = r; best = i; }
+      }
+      ++cnt[best];
+    }
+    for (int i = 0; i < nn; ++i)
+      for (int c = 0; c < cnt[i]; ++c) slot_role.push_back(i);
+    (void)tot;
+    return;
+  }
+  // nn > K: contiguous groups, greedy on the running weight
+  double tot = 0;
+  for (double x : wt) tot += x;
+  double acc = 0;
+  int r = 0;
+  for (int i = 0; i < nn; ++i) {
+    const int v = g.topo[i];
+    if (r < K - 1 && acc > 0 && acc + wt[v] / 2 > tot * (r + 1) / K) ++r;
+    acc += wt[v];
+    node_role[v] = r;
+  }
+  for (int i = 0; i < K; ++i) slot_role.push_back(std::min(i, r));
+}
+
+ktiler_status setup_flow(ktiler_plan_s* P) {
+  using namespace ktflow;
+  const kt::Graph& g = P->g;
+  const kt::Schedule& S = P->s;
+  const int nn = (int)g.nodes.size();
+  const int nsub = (int)S.subs.size();
+  if (nn > FMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: at most 32 nodes");
+  for (auto& n : g.nodes) {
+    if (n.op < KTILER_OP_GRAY || n.op > KTILER_OP_THRESH || n.scalar)
+      return fail(KTILER_E_UNSUPPORTED, "FLOW mode runs the vector image-pipeline built-ins (GRAY..THRESH) only");
+    if (n.gx() > 4096 || n.gy() > 4096 || n.gz() > 4096)
+      return fail(KTILER_E_UNSUPPORTED, "FLOW mode: grid exceeds the ticket (4096 blocks per axis and frames)");
+  }
+  // ---- node table ----
+  std::vector<int64_t> flag0(nn);
+  int64_t nflags = 0;
+  for (int v = 0; v < nn; ++v) {
+    flag0[v] = nflags;
+    nflags += g.nodes[v].nblocks;
+  }
+  std::vector<FNode> fnodes(nn);
+
+  for (int v = 0; v < nn; ++v) {
+    const kt::Node& n = g.nodes[v];
+    const kt::Access& w = n.acc[n.wacc];
+    const kt::Access& r = n.acc[n.racc];
+    FNode& q = fnodes[v];
+    std::memset(&q, 0, sizeof(q));
+    if (!make_tmap(g, n, &q.tmap, &q.box_bytes)) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: input tile map unavailable");
+    q.in = dbuf(g.bufs[r.buf]);
+    q.out = dbuf(g.bufs[w.buf]);
+    q.flag0 = flag0[v];
+    q.op = n.op;
+    q.tw = (int32_t)w.ax;
+    q.th = (int32_t)w.ay;
+    q.T = n.T;
+    q.gx = (int32_t)n.gx();
+    q.gy = (int32_t)n.gy();
+    q.leaf = g.out_ch[v].empty();
+    const kt::Buffer& ib = g.bufs[r.buf];
+    // evict-first reads: the graph input, and intermediates with one reader node (DESIGN A42)
+    q.in_stream = ib.readers.size() == 1 || !g.written_by_node(r.buf);
+    q.cdisc = (P->pol.flags & KTILER_PF_CONSUMER_DISCARD) && (n.op == KTILER_OP_DOWN2 || n.op == KTILER_OP_THRESH) &&
+              (ib.d.flags & KTILER_BUF_INTERNAL) && ib.readers.size() == 1 && !r.hl && !r.hr && !r.ht && !r.hb &&
+              discardable(ib) && g.written_by_node(r.buf);
+    if (g.in_ch[v].size() > 1) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: one producer per node");
+    for (auto& c : g.in_ch[v]) {
+      const kt::Node& pu = g.nodes[c.u];
+      const kt::Access& uw = pu.acc[c.w];
+      q.pflag0 = flag0[c.u];
+      q.pgx = (int32_t)pu.gx();
+      q.pgy = (int32_t)pu.gy();
+      q.rax = (int32_t)r.ax; q.ray = (int32_t)r.ay; q.rox = (int32_t)r.ox; q.roy = (int32_t)r.oy;
+      q.rhl = r.hl; q.rhr = r.hr; q.rht = r.ht; q.rhb = r.hb;
+      q.wax = (int32_t)uw.ax; q.way = (int32_t)uw.ay;
+    }
+
+  }
+  // ---- kernel variant, slots (CTAs) per SM, shared memory per CTA ----
+  int K = P->flow_slot_role.empty() ? 4 : (int)P->flow_slot_role.size();
+  if (K < 2 || K > 5) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: 2..5 slots (CTAs) per SM");
+  P->ffn = flow_variant(K);
+  P->fthreads = flow_threads(K);
+  int nsm = 0, smem_sm = 0, smem_blk = 0;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+  cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
+  cudaDeviceGetAttribute(&smem_blk, cudaDevAttrMaxSharedMemoryPerBlockOptin, P->device);
+  cudaFuncAttributes fa{};
+  cudaFuncGetAttributes(&fa, (const void*)P->ffn);
+  P->fsmem = (std::min(smem_sm / K - 1024, smem_blk) - (int)fa.sharedSizeBytes) & ~127;
+  {  // static + dynamic may pass the 48 KB default
+    cudaError_t ea = cudaFuncSetAttribute((const void*)P->ffn, cudaFuncAttributeMaxDynamicSharedMemorySize, P->fsmem);
+    if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (flow smem)");
+  }
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, P->ffn, P->fthreads, P->fsmem);
+  if (occ < K) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: " + std::to_string(K) + " CTAs do not fit an SM (" +
+                                                     std::to_string(occ) + ")");
+  P->fctas = nsm * K;
+  // ---- roles ----
+  std::vector<int32_t> node_role = P->flow_node_role, slot_role = P->flow_slot_role;
+  if (node_role.empty() || slot_role.empty()) flow_auto_roles(g, K, node_role, slot_role);
+  if ((int)node_role.size() != nn) return fail(KTILER_E_INVALID, "FLOW roles: one role per node");
+  int nroles = 0;
+  for (int r : node_role) nroles = std::max(nroles, r + 1);
+  if (nroles > FMAX_ROLES) return fail(KTILER_E_INVALID, "FLOW roles: at most 16");
+  std::vector<int> served(nroles, 0);
+  for (int r : slot_role) {
+    if (r < 0 || r >= nroles) return fail(KTILER_E_INVALID, "FLOW roles: slot role out of range");
+    served[r] = 1;
+  }
+  for (int r = 0; r < nroles; ++r)
+    if (!served[r]) return fail(KTILER_E_INVALID, "FLOW roles: every role needs a slot");
+  // ---- each role's ring: slots of its largest staged tile, as many as the CTA's smem holds ----
+  std::vector<int32_t> rstage(FMAX_ROLES, 128), rslots(FMAX_ROLES, 0);
+  for (int v = 0; v < nn; ++v) {
+    const kt::Node& n = g.nodes[v];
+    const kt::Access& w = n.acc[n.wacc];
+    rstage[node_role[v]] = std::max(rstage[node_role[v]], (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
+  }
+  int cap_slots = FSLOTS_MAX;
+  if (const char* ev = getenv("KTILER_FLOW_SLOTS")) cap_slots = std::min(FSLOTS_MAX, std::max(2, atoi(ev)));
+  for (int r = 0; r < nroles; ++r) {
+    rslots[r] = std::min(cap_slots, P->fsmem / rstage[r]);
+    if (rslots[r] < 2) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: tiles too large for two staging slots per CTA");
+  }
+  // ---- the global order: software pipeline over fragments (A37), deepest node first ----
+  std::vector<int> depth(nn, 0);
+  int dmax = 0;
+  for (int v : g.topo)
+    for (auto& c : g.in_ch[v]) depth[v] = std::max(depth[v], depth[c.u] + 1);
+  for (int v = 0; v < nn; ++v) dmax = std::max(dmax, depth[v]);
+  const int64_t nfrag = S.nfrag;
+  std::vector<std::vector<int>> by_frag(nfrag, std::vector<int>(nn, -1));
+  for (int i = 0; i < nsub; ++i) by_frag[S.subs[i].frag][S.subs[i].node] = i;
+  const int64_t k = P->pol.pipeline_skew > 0 ? P->pol.pipeline_skew : 1;
+  P->skew = k;
+  // run-ahead window: a source tile of fragment f waits for the leaf tiles of fragments
+  // <= f - W; W > dmax * k keeps every window dependency earlier in the global order
+  // window: policy.window fragments beyond the pipeline depth, or (0) as many fragments as
+  // the L2 budget holds of the intermediates they write (CheckCacheConst)
+  int64_t wextra = P->pol.window;
+  if (wextra <= 0) {
+    double inter = 0;
+    for (int v = 0; v < nn; ++v)
+      if (!fnodes[v].leaf) {
+        const kt::Node& n = g.nodes[v];
+        const kt::Access& w = n.acc[n.wacc];
+        inter += (double)n.nblocks * (double)w.ax * (double)w.ay * g.bufs[w.buf].d.elem_bytes;
+      }
+    const double per_frag = inter / std::max<int64_t>(1, nfrag);
+    wextra = per_frag > 0 ? (int64_t)std::floor((double)S.budget / per_frag) : 2;
+    wextra = std::max<int64_t>(2, std::min<int64_t>(wextra, nfrag));
+  }
+  const int64_t W = dmax * k + wextra;
+  std::vector<int64_t> leaf_upto(nfrag + 1, 0);  // leaf tiles of fragments < f
+  for (int64_t f = 0; f < nfrag; ++f) {
+    int64_t c = 0;
+    for (int v = 0; v < nn; ++v)
+      if (fnodes[v].leaf && by_frag[f][v] >= 0) c += S.subs[by_frag[f][v]].nblocks;
+    leaf_upto[f + 1] = leaf_upto[f] + c;
+  }
+  if (leaf_upto[nfrag] > (int64_t)FLOW_WAIT_MAX) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: too many leaf tiles");
+  std::vector<std::vector<uint64_t>> lists(nroles);
+  std::vector<int> rtopo(g.topo.rbegin(), g.topo.rend());
+  for (int64_t st = 0; st < nfrag + dmax * k; ++st)
+    for (int v : rtopo) {
+      const int64_t f = st - depth[v] * k;
+      if (f < 0 || f >= nfrag || by_frag[f][v] < 0) continue;
+      const kt::SubKernel& sk = S.subs[by_frag[f][v]];
+      const uint64_t wait = (depth[v] == 0 && f - W >= 0 && nn > 1) ? (uint64_t)leaf_upto[f - W + 1] : 0;
+      std::vector<uint64_t>& L = lists[node_role[v]];
+      for (auto& r : sk.rects)
+        for (int64_t z = r.z0; z < r.z1; ++z)
+          for (int64_t y = r.y0; y < r.y1; ++y)
+            for (int64_t x = r.x0; x < r.x1; ++x) L.push_back(flow_ticket((uint64_t)v, wait, x, y, z));
+    }
+  std::vector<int64_t> role_off(nroles + 1, 0);
+  for (int r = 0; r < nroles; ++r) role_off[r + 1] = role_off[r] + (int64_t)lists[r].size();
+  // ---- one device allocation: ctrl | claims | smslot | slot_role | role_off | flags | nodes | tickets ----
+  auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  const size_t o_ctrl = 0, o_claim = al(sizeof(FCtrl)), o_sms = o_claim + al(FMAX_ROLES * 4);
+  const size_t o_sr = o_sms + al(256 * 4), o_ro = o_sr + al(FMAX_SLOTS * 4), o_fl = o_ro + al((nroles + 1) * 8);
+  const size_t o_nd = o_fl + al((size_t)nflags * 4), o_tk = o_nd + al(fnodes.size() * sizeof(FNode));
+  const size_t total = o_tk + al((size_t)role_off[nroles] * 8 + 8);
+  char* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, total);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (flow tables)");
+  P->fmem = d;
+  if ((e = cudaMemset(d, 0, total)) != cudaSuccess) return cuda_fail(e, "cudaMemset");
+  const FCtrl c0{1, 0, 0, 0};
+  std::vector<int32_t> sr(FMAX_SLOTS, 0);
+  for (size_t i = 0; i < slot_role.size(); ++i) sr[i] = slot_role[i];
+  cudaMemcpy(d + o_ctrl, &c0, sizeof(c0), cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_sr, sr.data(), sr.size() * 4, cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_ro, role_off.data(), role_off.size() * 8, cudaMemcpyHostToDevice);
+  cudaMemcpy(d + o_nd, fnodes.data(), fnodes.size() * sizeof(FNode), cudaMemcpyHostToDevice);
+  for (int r = 0; r < nroles; ++r)
+    if (!lists[r].empty())
+      cudaMemcpy(d + o_tk + role_off[r] * 8, lists[r].data(), lists[r].size() * 8, cudaMemcpyHostToDevice);
+  if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "cudaMemcpy (flow tables)");
+  FParams& fp = P->fp;
+  fp.nodes = (const FNode*)(d + o_nd);
+  fp.tickets = (const uint64_t*)(d + o_tk);
+  fp.role_off = (const int64_t*)(d + o_ro);
+  fp.slot_role = (const int32_t*)(d + o_sr);
+  fp.claim = (unsigned int*)(d + o_claim);
+  fp.smslot = (unsigned int*)(d + o_sms);
+  fp.flags = (unsigned int*)(d + o_fl);
+  fp.ctrl = (FCtrl*)(d + o_ctrl);
+  for (int r = 0; r < FMAX_ROLES; ++r) {
+    fp.role_stage[r] = rstage[r];
+    fp.role_nslots[r] = rslots[r];
+  }
+  fp.nslots_sm = K;
+  fp.batch = 4;
+  if (const char* ev = getenv("KTILER_FLOW_BATCH")) fp.batch = std::min(32, std::max(1, atoi(ev)));
+  fp.tb = ktflow::FTrace{P->tb.rec, P->tb.n, P->tb.cap};
+  fp.nroles = nroles;
+  fp.nnodes = nn;
+  // watchdog: 2^24 sleeping polls (seconds) before a trap
+  fp.spin_limit = 1ull << 24;
+  P->flow_node_role = node_role;
+  P->flow_slot_role = slot_role;
+  return KTILER_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -1806,7 +2092,7 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
   kt::Graph* G = kt::graph_of(gh);
   ktiler_status s = G->finalize();
   if (s) return s;
-  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_GRAPH_WAVE)
+  if (pol->exec_mode < KTILER_EXEC_STREAM || pol->exec_mode > KTILER_EXEC_FLOW)
     return fail(KTILER_E_INVALID, "unknown exec_mode");
   if (cache_bytes == 0) {
     int dev = 0, l2 = 0;
@@ -1841,6 +2127,37 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
 }
 
 void ktiler_plan_destroy(ktiler_plan_t p) { delete p; }
+
+ktiler_status ktiler_plan_set_flow_roles(ktiler_plan_t p, const int32_t* node_role, int32_t n_nodes,
+                                         const int32_t* slot_role, int32_t n_slots) {
+  if (!p) return fail(KTILER_E_INVALID, "NULL plan");
+  if (p->pol.exec_mode != KTILER_EXEC_FLOW) return fail(KTILER_E_STATE, "roles apply to KTILER_EXEC_FLOW plans");
+  if (p->executed || p->device >= 0) return fail(KTILER_E_STATE, "roles must be set before the first execute");
+  if (n_nodes == 0 && n_slots == 0) {
+    p->flow_node_role.clear();
+    p->flow_slot_role.clear();
+    return KTILER_OK;
+  }
+  if (!node_role || !slot_role || n_nodes != (int32_t)p->g.nodes.size())
+    return fail(KTILER_E_INVALID, "FLOW roles: one role per node");
+  if (n_slots < 2 || n_slots > 5) return fail(KTILER_E_INVALID, "FLOW roles: 2..5 slots per SM");
+  int32_t nroles = 0;
+  for (int32_t i = 0; i < n_nodes; ++i) {
+    if (node_role[i] < 0 || node_role[i] >= ktflow::FMAX_ROLES) return fail(KTILER_E_INVALID, "FLOW roles: role out of range");
+    nroles = std::max(nroles, node_role[i] + 1);
+  }
+  std::vector<int> served(nroles, 0);
+  for (int32_t i = 0; i < n_slots; ++i) {
+    if (slot_role[i] < 0 || slot_role[i] >= nroles) return fail(KTILER_E_INVALID, "FLOW roles: slot role out of range");
+    served[slot_role[i]] = 1;
+  }
+  for (int32_t r = 0; r < nroles; ++r)
+    if (!served[r]) return fail(KTILER_E_INVALID, "FLOW roles: every role needs a slot");
+  p->flow_node_role.assign(node_role, node_role + n_nodes);
+  p->flow_slot_role.assign(slot_role, slot_role + n_slots);
+  kt::clear_error();
+  return KTILER_OK;
+}
 
 ktiler_status ktiler_plan_num_subkernels(ktiler_plan_t p, int64_t* n) {
   if (!p || !n) return fail(KTILER_E_INVALID, "NULL argument");
@@ -1878,7 +2195,7 @@ ktiler_status ktiler_plan_get_stats(ktiler_plan_t p, ktiler_plan_stats* out) {
   std::memset(out, 0, sizeof(*out));
   out->n_subkernels = (int64_t)p->s.subs.size();
   out->n_fragments = p->s.nfrag;
-  out->n_launches = p->pol.exec_mode == KTILER_EXEC_PERSISTENT
+  out->n_launches = (p->pol.exec_mode == KTILER_EXEC_PERSISTENT || p->pol.exec_mode == KTILER_EXEC_FLOW)
                         ? 1
                         : (int64_t)(p->launches.size() + p->dag_disc.size()) +
                               (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN ? 2 : 0);
@@ -1894,8 +2211,16 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
   if (!p) return fail(KTILER_E_INVALID, "NULL plan");
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e;
+  if (p->sticky) return fail(KTILER_E_STATE, "plan setup failed at its first execute; destroy and re-plan");
   if (p->device < 0) {
-    if ((e = cudaGetDevice(&p->device)) != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    // the plan is marked ready only once every setup step succeeded; a failure is sticky
+    // (a half-initialised PERSISTENT / CHAIN / halo-counter state must never launch)
+    auto setup_failed = [&](ktiler_status s) {
+      p->sticky = s;
+      p->device = -1;
+      return s;
+    };
+    if ((e = cudaGetDevice(&p->device)) != cudaSuccess) return setup_failed(cuda_fail(e, "cudaGetDevice"));
     if (p->pol.exec_mode == KTILER_EXEC_GRAPH_PERSIST_L2) {
       int maxp = 0;
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, p->device);
@@ -1903,19 +2228,22 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     }
     if (p->pol.exec_mode == KTILER_EXEC_PERSISTENT) {
       ktiler_status s = setup_persistent(p);
-      if (s) return s;
+      if (s) return setup_failed(s);
       p->pp.tb = p->tb;
+    } else if (p->pol.exec_mode == KTILER_EXEC_FLOW) {
+      ktiler_status s = setup_flow(p);
+      if (s) return setup_failed(s);
     } else {
       for (auto& L : p->launches)
         if (L.node >= 0 && L.n->op != KTILER_OP_CUSTOM && !L.n->scalar && L.kp.stage_bytes)
           L.kp.use_tmap = make_tmap(p->g, *L.n, &L.kp.tmap, &L.kp.box_bytes);
       {
         ktiler_status s = setup_halo_discard(p);
-        if (s) return s;
+        if (s) return setup_failed(s);
       }
       if (p->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN) {
         ktiler_status s = setup_chain(p);
-        if (s) return s;
+        if (s) return setup_failed(s);
       }
       int64_t lid = 0;
       for (auto& L : p->launches) {
@@ -1980,6 +2308,21 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
       cfg.dynamicSmemBytes = (size_t)p->psmem;
       cfg.stream = st;
       if ((e = cudaLaunchKernelEx(&cfg, p->pfn, p->pp)) != cudaSuccess) return cuda_fail(e, "persistent launch");
+      break;
+    }
+    case KTILER_EXEC_FLOW: {
+      // cooperative: every role's CTAs are guaranteed co-resident (flow.cuh, deadlock freedom)
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3((unsigned)p->fctas);
+      cfg.blockDim = dim3((unsigned)p->fthreads);
+      cfg.dynamicSmemBytes = (size_t)p->fsmem;
+      cfg.stream = st;
+      cudaLaunchAttribute at[1];
+      at[0].id = cudaLaunchAttributeCooperative;
+      at[0].val.cooperative = 1;
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      if ((e = cudaLaunchKernelEx(&cfg, p->ffn, p->fp)) != cudaSuccess) return cuda_fail(e, "flow launch");
       break;
     }
   }

@@ -155,6 +155,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t* m, unsigned parity) {
       : "memory");
 }
 
+// non-blocking probe of an mbarrier phase (parity)
+__device__ __forceinline__ bool mbar_test(uint64_t* m, unsigned parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred P;\n mbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n selp.u32 %0, 1, 0, P;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(m)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
 // Staged window of op's input for tile t: rows [ry0, ry0+nr) (clamped to the image for the
 // stencils), byte columns [xb0, xb0 + stride) (negative / beyond-width columns of the
 // stencils are filled by stage_fix with the replicate rule).

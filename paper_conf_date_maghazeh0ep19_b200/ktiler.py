@@ -19,12 +19,13 @@ BUF_INTERNAL = 1
 READ, WRITE = 1, 2
 OP_GRAY, OP_BLUR5, OP_DOWN2, OP_SOBEL3, OP_THRESH, OP_CUSTOM, OP_JACOBI, OP_GAUSS_F32 = range(8)
 FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1, FRAG_CHAIN = range(6)
-EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE = range(7)
+EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE, \
+    EXEC_FLOW = range(8)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL, PF_RESIDENT_BUDGET, PF_CONSUMER_DISCARD, PF_HALO_DISCARD = 1, 2, 4, 8, 16, 32
 
 EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
               "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG, "chain": EXEC_GRAPH_CHAIN,
-              "wave": EXEC_GRAPH_WAVE}
+              "wave": EXEC_GRAPH_WAVE, "flow": EXEC_FLOW}
 FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCED, "none": FRAG_NONE,
               "alg1": FRAG_ALG1, "chain": FRAG_CHAIN}
 
@@ -104,7 +105,8 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_plan_num_subkernels", "ktiler_plan_num_fragments", "ktiler_plan_get_subkernel",
            "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
            "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest", "ktiler_plan_num_clusters",
-           "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint"]
+           "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint",
+           "ktiler_plan_set_flow_roles"]
 
 _LIB = None
 
@@ -147,6 +149,7 @@ def lib() -> ctypes.CDLL:
         "ktiler_set_perf_table": ([vp, i32, i32, P(i64), P(ctypes.c_double), P(ctypes.c_double)], st),
         "ktiler_calibrate": ([vp, i32, i32, P(i64), i32, P(ctypes.c_double), P(ctypes.c_double)], st),
         "ktiler_discover_footprint": ([vp, i32, i32, i32, i32, i32, ctypes.c_uint64, P(FootprintRec), i32, P(i32)], st),
+        "ktiler_plan_set_flow_roles": ([vp, P(i32), i32, P(i32), i32], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -355,6 +358,14 @@ class Plan:
             out.append((sub.value, node.value, tiles.value))
             i += 1
         return out
+
+    def set_flow_roles(self, node_role, slot_role) -> None:
+        """KTILER_EXEC_FLOW roles (include/ktiler.h ktiler_plan_set_flow_roles): node_role[v]
+        = role of node v, slot_role[s] = role of the s-th CTA on every SM (2..5 slots);
+        empty lists restore the automatic roles.  Before the first execute."""
+        nr, sr = list(node_role), list(slot_role)
+        _check(lib().ktiler_plan_set_flow_roles(self._h, (ctypes.c_int32 * max(1, len(nr)))(*nr), len(nr),
+                                                (ctypes.c_int32 * max(1, len(sr)))(*sr), len(sr)))
 
     def execute(self, stream: int = 0) -> None:
         _check(lib().ktiler_execute(self._h, ctypes.c_void_p(stream)))

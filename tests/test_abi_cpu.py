@@ -247,3 +247,49 @@ def test_gauss_f32_params(K):
                      struct.pack("f", 1.0))
     g.add_kernel(K.OP_GAUSS_F32, (1, 2, 1), (64, 1, 1), [acc(a, K.READ, 64, 16, 3), acc(b, K.WRITE, 64, 16)],
                  struct.pack("f", 1.0))
+
+
+def _crop_pair(W=256, H=256):
+    """A graph that triggers reading A16b: A = gray (in -> intm, 32x8 tiles)
+    and B = a 2x2-mean consumer whose output is only the TOP HALF of down2's (W/2 x H/4),
+    so the bottom half of A's blocks feed no leaf block.  Oracle: B is down2 on the cropped
+    output (its tracer records exactly which intm rows B reads).  C++: B is an OP_CUSTOM node
+    declaring the same affine footprint (read 2x its 64x1 tile, write the tile), planned
+    only (never launched on CPU)."""
+    og = O.OGraph()
+    og.add_buf("in", W, H, 1, 3, external=True)
+    og.add_buf("intm", W, H, 1, 1)
+    og.add_buf("out", W // 2, H // 4, 1, 1)
+    og.add_node("A", O.GRAY, "in", "intm", 32, 8)
+    og.add_node("B", O.DOWN2, "intm", "out", 64, 1)
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler as K
+    bases = og.bases()
+    g = K.Graph()
+    bi = g.add_buffer(bases["in"], W, H, 3)
+    bm = g.add_buffer(bases["intm"], W, H, 1, internal=True)
+    bo = g.add_buffer(bases["out"], W // 2, H // 4, 1)
+    a = g.add_kernel(K.OP_GRAY, (W // 32, H // 8, 1), (32, 8, 1),
+                     [dict(buf=bi, mode=K.READ, ax=32, ay=8), dict(buf=bm, mode=K.WRITE, ax=32, ay=8)])
+    b = g.add_kernel(K.OP_CUSTOM, (W // 2 // 64, H // 4, 1), (64, 1, 1),
+                     [dict(buf=bm, mode=K.READ, ax=128, ay=2), dict(buf=bo, mode=K.WRITE, ax=64, ay=1)],
+                     launch=lambda *args: None)
+    g.add_edge(a, b, bm, 1.0)
+    return og, g
+
+
+@pytest.mark.parametrize("lines", [36, 68, 136, 1000])
+def test_planner_equals_oracle_a16b(K, lines):
+    """Reading A16b (blocks no leaf block depends on are picked as bottom blocks, last node
+    first, once every leaf block is taken) is exercised: C++ == O-8 sub-kernel by sub-kernel,
+    and the schedule has fragments of A blocks that no B block reads."""
+    og, g = _crop_pair()
+    tr = O.trace(og)
+    ref = O.cluster_tile(og, tr, lines * 128)
+    plan = g.plan(lines * 128, kind="budget", exec_mode="stream")
+    ours = _blocks_by_sub(plan)
+    assert [(n, b, f) for n, b, f in ours] == [(n, sorted(b), f) for (n, b), f in zip(ref.seq, ref.frag)]
+    assert not O.validate_schedule(og, tr, [(n, b) for n, b, _ in ours], lines * 128, [f for _, _, f in ours])
+    b_frags = {f for n, _, f in ours if n == 1}
+    orphan = [f for n, b, f in ours if n == 0 and f not in b_frags]
+    assert orphan, "A16b not triggered"
+    assert all(by >= 16 for n, b, f in ours if f in orphan for (_, by, _) in b)

@@ -143,15 +143,31 @@ def test_b200_geometry_tiled(mode):
     assert _eq(out["mask"], ref["mask"])
 
 
-def test_replay_is_idempotent():
-    """A plan executes many times (GRAPH replays, persistent epochs) with identical output."""
+REPLAY = [("graph", dict(discard=True)), ("persistent", dict(discard=True)), ("chain", dict(discard=True)),
+          ("wave", dict(discard=True)),
+          # bench.py's executor and its discard variants: the halo-reader counters persist
+          # across executes and must reset themselves
+          ("dag", dict(window=2, resident_budget=True, consumer_discard=True)),
+          ("dag", dict(window=2, consumer_discard=True, halo_discard=True)),
+          ("dag", dict(window=2, consumer_discard=True, halo_discard=True, discard=True)),
+          ("flow", dict(kind="rows", rows=1, consumer_discard=True)),
+          ("flow", dict(kind="rows", rows=2, consumer_discard=True, window=3))]
+
+
+@pytest.mark.parametrize("mode,pol", REPLAY, ids=[f"{m}-{'-'.join(sorted(k))}" for m, k in REPLAY])
+def test_replay_is_idempotent(mode, pol):
+    """A plan executes many times (GRAPH replays, persistent epochs, per-execute counters)
+    with identical output, alternating inputs."""
     from paper_conf_date_maghazeh0ep19_b200 import Pipeline
     W, H, F = 1024, 128, 1
-    for mode in ("graph", "persistent", "chain", "wave"):
+    pol = dict(pol)
+    kind = pol.pop("kind", "budget")
+    if True:
         p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
         a = synth.uniform(1, W, H, F)
         b = synth.scene(2, W, H, F)
-        p.plan(100 * 1024, kind="budget", exec_mode=mode, discard=True)
+        plan = p.plan(100 * 1024, kind=kind, exec_mode=mode, **pol)
+        assert plan.num_fragments() > 1
         for it in range(6):
             x = a if it % 2 == 0 else b
             p.view("rgb").copy_(torch.from_numpy(x))

@@ -145,3 +145,32 @@ def test_planner_alg1_equals_oracle(K, tables, budget):
                         for z in range(z0, z1) for y in range(y0, y1) for x in range(x0, x1))
         got_s.append((sk["node"], blocks, sk["cluster"]))
     assert got_s == [(v, sorted(b), c) for v, b, c in want_s]
+
+
+@pytest.mark.parametrize("rows", [1, 2, 3, 5])
+@pytest.mark.parametrize("budget", [6000, 20000])
+def test_planner_frag_chain_equals_oracle(K, rows, budget):
+    """KTILER_FRAG_CHAIN (DESIGN A40): the fixed partition into consecutive groups of `rows`
+    nodes (topological order), each group tiled by the literal Alg. 2 (O-8 with cluster=the
+    group) under the budget and the groups run one after another.  C++ == O-8 per cluster,
+    sub-kernel by sub-kernel (FRAG_CHAIN had no tests)."""
+    W, H, F = 64, 96, 2
+    og, tr, p = _both(W, H, F)
+    want, inf = [], False
+    for c, lo in enumerate(range(0, 5, rows)):
+        t = O.cluster_tile(og, tr, budget, cluster=list(range(lo, min(5, lo + rows))))
+        inf |= t.cost == O.INF
+        want += [(v, sorted(b), c) for (v, b) in t.seq]
+    if inf:  # a group's leaf closure exceeds the budget: the paper's infinity (A18)
+        with pytest.raises(K.KtilerError) as e:
+            p.graph.plan(budget, kind="chain", rows=rows, exec_mode="stream")
+        assert e.value.status == K.E_UNTILEABLE
+        return
+    plan = p.graph.plan(budget, kind="chain", rows=rows, exec_mode="stream")
+    got = []
+    for sk in plan.subkernels():
+        blocks = sorted((x, y, z) for (x0, y0, z0, x1, y1, z1) in sk["rects"]
+                        for z in range(z0, z1) for y in range(y0, y1) for x in range(x0, x1))
+        got.append((sk["node"], blocks, sk["cluster"]))
+    assert got == want
+    assert [c for c, _ in plan.clusters()] == [list(range(lo, min(5, lo + rows))) for lo in range(0, 5, rows)]

@@ -272,3 +272,54 @@ def test_lru_model_tiling_reduces_dram(small_pipe):
     assert td["write_incl_tail"] < ti["write_incl_tail"]
     compulsory = g.bufs["rgb"].nbytes + g.bufs["mask"].nbytes
     assert td["read"] + td["write_incl_tail"] >= compulsory
+
+
+def _lru_tiny():
+    """Fig. 1's A -> B on a 128 x 2 image: A tiles 128 x 1 (2 blocks, one image row each),
+    B tile 64 x 1 (1 block, reads both intm rows).  Every buffer row is a whole number of
+    128-B lines at 128-B-aligned bases: in rows are 3 lines each (384 B),
+    intm rows 1 line each, out 1 line (64 B)."""
+    g = O.motivational_graph(W=128, H=2, a_tile=(128, 1), b_tile=(64, 1))
+    return g, O.trace(g)
+
+
+def test_lru_model_exact_hand_trace():
+    """O-12 pinned to a hand-worked trace (O-12 was parity-unpinned).  Untiled
+    order A0, A1, B0; each block reads its lines in ascending order, then writes.
+
+    cache 4 lines:
+      A0  miss in0 in1 in2 (rd 3)               LRU [in0 in1 in2]; write i0* -> [in0 in1 in2 i0*]
+      A1  miss in3 in4 in5 (rd 6), evicting in0 in1 in2 (clean)   -> [i0* in3 in4 in5]
+          write i1*: evicts i0* DIRTY (wr 1)                        -> [in3 in4 in5 i1*]
+      B0  i0 misses again (rd 7), evicts in3; i1 hits               -> [in4 in5 i0 i1*]
+          write o0*: evicts in4                                     -> [in5 i0 i1* o0*]
+      => read 7 lines, write 1 line, dirty tail {i1, o0} = 2 lines.
+      With the discard of dead intermediates, i0 and i1 die after B0 (their last reader):
+      the write-back of i0 already happened, i1's never does -> tail {o0} = 1 line.
+    cache 64 lines (everything fits): read 6, write 0, tail {i0, i1, o0} = 3 lines;
+      with discard: tail {o0} = 1 line."""
+    g, tr = _lru_tiny()
+    L = 128
+    s = O.untiled_schedule(g)
+    assert O.lru_dram_bytes(g, tr, s, 4 * L) == {"read": 7 * L, "write": 1 * L, "write_incl_tail": 3 * L}
+    assert O.lru_dram_bytes(g, tr, s, 4 * L, discard_dead=True) == {"read": 7 * L, "write": 1 * L,
+                                                                     "write_incl_tail": 2 * L}
+    assert O.lru_dram_bytes(g, tr, s, 64 * L) == {"read": 6 * L, "write": 0, "write_incl_tail": 3 * L}
+    assert O.lru_dram_bytes(g, tr, s, 64 * L, discard_dead=True) == {"read": 6 * L, "write": 0,
+                                                                      "write_incl_tail": 1 * L}
+
+
+def test_lru_model_exact_reordered_trace():
+    """Same graph, cache 4 lines, order A1, A0, B0 (another valid order):
+      A1  miss in3 in4 in5 (rd 3); write i1*       -> [in3 in4 in5 i1*]
+      A0  miss in0 (rd 4) evicts in3; in1 evicts in4; in2 evicts in5 (all clean)
+                                                   -> [i1* in0 in1 in2]
+          write i0*: evicts i1* DIRTY (wr 1)       -> [in0 in1 in2 i0*]
+      B0  i0 hits; i1 misses (the 7th line read), evicts in0
+                                                   -> [in1 in2 i0* i1]
+          write o0*: evicts in1                    -> [in2 i0* i1 o0*]
+      => read 7, write 1, dirty tail {i0, o0} = 2 lines (i1 was re-read clean)."""
+    g, tr = _lru_tiny()
+    L = 128
+    s = [(0, [(0, 1, 0)]), (0, [(0, 0, 0)]), (1, [(0, 0, 0)])]
+    assert O.lru_dram_bytes(g, tr, s, 4 * L) == {"read": 7 * L, "write": 1 * L, "write_incl_tail": 3 * L}

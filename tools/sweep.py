@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--configs", default="default", help="default | json list of plan kwargs")
     ap.add_argument("--geom", default="", help='json {op: [tile_w, tile_h, threads]} overriding B200_GEOMETRY')
+    ap.add_argument("--check", action="store_true", help="compare every config's mask with the untiled graph's")
     args = ap.parse_args()
     import torch
 
@@ -49,9 +50,23 @@ def main():
     else:
         cfgs = json.loads(args.configs)
     pix = args.W * args.H * args.F
+    ref = None
+    if args.check:
+        pl = p.b.g.plan(0, kind="none", exec_mode="graph")
+        pl.execute(s.cuda_stream)
+        torch.cuda.synchronize()
+        ref = p.view("mask").clone()
+        del pl
     for c in cfgs:
         try:
+            c = dict(c)
+            roles = c.pop("roles", None)
             pl = p.b.g.plan(0, **c)
+            if roles:
+                pl.set_flow_roles(roles[0], roles[1])
+            if ref is not None:
+                p.view("mask").fill_(77)
+            c["roles"] = roles
             for _ in range(2):
                 pl.execute(s.cuda_stream)
             ts = []
@@ -64,9 +79,13 @@ def main():
                 ts.append(e0.elapsed_time(e1))
             ms = statistics.median(ts)
             st = pl.stats()
+            ok = None
+            if ref is not None:
+                torch.cuda.synchronize()
+                ok = bool(torch.equal(p.view("mask"), ref))
             print(json.dumps({"cfg": c, "geom": args.geom or "default", "minb": os.environ.get("KTILER_PERSIST_MINB", "default"), "ms": round(ms, 4),
                               "Mpix/s": round(pix / ms / 1e3, 1), "fragments": st["n_fragments"],
-                              "launches": st["n_launches"]}), flush=True)
+                              "launches": st["n_launches"], "match": ok}), flush=True)
             del pl
         except Exception as e:
             print(json.dumps({"cfg": c, "error": str(e)}), flush=True)
