@@ -9,7 +9,8 @@ sharding with no data-path collective: by default the one 64-frame batch is spli
 contiguous frame ranges (64/N frames per GPU, "scaling": "strong"; frames.frame_range);
 --scaling weak gives every rank a whole batch of its own instead.  Workload
 ``strip_65536`` (configs[4]) splits one 65536x65536 image into row strips whose 4 halo
-rows per side move over NCCL send/recv before each step.
+rows per side move over NCCL send/recv (libktiler's ktiler_halo_exchange, captured into
+the plan's graph ahead of the schedule) in each step.
 
 A step = one ktiler_execute of the plan over the rank's whole share (all five kernels).
 Timing: W untimed warm-up steps, then exactly K steps bracketed by a barrier + cuda
@@ -61,7 +62,7 @@ def parse(argv=None):
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ktiler", choices=["ktiler", "reference"])
     ap.add_argument("--workload", default="batch64_8k", choices=sorted(WORKLOADS))
-    ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave"])
+    ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave", "flow"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
     ap.add_argument("--l2-fraction", type=float, default=0.85)
@@ -372,9 +373,16 @@ def main():
             step_ms[:] = [(e0 if k == 0 else marks[k - 1]).elapsed_time(marks[k]) for k in range(steps)]
         return FR.max_over_ranks(ms, world, device="cuda")
 
+    comm = None
+    if sp is not None and world > 1:
+        # the strip halo exchange runs inside libktiler (ncclSend/ncclRecv in one group),
+        # captured into the plan's graph ahead of the schedule: one execute per step
+        from paper_conf_date_maghazeh0ep19_b200 import strips as SM
+        comm = SM.nccl_comm(world, rank)
+        sp.register(comm)
+        plan.attach_halo(comm, rank, SM.HALO_ROWS)
+
     def step():
-        if sp is not None and world > 1:
-            sp.exchange()
         plan.execute(s)
 
     clk = Clocks(local)
@@ -434,8 +442,9 @@ def main():
                                   "floor_ms": floor_ms, "frac": floor_ms / ms, "source": l2["source"]}
     if not args.no_untiled:
         un = p.b.g.plan(0, kind="none", exec_mode="graph", discard=False)
-        ms_un = timed(lambda: (sp.exchange() if sp is not None and world > 1 else None, un.execute(s)),
-                      max(3, args.steps // 2), 2)
+        if comm is not None:
+            un.attach_halo(comm, rank, SM.HALO_ROWS)
+        ms_un = timed(lambda: un.execute(s), max(3, args.steps // 2), 2)
         line["untiled"] = {"value": pix / (ms_un / 1000) / 1e6, "ms_per_step": ms_un,
                            "tiled_speedup": ms_un / ms,
                            "achieved_gbs": 9.75 * pix / (ms_un / 1000) / 1e9,

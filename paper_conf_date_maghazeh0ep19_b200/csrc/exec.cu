@@ -854,6 +854,9 @@ struct ktiler_plan_s {
   void (*ffn)(ktflow::FParams) = nullptr;
   int fctas = 0, fthreads = 0, fsmem = 0;
   void* fmem = nullptr;
+  // ktiler_plan_attach_halo: the strip exchange run before the schedule in every execute
+  ktiler_comm_t halo_comm = nullptr;
+  int32_t halo_rank = 0, halo_rows = 0;
   // GRAPH_CHAIN state: one device block (epoch | flags | dcount | prefix) and the tail
   void* cmem = nullptr;
   std::vector<void*> hmem;  // halo-reader counters of consumer discards
@@ -948,6 +951,7 @@ void build_launches(ktiler_plan_s* P) {
       Launch L;
       L.node = sk.node;
       L.n = const_cast<kt::Node*>(&n);
+      L.sub = (int)si;  // GRAPH_DAG adds launches by sub-kernel
       for (auto& r : sk.rects) {
         int32_t v[6] = {r.x0, r.y0, r.z0, r.x1, r.y1, r.z1};
         L.crects.insert(L.crects.end(), v, v + 6);
@@ -1288,6 +1292,26 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   static const bool pdl_all = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "all");
   auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, const std::vector<uint8_t>& prog,
                       cudaGraphNode_t* node) -> ktiler_status {
+    if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
+      // a user kernel (KTILER_OP_CUSTOM): its launch callback, stream-captured once for this
+      // sub-kernel's rect list, becomes a child graph node with the same dependency edges
+      cudaStream_t cs;
+      cudaError_t ce = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+      if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamCreate");
+      if ((ce = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal)) != cudaSuccess) {
+        cudaStreamDestroy(cs);
+        return cuda_fail(ce, "cudaStreamBeginCapture (custom)");
+      }
+      L.n->launch(L.n->user, L.crects.data(), (int32_t)(L.crects.size() / 6), (void*)cs);
+      cudaGraph_t cg = nullptr;
+      ce = cudaStreamEndCapture(cs, &cg);
+      cudaStreamDestroy(cs);
+      if (ce != cudaSuccess) return cuda_fail(ce, "cudaStreamEndCapture (custom launch callback)");
+      ce = cudaGraphAddChildGraphNode(node, gr, deps.data(), deps.size(), cg);
+      cudaGraphDestroy(cg);
+      if (ce != cudaSuccess) return cuda_fail(ce, "cudaGraphAddChildGraphNode (custom)");
+      return KTILER_OK;
+    }
     kfn_t fn = launch_fn(L);
     int64_t grid = 0;
     ktiler_status ps = prep_launch(P, L, fn, &grid);
@@ -1819,13 +1843,13 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
 typedef void (*ffn_t)(ktflow::FParams);
 ffn_t flow_variant(int k) {
   switch (k) {
-    case 2: return ktflow::flow_kernel<4, 2>;
+    case 2: return ktflow::flow_kernel<8, 2>;
     case 3: return ktflow::flow_kernel<4, 3>;
     case 5: return ktflow::flow_kernel<3, 5>;
     default: return ktflow::flow_kernel<4, 4>;
   }
 }
-int flow_threads(int k) { return k == 5 ? 128 : 160; }
+int flow_threads(int k) { return k == 5 ? 128 : (k == 2 ? 288 : 160); }
 
 // Automatic roles: every node its own role when the slots allow, the slots shared out in
 // proportion to each node's staged + written bytes (at least one each); otherwise
@@ -2072,6 +2096,9 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
   fp.nslots_sm = K;
   fp.batch = 4;
   if (const char* ev = getenv("KTILER_FLOW_BATCH")) fp.batch = std::min(32, std::max(1, atoi(ev)));
+  fp.pending = 16;
+  if (const char* ev = getenv("KTILER_FLOW_PENDING")) fp.pending = std::min(32, std::max(1, atoi(ev)));
+  fp.pending = std::max(fp.pending, fp.batch);
   fp.tb = ktflow::FTrace{P->tb.rec, P->tb.n, P->tb.cap};
   fp.nroles = nroles;
   fp.nnodes = nn;
@@ -2079,6 +2106,41 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
   fp.spin_limit = 1ull << 24;
   P->flow_node_role = node_role;
   P->flow_slot_role = slot_role;
+  return KTILER_OK;
+}
+
+
+// GRAPH_DAG / GRAPH_WAVE with an attached strip exchange: the exchange, stream-captured into
+// a child graph, becomes a root every former root of the DAG depends on — one graph per
+// execute, exchange then schedule.
+ktiler_status prepend_halo(ktiler_plan_s* P, cudaGraph_t gr) {
+  size_t nroot = 0;
+  cudaError_t e = cudaGraphGetRootNodes(gr, nullptr, &nroot);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGraphGetRootNodes");
+  std::vector<cudaGraphNode_t> roots(nroot);
+  if (nroot && (e = cudaGraphGetRootNodes(gr, roots.data(), &nroot)) != cudaSuccess)
+    return cuda_fail(e, "cudaGraphGetRootNodes");
+  cudaStream_t cs;
+  if ((e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking)) != cudaSuccess) return cuda_fail(e, "cudaStreamCreate");
+  if ((e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal)) != cudaSuccess) {
+    cudaStreamDestroy(cs);
+    return cuda_fail(e, "cudaStreamBeginCapture");
+  }
+  ktiler_status s = kt::halo_exchange(P->halo_comm, P->halo_rank, P->halo_rows, cs);
+  cudaGraph_t hx = nullptr;
+  cudaError_t e2 = cudaStreamEndCapture(cs, &hx);
+  cudaStreamDestroy(cs);
+  if (s) {
+    if (hx) cudaGraphDestroy(hx);
+    return s;
+  }
+  if (e2 != cudaSuccess) return cuda_fail(e2, "cudaStreamEndCapture (halo)");
+  cudaGraphNode_t xn;
+  e = cudaGraphAddChildGraphNode(&xn, gr, nullptr, 0, hx);
+  cudaGraphDestroy(hx);  // the node holds a copy
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGraphAddChildGraphNode (halo)");
+  for (cudaGraphNode_t r : roots)
+    if ((e = cudaGraphAddDependencies(gr, &xn, &r, 1)) != cudaSuccess) return cuda_fail(e, "cudaGraphAddDependencies");
   return KTILER_OK;
 }
 
@@ -2127,6 +2189,16 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
 }
 
 void ktiler_plan_destroy(ktiler_plan_t p) { delete p; }
+
+ktiler_status ktiler_plan_attach_halo(ktiler_plan_t p, ktiler_comm_t c, int32_t rank, int32_t halo_rows) {
+  if (!p || !c || rank < 0 || halo_rows < 0) return fail(KTILER_E_INVALID, "bad argument");
+  if (p->executed || p->device >= 0) return fail(KTILER_E_STATE, "attach the halo exchange before the first execute");
+  p->halo_comm = c;
+  p->halo_rank = rank;
+  p->halo_rows = halo_rows;
+  kt::clear_error();
+  return KTILER_OK;
+}
 
 ktiler_status ktiler_plan_set_flow_roles(ktiler_plan_t p, const int32_t* node_role, int32_t n_nodes,
                                          const int32_t* slot_role, int32_t n_slots) {
@@ -2257,6 +2329,11 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     }
   }
   p->executed = true;
+  if (p->halo_comm && (p->pol.exec_mode == KTILER_EXEC_STREAM || p->pol.exec_mode == KTILER_EXEC_PERSISTENT ||
+                       p->pol.exec_mode == KTILER_EXEC_FLOW)) {
+    ktiler_status hs = kt::halo_exchange(p->halo_comm, p->halo_rank, p->halo_rows, st);
+    if (hs) return hs;
+  }
   switch (p->pol.exec_mode) {
     case KTILER_EXEC_STREAM: {
       ktiler_status s = enqueue(p, st);
@@ -2266,10 +2343,13 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
     case KTILER_EXEC_GRAPH_DAG:
     case KTILER_EXEC_GRAPH_WAVE: {
       if (!p->exec) {
-        if (p->has_custom) return fail(KTILER_E_UNSUPPORTED, "GRAPH_DAG / GRAPH_WAVE run built-in ops only");
         cudaGraph_t gr = nullptr;
         ktiler_status s = build_dag(p, &gr);
         if (s) return s;
+        if (p->halo_comm && (s = prepend_halo(p, gr))) {
+          cudaGraphDestroy(gr);
+          return s;
+        }
         p->graph = gr;
         if ((e = cudaGraphInstantiate(&p->exec, gr, 0)) != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
       }
@@ -2286,7 +2366,8 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
           cudaStreamDestroy(cs);
           return cuda_fail(e, "cudaStreamBeginCapture");
         }
-        ktiler_status s = enqueue(p, cs);
+        ktiler_status s = p->halo_comm ? kt::halo_exchange(p->halo_comm, p->halo_rank, p->halo_rows, cs) : KTILER_OK;
+        if (!s) s = enqueue(p, cs);
         cudaGraph_t gr = nullptr;
         cudaError_t e2 = cudaStreamEndCapture(cs, &gr);
         cudaStreamDestroy(cs);

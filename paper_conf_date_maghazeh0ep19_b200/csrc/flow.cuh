@@ -100,7 +100,7 @@ struct FParams {
   int32_t nnodes;
   uint64_t spin_limit;        // watchdog: polls before __trap (0 = none)
   int32_t batch;              // tickets per claim (1..32)
-  int32_t pad;
+  int32_t pending;            // claimed, unstaged tickets a producer warp may hold (batch..32)
   FTrace tb;                  // rec == NULL: tracing off
 };
 
@@ -275,14 +275,20 @@ __global__ void __launch_bounds__(32 * (NW + 1), MINB) flow_kernel(const __grid_
   const int64_t stage_bytes = p.role_stage[role];
   if (warp == NW) {
     // ------------------------------ producer warp ------------------------------
+    // Lane j holds pending ticket j (claimed, not staged yet; bit j of `left`) and its
+    // claim position `pos`.  Batches of `batch` tickets are claimed whenever the pending set
+    // has room (at most p.pending), so a CTA whose oldest tickets wait on dependencies
+    // still finds ready work further on; ready tickets are staged oldest first.
     const uint64_t* tk = p.tickets + p.role_off[role];
     const unsigned ntk = (unsigned)(p.role_off[role + 1] - p.role_off[role]);
     const unsigned B = (unsigned)p.batch;
+    const int cap = p.pending;
     unsigned next = 0;  // lane 0: base of the batch claimed in advance
     if (lane == 0) next = atomicAdd(p.claim + role, B);
-    uint64_t mine = FLOW_STOP;  // lane j < qn: ticket j of the current batch
-    unsigned left = 0;          // tiles of the batch not staged yet
-    int k_iss = 0;              // tiles staged
+    uint64_t mine = FLOW_STOP;
+    unsigned pos = 0xFFFFFFFFu;  // claim position of this lane's ticket
+    unsigned left = 0, rdy = 0;  // pending tickets; those known ready
+    int k_iss = 0;               // tiles staged
     bool claims_done = false;
     uint64_t idle = 0, t_batch = 0;
     auto slot_free = [&](int k) {  // slot of tile k: its previous tile (k - S) computed
@@ -292,27 +298,37 @@ __global__ void __launch_bounds__(32 * (NW + 1), MINB) flow_kernel(const __grid_
     };
     for (;;) {
       bool progress = false;
-      if (left == 0 && !claims_done) {  // claim the next batch
+      // ---- claim while the pending set has room ----
+      while (!claims_done && __popc(left) + (int)B <= cap) {
         const unsigned base = __shfl_sync(0xFFFFFFFFu, next, 0);
         if (base >= ntk) {
           claims_done = true;
-        } else {
-          if (lane == 0) next = atomicAdd(p.claim + role, B);
-          const int qn = (int)min(B, ntk - base);
-          mine = lane < qn ? __ldg(tk + base + lane) : FLOW_STOP;
-          left = qn >= 32 ? 0xFFFFFFFFu : ((1u << qn) - 1u);
-          if (p.tb.rec) t_batch = fl_timer();
+          break;
         }
+        if (lane == 0) next = atomicAdd(p.claim + role, B);
+        const int qn = (int)min(B, ntk - base);
+        // the i-th free lane (i < qn) takes ticket base + i
+        const unsigned freem = ~left;
+        const int rank = __popc(freem & ((1u << lane) - 1u));
+        if (((freem >> lane) & 1u) && rank < qn) {
+          mine = __ldg(tk + base + rank);
+          pos = base + rank;
+        }
+        left |= __ballot_sync(0xFFFFFFFFu, ((freem >> lane) & 1u) && rank < qn);
+        if (p.tb.rec) t_batch = fl_timer();
         progress = true;
       }
       if (left) {
         if (slot_free(k_iss)) {
-          unsigned rdy = flow_ready(p, mine, left, epoch, lane) & left;
-          while (rdy) {
+          if ((rdy & left) != left) rdy |= flow_ready(p, mine, left & ~rdy, epoch, lane) & left;
+          while (rdy & left) {
             if (!slot_free(k_iss)) break;
-            const int j = __ffs(rdy) - 1;
-            rdy &= rdy - 1;
+            // oldest ready ticket
+            const bool cand = ((rdy & left) >> lane) & 1u;
+            const unsigned best = __reduce_min_sync(0xFFFFFFFFu, cand ? pos : 0xFFFFFFFFu);
+            const int j = __ffs(__ballot_sync(0xFFFFFFFFu, cand && pos == best)) - 1;
             left &= ~(1u << j);
+            rdy &= ~(1u << j);
             const uint64_t d = __shfl_sync(0xFFFFFFFFu, mine, j);
             if (lane == 0) {
               const FNode& nd = p.nodes[d >> 59];

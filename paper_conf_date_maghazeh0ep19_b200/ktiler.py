@@ -31,6 +31,7 @@ FRAG_KINDS = {"budget": FRAG_BUDGET, "rows": FRAG_ROWS, "balanced": FRAG_BALANCE
 
 
 SELFTEST_SQRT = 0
+COMM_NCCL, COMM_LOOPBACK = 0, 1
 
 
 def selftest(which: int = SELFTEST_SQRT) -> int:
@@ -94,6 +95,11 @@ class TraceRecord(ctypes.Structure):
                 ("t0_ns", ctypes.c_uint64), ("t1_ns", ctypes.c_uint64)]
 
 
+class Strip(ctypes.Structure):
+    _fields_ = [("base", ctypes.c_void_p), ("pitch_bytes", ctypes.c_int64), ("row_bytes", ctypes.c_int64),
+                ("o0", ctypes.c_int64), ("o1", ctypes.c_int64), ("e0", ctypes.c_int64), ("e1", ctypes.c_int64)]
+
+
 class HostCopy(ctypes.Structure):
     _fields_ = [("buf_id", ctypes.c_int32), ("pad", ctypes.c_int32), ("host", ctypes.c_void_p),
                 ("frame0", ctypes.c_int64), ("frames", ctypes.c_int64)]
@@ -106,7 +112,9 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_plan_get_stats", "ktiler_execute", "ktiler_execute_host", "ktiler_trace_enable",
            "ktiler_trace_read", "ktiler_plan_get_launch", "ktiler_selftest", "ktiler_plan_num_clusters",
            "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint",
-           "ktiler_plan_set_flow_roles"]
+           "ktiler_plan_set_flow_roles", "ktiler_comm_unique_id", "ktiler_comm_init_nccl",
+           "ktiler_comm_init_loopback", "ktiler_comm_destroy", "ktiler_comm_register_strip", "ktiler_halo_exchange",
+           "ktiler_plan_attach_halo"]
 
 _LIB = None
 
@@ -150,6 +158,13 @@ def lib() -> ctypes.CDLL:
         "ktiler_calibrate": ([vp, i32, i32, P(i64), i32, P(ctypes.c_double), P(ctypes.c_double)], st),
         "ktiler_discover_footprint": ([vp, i32, i32, i32, i32, i32, ctypes.c_uint64, P(FootprintRec), i32, P(i32)], st),
         "ktiler_plan_set_flow_roles": ([vp, P(i32), i32, P(i32), i32], st),
+        "ktiler_comm_unique_id": ([P(ctypes.c_uint8)], st),
+        "ktiler_comm_init_nccl": ([P(ctypes.c_uint8), i32, i32, P(vp)], st),
+        "ktiler_comm_init_loopback": ([i32, P(vp)], st),
+        "ktiler_comm_destroy": ([vp], None),
+        "ktiler_comm_register_strip": ([vp, i32, P(Strip)], st),
+        "ktiler_halo_exchange": ([vp, i32, i32, vp], st),
+        "ktiler_plan_attach_halo": ([vp, vp, i32, i32], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -202,7 +217,11 @@ class Graph:
         _check(lib().ktiler_add_buffer(self._h, ctypes.byref(d), ctypes.byref(out)))
         return out.value
 
-    def add_kernel(self, op: int, grid, block, accesses, params: bytes | None = None, launch=None) -> int:
+    def add_kernel(self, op: int, grid, block, accesses, params: bytes | None = None, launch=None,
+                   user: int | None = None) -> int:
+        """launch (OP_CUSTOM): a Python callable, or the integer address of a C function with
+        the ktiler_launch_fn signature (a user's compiled kernel launcher); user: its
+        opaque pointer."""
         acc = (Access * len(accesses))()
         for i, a in enumerate(accesses):
             acc[i] = Access(a["buf"], a["mode"], a["ax"], a["ay"], a.get("ox", 0), a.get("oy", 0),
@@ -212,7 +231,7 @@ class Graph:
         if launch is not None:
             self._keep.append(fn)
         d = KernelDesc(op, (ctypes.c_uint32 * 3)(*grid), (ctypes.c_uint32 * 3)(*block), len(accesses), acc,
-                       ctypes.cast(pbuf, ctypes.c_void_p) if pbuf else None, len(params) if params else 0, fn, None)
+                       ctypes.cast(pbuf, ctypes.c_void_p) if pbuf else None, len(params) if params else 0, fn, user)
         out = ctypes.c_int32()
         _check(lib().ktiler_add_kernel(self._h, ctypes.byref(d), ctypes.byref(out)))
         return out.value
@@ -367,6 +386,12 @@ class Plan:
         _check(lib().ktiler_plan_set_flow_roles(self._h, (ctypes.c_int32 * max(1, len(nr)))(*nr), len(nr),
                                                 (ctypes.c_int32 * max(1, len(sr)))(*sr), len(sr)))
 
+    def attach_halo(self, comm: "Comm", rank: int, halo_rows: int) -> None:
+        """Run rank's strip exchange first in every execute, inside the plan's CUDA graph
+        (include/ktiler.h ktiler_plan_attach_halo).  Before the first execute."""
+        _check(lib().ktiler_plan_attach_halo(self._h, comm._h, rank, halo_rows))
+        self._comm_keep = comm
+
     def execute(self, stream: int = 0) -> None:
         _check(lib().ktiler_execute(self._h, ctypes.c_void_p(stream)))
 
@@ -375,3 +400,49 @@ class Plan:
         ci = (HostCopy * max(1, len(inputs)))(*[HostCopy(b, 0, p, f0, nf) for b, p, f0, nf in inputs])
         co = (HostCopy * max(1, len(outputs)))(*[HostCopy(b, 0, p, f0, nf) for b, p, f0, nf in outputs])
         _check(lib().ktiler_execute_host(self._h, ci, len(inputs), co, len(outputs), ctypes.c_void_p(stream)))
+
+
+def comm_unique_id() -> bytes:
+    """128 opaque bytes (an ncclUniqueId) for Comm.nccl, made on one rank."""
+    buf = (ctypes.c_uint8 * 128)()
+    _check(lib().ktiler_comm_unique_id(buf))
+    return bytes(buf)
+
+
+class Comm:
+    """Owning wrapper of a ktiler_comm_t (strip halo exchange, include/ktiler.h)."""
+
+    def __init__(self, h):
+        self._h = h
+
+    @classmethod
+    def nccl(cls, uid: bytes, nranks: int, rank: int) -> "Comm":
+        h = ctypes.c_void_p()
+        buf = (ctypes.c_uint8 * 128)(*uid)
+        _check(lib().ktiler_comm_init_nccl(buf, nranks, rank, ctypes.byref(h)))
+        return cls(h)
+
+    @classmethod
+    def loopback(cls, nranks: int) -> "Comm":
+        h = ctypes.c_void_p()
+        _check(lib().ktiler_comm_init_loopback(nranks, ctypes.byref(h)))
+        return cls(h)
+
+    def register_strip(self, rank: int, base: int, pitch_bytes: int, row_bytes: int, o0: int, o1: int, e0: int,
+                       e1: int) -> None:
+        st = Strip(base, pitch_bytes, row_bytes, o0, o1, e0, e1)
+        _check(lib().ktiler_comm_register_strip(self._h, rank, ctypes.byref(st)))
+
+    def exchange(self, rank: int, halo_rows: int, stream: int = 0) -> None:
+        _check(lib().ktiler_halo_exchange(self._h, rank, halo_rows, ctypes.c_void_p(stream)))
+
+    def close(self):
+        if self._h:
+            lib().ktiler_comm_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -9,9 +9,12 @@ in full-resolution rows: mask row m needs sob row m, down rows m-1..m+1, blur ro
 there the kernels clamp (replicate border), exactly as the 1-GPU run does, and
 inside the image the halo makes every owned output identical to the whole-image result.
 
-This module holds only row bookkeeping and the exchange; the compute is the ordinary
-Pipeline (libktiler) on the extended strip.  The same exchange runs over gloo on CPU
-tensors in the tests.
+This module holds only row bookkeeping; the compute is the ordinary Pipeline (libktiler)
+on the extended strip.  The exchange itself runs in libktiler (comm.cpp:
+ktiler_halo_exchange — ncclSend/ncclRecv in one group, or the 1-GPU loopback backend), and
+``StripPipeline.attach`` puts it into the plan's CUDA graph ahead of the schedule.
+``exchange_halo`` is the same row bookkeeping over torch.distributed, used by the CPU
+(gloo) tests.
 """
 from __future__ import annotations
 
@@ -78,7 +81,19 @@ class StripPipeline:
         return self.pipe.view("mask")[0, self.m0:self.m1]
 
     def exchange(self, group=None) -> int:
+        """torch.distributed exchange (the gloo tests; kept for comparison)."""
         return exchange_halo(self.rgb_ext(), self.o0, self.o1, self.e0, self.e1, self.rank, self.world, group)
+
+    def register(self, comm) -> None:
+        """Register this rank's extended rgb strip with a libktiler comm (ktiler.Comm)."""
+        bid, W, H, F, elem, pitch = self.pipe.b.bufs["rgb"]
+        comm.register_strip(self.rank, self.rgb_ext().data_ptr(), pitch, W * elem, self.o0, self.o1, self.e0, self.e1)
+
+    def attach(self, comm) -> None:
+        """Register the strip and put the exchange into the current plan's graph, ahead of
+        the schedule (ktiler_plan_attach_halo): one execute = exchange + tiled schedule."""
+        self.register(comm)
+        self.pipe.plan_obj.attach_halo(comm, self.rank, HALO_ROWS)
 
     def plan(self, cache_bytes: int = 0, **policy):
         return self.pipe.plan(cache_bytes, **policy)
@@ -87,3 +102,13 @@ class StripPipeline:
         if self.world > 1:
             self.exchange(group)
         self.pipe.run(stream)
+
+
+def nccl_comm(world: int, rank: int):
+    """A libktiler NCCL comm over the ranks of the default torch.distributed group (the
+    unique id travels through the process group's broadcast)."""
+    import torch.distributed as dist
+    from . import ktiler as K
+    obj = [K.comm_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    return K.Comm.nccl(obj[0], world, rank)

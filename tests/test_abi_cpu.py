@@ -293,3 +293,49 @@ def test_planner_equals_oracle_a16b(K, lines):
     orphan = [f for n, b, f in ours if n == 0 and f not in b_frags]
     assert orphan, "A16b not triggered"
     assert all(by >= 16 for n, b, f in ours if f in orphan for (_, by, _) in b)
+
+
+def test_comm_abi_host_paths(K):
+    """Strip halo comm (include/ktiler.h, comm.cpp) host-side paths, no GPU: loopback
+    registration checks, missing-neighbour and misuse errors, attaching to a plan."""
+    c = K.Comm.loopback(3)
+    with pytest.raises(K.KtilerError) as e:  # e0 <= o0 < o1 <= e1 violated
+        c.register_strip(0, 1 << 20, 768, 768, 8, 4, 0, 12)
+    assert e.value.status == K.E_INVALID
+    with pytest.raises(K.KtilerError) as e:  # pitch < row bytes
+        c.register_strip(0, 1 << 20, 512, 768, 0, 8, 0, 12)
+    assert e.value.status == K.E_INVALID
+    c.register_strip(0, 1 << 20, 768, 768, 0, 8, 0, 12)
+    c.register_strip(1, 2 << 20, 768, 768, 8, 16, 4, 20)
+    with pytest.raises(K.KtilerError) as e:  # rank 1's bottom neighbour (rank 2) not registered
+        c.exchange(1, 4, 0)
+    assert e.value.status == K.E_STATE
+    with pytest.raises(K.KtilerError):
+        c.register_strip(3, 1 << 20, 768, 768, 0, 8, 0, 12)  # rank out of range
+    # a plan takes the exchange before its first execute (planning needs no GPU)
+    og, p = _pipe_pair(64, 96, 1, SMALL)
+    plan = p.plan(20000, kind="budget", exec_mode="dag")
+    plan.attach_halo(c, 0, 4)
+    uid = K.comm_unique_id()  # NCCL is loadable here (no GPU needed for the id)
+    assert len(uid) == 128
+    c.close()
+
+
+def test_flow_roles_abi(K):
+    """ktiler_plan_set_flow_roles validation (host side, before any execute)."""
+    og, p = _pipe_pair(64, 96, 1, SMALL)
+    plan = p.plan(20000, kind="rows", rows=1, exec_mode="flow", consumer_discard=True)
+    plan.set_flow_roles([0, 0, 0, 0, 0], [0, 0, 0, 0])
+    plan.set_flow_roles([0, 1, 2, 3, 4], [0, 1, 2, 3, 4])
+    plan.set_flow_roles([], [])  # automatic roles
+    for nr, sr in (([0, 1], [0, 1]),                    # one role per node
+                   ([0, 1, 1, 1, 1], [0, 0, 0]),          # role 1 has no slot
+                   ([0, 0, 0, 0, 0], [0]),                # < 2 slots
+                   ([0, 0, 0, 0, 0], [0] * 6)):           # > 5 slots
+        with pytest.raises(K.KtilerError) as e:
+            plan.set_flow_roles(nr, sr)
+        assert e.value.status == K.E_INVALID
+    dag = p.plan(20000, kind="budget", exec_mode="dag")
+    with pytest.raises(K.KtilerError) as e:
+        dag.set_flow_roles([0] * 5, [0, 0])
+    assert e.value.status == K.E_STATE

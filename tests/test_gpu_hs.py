@@ -58,3 +58,28 @@ def test_every_iterate_bit_exact():
     for k in range(1, K + 1):
         got = h.get(f"s{k}")
         assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 2.0, k).view(np.uint32)), k
+
+
+@pytest.mark.parametrize("rows", [2, 3])
+def test_frag_chain_bit_exact(rows):
+    """KTILER_FRAG_CHAIN (DESIGN A40, the policy the HS measurements use): clusters of
+    `rows` consecutive JI nodes, each tiled by Alg. 2, bit-exact vs O-14."""
+    W, H, K = 256, 128, 8
+    got, plan, coef, s0, _ = _run(W, H, 1, K, 0.5, 17, internal=True, kind="chain", rows=rows, exec_mode="dag",
+                                  cache_bytes=2 << 20)
+    assert len(plan.clusters()) == -(-K // rows) and plan.num_fragments() > 1
+    assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 0.5, K).view(np.uint32))
+
+
+def test_paper_shape_500_iterations():
+    """The paper's finest pyramid level (Fig. 4): 500 JI iterations on
+    a 1024^2 frame, tiled across iterations by the measured configuration (FRAG_CHAIN
+    clusters of 4 nodes under half the device L2, GRAPH_DAG), bit-exact vs the f32 oracle
+    after all 500 iterations (parity stopped at K = 8)."""
+    W = H = 1024
+    K = 500
+    got, plan, coef, s0, _ = _run(W, H, 1, K, 0.5, 2024, internal=True, kind="chain", rows=4, exec_mode="dag",
+                                  cache_bytes=0, l2_fraction=0.5)
+    assert len(plan.clusters()) == K // 4
+    ref = O.hs_jacobi(coef, s0, 0.5, K)
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))

@@ -293,23 +293,55 @@ def test_trace_records(mode):
 
 
 @pytest.mark.parametrize("world", [2, 4])
-@pytest.mark.parametrize("mode", ["graph", "dag", "wave"])
+@pytest.mark.parametrize("mode", ["graph", "dag", "wave", "stream", "flow"])
 def test_strips_on_one_gpu(world, mode):
-    """§8(e) strip path, GPU side: each rank's extended strip (owned rows + the halo the
-    exchange delivers) through libktiler; concatenated owned masks == whole-image oracle."""
+    """§8(e) strip path, GPU side, through the real exchange: every emulated rank holds only
+    its OWN rows; the 1-GPU loopback comm (libktiler ktiler_halo_exchange, one
+    cudaMemcpy2DAsync per halo) attached to each rank's plan fills the halo rows inside the
+    plan's graph; concatenated owned masks == whole-image oracle.  The halo rows are
+    poisoned first, so a missing exchange cannot pass."""
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler as K
     from paper_conf_date_maghazeh0ep19_b200.strips import StripPipeline
     W, H = 1024, 512
     full = synth.scene(77, W, H, 1)[0]
     want = O.pipeline(full[None], T=45.0)["mask"][0]
-    got = []
+    comm = K.Comm.loopback(world)
+    sps = []
     for r in range(world):
         sp = StripPipeline(W, H, world, r, T=45.0, geometry=SMALL, internal=True)
-        sp.rgb_ext().copy_(torch.from_numpy(full[sp.e0:sp.e1]))
-        sp.plan(64 * 1024, kind="budget", exec_mode=mode, discard=True)
+        sp.rgb_ext().fill_(0xA5)
+        sp.rgb_ext()[sp.own_offset:sp.own_offset + (sp.o1 - sp.o0)].copy_(torch.from_numpy(full[sp.o0:sp.o1]))
+        pol = dict(kind="rows", rows=1, consumer_discard=True) if mode == "flow" else dict(kind="budget", discard=True)
+        sp.plan(64 * 1024, exec_mode=mode, **pol)
+        sps.append(sp)
+    for sp in sps:  # every strip registered before any exchange runs
+        sp.register(comm)
+    got = []
+    for sp in sps:
+        sp.pipe.plan_obj.attach_halo(comm, sp.rank, 4)
         sp.pipe.run()
         torch.cuda.synchronize()
+        assert np.array_equal(sp.rgb_ext().cpu().numpy(), full[sp.e0:sp.e1])  # halo rows delivered
         got.append(sp.mask_owned().cpu().numpy())
     assert np.array_equal(np.concatenate(got), want)
+
+
+def test_halo_exchange_nccl_single_rank():
+    """The NCCL backend through the C ABI on one rank (the only NCCL world one GPU allows):
+    unique id, communicator, strip registration, the exchange attached to a DAG plan (no
+    neighbour: no rows move); the output equals the oracle."""
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler as K
+    from paper_conf_date_maghazeh0ep19_b200.strips import StripPipeline
+    W, H = 512, 128
+    full = synth.scene(5, W, H, 1)[0]
+    comm = K.Comm.nccl(K.comm_unique_id(), 1, 0)
+    sp = StripPipeline(W, H, 1, 0, T=45.0, geometry=SMALL, internal=True)
+    sp.rgb_ext().copy_(torch.from_numpy(full))
+    sp.plan(64 * 1024, kind="budget", exec_mode="dag")
+    sp.attach(comm)
+    sp.pipe.run()
+    torch.cuda.synchronize()
+    assert np.array_equal(sp.mask_owned().cpu().numpy(), O.pipeline(full[None], T=45.0)["mask"][0])
 
 
 def test_selftest_sqrt_exhaustive():
