@@ -72,6 +72,8 @@ def parse(argv=None):
                     help="frames: strong (default) = the one batch split into contiguous frame ranges "
                          "(BASELINE configs[3]); weak = every rank runs a whole batch of its own")
     ap.add_argument("--window", type=int, default=2)
+    ap.add_argument("--ring-frames", type=int, default=0,
+                    help="intermediates as WAR-aware rings of this many frames (SURVEY f4; 0 = full batch)")
     ap.add_argument("--discard", action="store_true",
                     help="discard dead intermediate lines (DRAM -55%% but slower on B200: DESIGN.md §6)")
     ap.add_argument("--no-discard", action="store_true", help="(default) keep dead lines")
@@ -91,6 +93,7 @@ def parse(argv=None):
     ap.add_argument("--no-untiled", action="store_true")
     ap.add_argument("--no-trace", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-ncu", action="store_true", help="skip the in-run ncu DRAM / L2-hit capture")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     return ap.parse_args(argv)
 
@@ -175,26 +178,63 @@ def traffic_for(cfg: dict):
     return None, None
 
 
+def _oracle_frame(job):
+    """One worker of the all-cores oracle: frame f of the workload through O-6."""
+    W, rows, T, seed, f = job
+    from inputs import synth
+    from oracle import oracle as O
+    t0 = time.perf_counter()
+    O.pipeline(synth.scene(seed + f, W, rows, 1), T=T)
+    return time.perf_counter() - t0
+
+
 def cpu_baseline(W, H, T, seed, target_s):
     """The oracle as it stands (single-threaded C, O-6) on a bounded sample: whole frames
     of the workload, as many as fit ~target_s seconds (at least one; a row band for
-    images larger than one 8K frame)."""
+    images larger than one 8K frame), on ONE core (the process pinned to CPU 0 for the
+    duration); then the all-cores figure: nproc processes x one frame each,
+    wall time of the whole set (BASELINE configs[3] "the oracle timed on the box's own host
+    cores")."""
     from inputs import synth
     from oracle import oracle as O
     rows = H if W * H <= 7680 * 4320 else max(64, (7680 * 4320 // W) // 16 * 16)
     rgb = synth.scene(seed, W, rows, 1)
-    t0 = time.perf_counter()
-    O.pipeline(rgb, T=T)
-    one = time.perf_counter() - t0
-    n, dt = 1, one
-    while dt + one <= target_s:
-        t1 = time.perf_counter()
+    old_aff = None
+    try:
+        old_aff = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {min(old_aff)})
+    except (AttributeError, OSError):
+        pass
+    try:
+        t0 = time.perf_counter()
         O.pipeline(rgb, T=T)
-        dt += time.perf_counter() - t1
-        n += 1
-    return {"value": W * rows * n / dt / 1e6, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} x {W}x{rows} scene image(s) through the untiled oracle graph, 1 thread, {dt:.1f} s",
-            "host": host_cpu()}
+        one = time.perf_counter() - t0
+        n, dt = 1, one
+        while dt + one <= target_s:
+            t1 = time.perf_counter()
+            O.pipeline(rgb, T=T)
+            dt += time.perf_counter() - t1
+            n += 1
+    finally:
+        if old_aff:
+            os.sched_setaffinity(0, old_aff)
+    out = {"value": W * rows * n / dt / 1e6, "unit": "Mpix/s", "cores": 1, "kind": "oracle",
+           "sample": f"{n} x {W}x{rows} scene image(s) through the untiled oracle graph, 1 thread pinned to "
+                     f"CPU {min(old_aff) if old_aff else '?'}, {dt:.1f} s",
+           "host": host_cpu()}
+    ncores = len(old_aff) if old_aff else (os.cpu_count() or 1)
+    if ncores > 1:
+        import concurrent.futures as cf
+        import multiprocessing as mp
+        jobs = [(W, rows, T, seed, f) for f in range(ncores)]
+        t0 = time.perf_counter()
+        with cf.ProcessPoolExecutor(ncores, mp_context=mp.get_context("spawn")) as ex:
+            list(ex.map(_oracle_frame, jobs))
+        wall = time.perf_counter() - t0
+        out["all_cores"] = {"value": W * rows * ncores / wall / 1e6, "unit": "Mpix/s", "cores": ncores,
+                            "sample": f"{ncores} processes x one {W}x{rows} frame each (frames seed+0..{ncores - 1}), "
+                                      f"wall {wall:.1f} s including process start"}
+    return out
 
 
 def host_cpu() -> dict:
@@ -284,6 +324,60 @@ def trace_shares(pipe, pol):
     return out, span / 1e6, per
 
 
+def ktiler_env() -> dict:
+    """Every KTILER_* variable of the environment (experiment knobs the library reads):
+    echoed into the line so a stray knob can never silently change the measured config."""
+    return {k: v for k, v in sorted(os.environ.items()) if k.startswith("KTILER_")}
+
+
+def ncu_traffic(args, pols, timeout_s=420, ring=0):
+    """DRAM bytes and L2 sector hit rate of one execute of each policy in `pols`, measured
+    in THIS run by ncu (graph-level ranges, caches flushed before each, 3rd execute of
+    tools/sweep.py's 2 warm-ups + 1), on the workload's own shape.  None if ncu is absent
+    or fails (then profiles/traffic.json, if it matches, is reported instead)."""
+    import shutil
+    import subprocess
+    import tempfile
+    ncu = shutil.which("ncu") or ("/usr/local/cuda/bin/ncu" if os.path.exists("/usr/local/cuda/bin/ncu") else None)
+    if not ncu:
+        return None
+    W, H, Ftot, _, _ = WORKLOADS[args.workload]
+    with tempfile.TemporaryDirectory() as d:
+        csv_path = os.path.join(d, "t.csv")
+        cmd = [ncu, "--graph-profiling", "graph", "--cache-control", "all", "--clock-control", "none", "--metrics",
+               "dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__time_duration.sum", "--csv",
+               "--log-file", csv_path, sys.executable, os.path.join(ROOT, "tools", "sweep.py"), "--W", str(W), "--H",
+               str(H), "--F", str(Ftot), "--reps", "1", "--ring", str(ring), "--configs", json.dumps(pols)]
+        try:
+            r = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout_s, cwd=ROOT)
+            if r.returncode:
+                return None
+            rows = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "traffic_summary.py"), csv_path],
+                                  capture_output=True, text=True, check=True).stdout.splitlines()
+        except Exception:
+            return None
+    rows = [json.loads(x) for x in rows]
+    per = len(rows) // max(1, len(pols))
+    if per < 3:
+        return None
+    out = []
+    for i in range(len(pols)):
+        g = rows[i * per:(i + 1) * per]
+        r3 = g[2]  # the 3rd execute (2 warm-ups)
+        if per > 3:  # non-graph executors (several ranges per execute): sum the last execute's ranges
+            k = (per) // 3
+            last = g[2 * k:3 * k]
+            r3 = {"read_GB": sum(x["read_GB"] for x in last), "write_GB": sum(x["write_GB"] for x in last),
+                  "dram_GB": sum(x["dram_GB"] for x in last), "l2_hit_pct": None,
+                  "ms": sum(x["ms"] for x in last)}
+        out.append({"dram_bytes": r3["dram_GB"] * 1e9, "dram_read": r3["read_GB"] * 1e9,
+                    "dram_write": r3["write_GB"] * 1e9, "lts_sector_hit_rate_pct": r3["l2_hit_pct"],
+                    "ncu_duration_ms": r3["ms"],
+                    "source": "ncu in this bench run (--graph-profiling graph --cache-control all --clock-control none, "
+                              "tools/sweep.py 3rd execute; serialised under the profiler: bytes, not time)"})
+    return out
+
+
 def policy(args) -> dict:
     """The fragment policy of the timed step (also used by tests/test_gpu_fullsize.py)."""
     return dict(kind=args.kind, rows=args.rows, l2_fraction=args.l2_fraction, exec_mode=args.mode,
@@ -335,7 +429,7 @@ def main():
         else:  # weak: every rank its own whole batch (frames Ftot*rank ...)
             f0, per = (rank * Ftot if shard == "frames" else 0), Ftot
             pix_ranks = [W * H * Ftot] * world
-        p = Pipeline(W, H, per, T=args.T, internal=True)
+        p = Pipeline(W, H, per, T=args.T, internal=True, ring_frames=args.ring_frames)
         G.fill("scene", args.seed, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, f0=f0, F=per, stream=s)
         pix_rank = W * H * per
     torch.cuda.synchronize()
@@ -416,12 +510,13 @@ def main():
                    "sharding": shard if world > 1 else "none", "pixels_per_gpu": pix_rank, "mode": args.mode,
                    "policy": args.kind, "rows": args.rows, "l2_fraction": args.l2_fraction, "window": args.window,
                    "resident_budget": resident, "discard": discard, "consumer_discard": pol["consumer_discard"],
-                   "halo_discard": pol["halo_discard"],
+                   "halo_discard": pol["halo_discard"], "ring_frames": args.ring_frames,
                    "pdl": args.pdl,
                    "l2_flush": "not needed: each step reads >= 6.4 GB of input (>> 126 MB L2)" if Ftot > 1 or W >= 16384
                    else "none (input smaller than L2: steady-state replay)",
                    "fragments": st["n_fragments"], "subkernels": st["n_subkernels"],
-                   "plan_ms": round(st["plan_ms"], 1), "input": f"scene(seed={args.seed}) per frame"},
+                   "plan_ms": round(st["plan_ms"], 1), "input": f"scene(seed={args.seed}) per frame",
+                   "env": ktiler_env()},
         "gpu_launches": int(st["n_launches"]) * args.steps,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "traffic_source": traffic_src,
@@ -440,8 +535,12 @@ def main():
         line["roofline"]["l2"] = {"bound": "l2", "read_peak": l2["read"], "write_peak": l2["write"], "unit": "GB/s",
                                   "algorithmic_bytes": "6.25 B/px read + 3.5 B/px written (all five kernels)",
                                   "floor_ms": floor_ms, "frac": floor_ms / ms, "source": l2["source"]}
+    pu = p  # the untiled baseline's pipeline (full-batch intermediates when the tiled one uses rings)
+    if args.ring_frames and sp is None:
+        pu = Pipeline(W, H, per, T=args.T, internal=True)
+        pu.view("rgb").copy_(p.view("rgb"))
     if not args.no_untiled:
-        un = p.b.g.plan(0, kind="none", exec_mode="graph", discard=False)
+        un = pu.b.g.plan(0, kind="none", exec_mode="graph", discard=False)
         if comm is not None:
             un.attach_halo(comm, rank, SM.HALO_ROWS)
         ms_un = timed(lambda: un.execute(s), max(3, args.steps // 2), 2)
@@ -454,7 +553,7 @@ def main():
     if not args.no_trace and rank == 0:
         try:
             tiled_sh, tiled_span, per_node = trace_shares(p, pol) if args.mode != "persistent" else (None, None, None)
-            un_sh, un_span, _ = trace_shares(p, dict(kind="none", exec_mode="graph"))
+            un_sh, un_span, _ = trace_shares(pu, dict(kind="none", exec_mode="graph"))
             line["trace"] = {"tiled_cta_share": tiled_sh, "tiled_span_ms": tiled_span, "untiled_cta_share": un_sh,
                              "untiled_span_ms": un_span}
             if per_node:
@@ -520,6 +619,25 @@ def main():
                        "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                        "path": (e2e_path or "ktiler_execute_host (pinned host rgb -> device -> plan -> host mask)")
                        if sp is None else "pinned host rows -> device, halo exchange, ktiler_execute, mask -> host"}
+    if rank == 0 and world == 1 and not args.no_ncu and sp is None:
+        # DRAM bytes and L2 hit rate of the tiled step and of the untiled one, measured by
+        # ncu on this run's exact configuration (the metric's "DRAM bytes & L2 hit rate")
+        if args.ring_frames:  # the untiled schedule needs full-batch intermediates
+            mt = ncu_traffic(args, [pol], ring=args.ring_frames)
+            mu = ncu_traffic(args, [dict(kind="none", exec_mode="graph")])
+            meas = mt + mu if mt and mu else None
+        else:
+            meas = ncu_traffic(args, [pol, dict(kind="none", exec_mode="graph")])
+        if meas:
+            t, u = meas
+            line["roofline"]["traffic"] = t["dram_bytes"]
+            line["roofline"]["traffic_source"] = t["source"]
+            line["dram"] = {"tiled_bytes": t["dram_bytes"], "tiled_read": t["dram_read"], "tiled_write": t["dram_write"],
+                            "untiled_bytes": u["dram_bytes"], "untiled_read": u["dram_read"],
+                            "untiled_write": u["dram_write"], "reduction": 1.0 - t["dram_bytes"] / u["dram_bytes"],
+                            "compulsory_bytes": comp_bytes, "source": t["source"]}
+            line["l2_hit_rate"] = {"tiled_pct": t["lts_sector_hit_rate_pct"], "untiled_pct": u["lts_sector_hit_rate_pct"],
+                                   "metric": "lts__t_sector_hit_rate.pct", "source": t["source"]}
     if rank == 0 and world == 1 and not args.no_cpu:
         line["cpu_baseline"] = cpu_baseline(W, H, args.T, args.seed, args.cpu_seconds)
     if rank == 0:

@@ -42,11 +42,15 @@ constexpr int PMAX_NODES = 8;
 struct LRect {
   int32_t x0, y0, z0, x1, y1, z1;
 };
-struct DRect {  // whole 128-B lines: row r -> base + z*fs + y*pitch + lb0 + k*128, k < lpr
+struct DRect {  // whole 128-B lines: row r -> base + (z mod ring)*fs + y*pitch + lb0 + k*128, k < lpr
   uint8_t* base;
   int64_t pitch, fstride, lb0, lpr;
   int32_t y0, y1, z0, z1;
+  int32_t ring, pad;
 };
+__device__ __forceinline__ int64_t drect_zoff(const DRect& d, int64_t z) {
+  return (d.ring ? (int64_t)((uint32_t)z % (uint32_t)d.ring) : z) * d.fstride;
+}
 // Device-side trace ring (ktiler_trace_enable): NULL rec = tracing off.
 struct TraceBuf {
   ktiler_trace_record* rec;
@@ -114,6 +118,19 @@ __device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
 __device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// Watchdog for every spin on another CTA's progress (CHAIN flags and prefixes, PERSISTENT
+// counters): sleep between polls, and after KT_SPIN_LIMIT polls (seconds) trap with the
+// waiter's identity in the message instead of hanging the GPU — an unsatisfiable wait is
+// a schedule bug (every executor's order is deadlock-free by construction).
+constexpr unsigned long long KT_SPIN_LIMIT = 1ull << 25;
+__device__ __noinline__ void kt_watchdog_trap(const char* what, long long id, unsigned long long n) {
+  printf("libktiler watchdog: %s (id %lld) waited %llu polls: trapping\n", what, id, n);
+  __trap();
+}
+__device__ __forceinline__ void kt_spin(unsigned long long& n, unsigned ns, const char* what, long long id) {
+  __nanosleep(ns);
+  if (++n > KT_SPIN_LIMIT) kt_watchdog_trap(what, id, n);
+}
 
 // GRAPH_CHAIN, one warp: wait until every producer block of output block (bx, by, bz)
 // has published this epoch.  Producer range = closed form of the affine footprints
@@ -128,7 +145,7 @@ __device__ __forceinline__ void chain_wait(const KParams& p, int bx, int by, int
   for (int i = lane; i < n; i += 32) {
     const int dy = i / pw;
     const unsigned int* f = p.pflags + ((int64_t)bz * p.pgy + py0 + dy) * p.pgx + px0 + (i - dy * pw);
-    while (ld_acquire(f) != epoch) __nanosleep(64);
+    for (unsigned long long w = 0; ld_acquire(f) != epoch;) kt_spin(w, 64, "CHAIN producer-block flag", (long long)(f - p.pflags));
   }
   __syncwarp();
 }
@@ -147,7 +164,7 @@ __device__ __forceinline__ void do_discards(const KParams& p) {
     int64_t row = j / d.lpr, l = j % d.lpr;
     int64_t h = d.y1 - d.y0;
     int64_t z = d.z0 + row / h, y = d.y0 + row % h;
-    ktd::discard_line(d.base + z * d.fstride + y * d.pitch + d.lb0 + 128 * l);
+    ktd::discard_line(d.base + drect_zoff(d, z) + y * d.pitch + d.lb0 + 128 * l);
   }
 }
 
@@ -189,7 +206,7 @@ __device__ __forceinline__ void chain_finish(const KParams& p, unsigned epoch, b
   if (old == gridDim.x - 1) {
     *p.dcount = 0;  // ready for the next execute (every CTA of this launch has counted)
     if (!first_launch)
-      while (ld_acquire(p.prefix - 1) != epoch) __nanosleep(128);
+      for (unsigned long long w = 0; ld_acquire(p.prefix - 1) != epoch;) kt_spin(w, 128, "CHAIN launch prefix", 0);
     __threadfence();
     st_release(p.prefix, epoch);
   }
@@ -201,7 +218,7 @@ template <int OP>
 __device__ __forceinline__ void consumer_discard(const KParams& p, const ktd::Tile& t, int nt, int tid) {
   constexpr int EB = OP == 2 ? 2 : 4;  // input bytes per output pixel along x (down2: 2 u8; thresh: 1 f32)
   const int64_t y0 = OP == 2 ? 2 * t.y0 : t.y0, nrows = OP == 2 ? 2 * (t.y1 - t.y0) : t.y1 - t.y0;
-  const uint8_t* base = p.in.p + t.z * p.in.fstride;
+  const uint8_t* base = p.in.p + ktd::zoff(p.in, t.z);
   const int64_t b0 = EB * t.x0, b1 = EB * t.x1;
   for (int64_t i = tid;; i += nt) {
     // lines of row r: [ceil(a / 128), floor(b / 128)) of absolute addresses a, b
@@ -226,7 +243,7 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
   const int px0 = rx0 / p.wax, px1 = min(p.pgx, (rx1 + p.wax - 1) / p.wax);
   const int py0 = ry0 / p.way, py1 = min(p.pgy, (ry1 + p.way - 1) / p.way);
   const int pw = px1 - px0, n = pw * (py1 - py0);
-  const uint8_t* fb = p.in.p + (int64_t)bz * p.in.fstride;
+  const uint8_t* fb = p.in.p + ktd::zoff(p.in, bz);
   for (int i0 = 0; i0 < n; i0 += 32) {
     const int i = i0 + lane;
     const int py = py0 + i / max(pw, 1), px = px0 + i % max(pw, 1);
@@ -367,7 +384,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     if (tid == 0) chain_finish(p, s_epoch, p.chain == 2);
     if (p.ndisc) {  // lines dead after an earlier launch: wait until it and all before it finished
       if (tid == 0)
-        while (ld_acquire(p.disc_prefix) != s_epoch) __nanosleep(128);
+        for (unsigned long long w = 0; ld_acquire(p.disc_prefix) != s_epoch;) kt_spin(w, 128, "CHAIN discard prefix", 0);
       __syncthreads();
       do_discards(p);
     }
@@ -386,7 +403,7 @@ __global__ void chain_tail_kernel(const __grid_constant__ KParams p) {
   __shared__ unsigned int s_ep;
   if (threadIdx.x == 0) {
     s_ep = *(volatile const unsigned int*)p.epoch;
-    while (ld_acquire(p.disc_prefix) != s_ep) __nanosleep(256);
+    for (unsigned long long w = 0; ld_acquire(p.disc_prefix) != s_ep;) kt_spin(w, 256, "CHAIN tail prefix", 0);
   }
   __syncthreads();
   if (p.ndisc) do_discards(p);
@@ -532,7 +549,8 @@ __device__ __forceinline__ void wait_group(const PParams& p, int group, unsigned
     const PDep dp = p.deps[i];
     const unsigned target = epoch * dp.ntiles;
     if ((int)(ld_relaxed(p.cnt + dp.sub) - target) < 0) {
-      while ((int)(ld_relaxed(p.cnt + dp.sub) - target) < 0) __nanosleep(100);
+      for (unsigned long long w = 0; (int)(ld_relaxed(p.cnt + dp.sub) - target) < 0;)
+        kt_spin(w, 100, "PERSISTENT sub-kernel counter", dp.sub);
     }
     (void)ld_acquire(p.cnt + dp.sub);
   }
@@ -567,7 +585,8 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
   __shared__ uint64_t s_desc[PSTAGES_MAX];
   __shared__ ktd::Tile s_tile[PSTAGES_MAX];
   __shared__ int32_t s_pub[PUBQ];          // group of finished ticket k (k mod PUBQ)
-  __shared__ volatile int32_t s_pubk;      // tickets the publisher has consumed
+  __shared__ int32_t s_pubk;  // tickets the publisher has consumed (shared atomics: a lock-free
+                              // progress counter, written by the publisher, read by the producer)
   __shared__ __align__(64) PNode s_nodes[PMAX_NODES];
   __shared__ unsigned int s_epoch;
   __shared__ int32_t s_okg[64];
@@ -612,7 +631,8 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
       }
       const uint64_t d = __shfl_sync(FULL, batch, dyn ? (int)(k % DYN_B) : (int)(k & 31));
       if (k >= S) ktd::mbar_wait(&s_empty[s], ((ph >> s) & 1u) ^ 1u);
-      while ((int)k - s_pubk > PUBQ - PSTAGES_MAX) __nanosleep(200);  // publisher queue bound
+      for (unsigned long long w = 0; (int)k - atomicAdd(&s_pubk, 0) > PUBQ - PSTAGES_MAX;)  // publisher queue bound
+        kt_spin(w, 200, "PERSISTENT publisher queue", k);
       const uint64_t kind = d >> 60;
       if (kind == PK_STOP) {  // one STOP per compute group: tickets k .. k+NG-1
         if (lane == 0) {
@@ -671,10 +691,10 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
         if (lane == 0) red_release_add(p.cnt + cur, pend);
         pend = 0;
       }
-      while (!mbar_test(&s_done[q], par)) __nanosleep(64);
+      for (unsigned long long w = 0; !mbar_test(&s_done[q], par);) kt_spin(w, 64, "PERSISTENT finished tile", k);
       const int group = s_pub[q];
       __syncwarp();
-      if (lane == 0) s_pubk = k + 1;
+      if (lane == 0) atomicExch(&s_pubk, k + 1);
       ph ^= 1ull << q;
       if (group < 0) {  // STOP of one compute group
         if (++stops == NG) break;
@@ -711,7 +731,7 @@ __global__ void __launch_bounds__(NG * PCOMP_THREADS + 64, MINB) persistent_kern
         for (int64_t i = gtid; i < c.n; i += PCOMP_THREADS) {
           const int64_t j = c.l0 + i, row = j / r.lpr, l = j - row * r.lpr;
           const int64_t z = r.z0 + row / h, y = r.y0 + row % h;
-          ktd::discard_line(r.base + z * r.fstride + y * r.pitch + r.lb0 + 128 * l);
+          ktd::discard_line(r.base + drect_zoff(r, z) + y * r.pitch + r.lb0 + 128 * l);
         }
       } else {
         const PNode& nd = s_nodes[kind];
@@ -848,6 +868,9 @@ struct ktiler_plan_s {
   TraceBuf tb{nullptr, nullptr, 0};
   bool executed = false;
   ktiler_status sticky = KTILER_OK;  // a failed first-execute setup: the plan stays unusable
+  // ring buffers (ktiler_buffer_desc.ring_frames): per sub-kernel, the earlier sub-kernels
+  // that must finish first because they read (or write) the frame its writes overwrite
+  std::vector<std::vector<int32_t>> war;
   // FLOW state (KTILER_EXEC_FLOW): roles (ktiler_plan_set_flow_roles; empty = automatic)
   std::vector<int32_t> flow_node_role, flow_slot_role;
   ktflow::FParams fp{};
@@ -878,7 +901,8 @@ namespace {
 using kt::fail;
 
 DBuf dbuf(const kt::Buffer& b) {
-  return DBuf{(uint8_t*)b.d.base, b.d.width, b.d.height, b.d.pitch_bytes, b.d.frame_stride_bytes};
+  return DBuf{(uint8_t*)b.d.base, b.d.width, b.d.height, b.d.pitch_bytes, b.d.frame_stride_bytes,
+              (int32_t)b.d.ring_frames, 0};
 }
 
 bool discardable(const kt::Buffer& b) { return (b.d.pitch_bytes % 128 == 0) && (b.d.frame_stride_bytes % 128 == 0); }
@@ -908,11 +932,75 @@ DRect drect(const kt::Graph& g, const kt::Discard& d) {
   r.base = (uint8_t*)b.d.base;
   r.pitch = b.d.pitch_bytes;
   r.fstride = b.d.frame_stride_bytes;
+  r.ring = (int32_t)b.d.ring_frames;
+  r.pad = 0;
   r.lb0 = (d.xb0 + 127) & ~127ll;
   int64_t lb1 = d.xb1 & ~127ll;
   r.lpr = lb1 > r.lb0 ? (lb1 - r.lb0) / 128 : 0;
   r.y0 = d.y0; r.y1 = d.y1; r.z0 = d.z0; r.z1 = d.z1;
   return r;
+}
+
+// Ring buffers: frame z of a ring of R frames overwrites the slot of frame
+// z - R, so every writer of frame z must follow every reader (and the writer) of frame
+// z - R — write-after-read / write-after-write order the paper's RAW-only model
+// does not have.  Per sub-kernel, the list of such earlier sub-kernels
+// (P->war).  Total-order executors (STREAM, GRAPH) need them to precede it in the order
+// (else KTILER_E_UNTILEABLE: a fragment spans R frames or more); GRAPH_DAG adds them as
+// edges; the other executors do not support rings.
+ktiler_status ring_analysis(ktiler_plan_s* P) {
+  const kt::Graph& g = P->g;
+  const kt::Schedule& S = P->s;
+  const int nsub = (int)S.subs.size();
+  P->war.assign(nsub, {});
+  bool any = false;
+  for (auto& b : g.bufs) any |= b.d.ring_frames > 0;
+  if (!any) return KTILER_OK;
+  const int m = P->pol.exec_mode;
+  if (m != KTILER_EXEC_STREAM && m != KTILER_EXEC_GRAPH && m != KTILER_EXEC_GRAPH_DAG)
+    return fail(KTILER_E_UNSUPPORTED, "ring buffers (ring_frames) need STREAM, GRAPH or GRAPH_DAG");
+  for (int bi = 0; bi < (int)g.bufs.size(); ++bi) {
+    const kt::Buffer& B = g.bufs[bi];
+    const int64_t R = B.d.ring_frames, F = B.d.frames;
+    if (!R) continue;
+    std::vector<std::vector<int32_t>> users(F);  // per frame: sub-kernels reading or writing it
+    std::vector<std::vector<int32_t>> writers(F);
+    for (int si = 0; si < nsub; ++si) {
+      const kt::SubKernel& sk = S.subs[si];
+      const kt::Node& n = g.nodes[sk.node];
+      bool rd = false, wr = false;
+      for (auto& a : n.acc)
+        if (a.buf == bi) (a.mode == KTILER_WRITE ? wr : rd) = true;
+      if (!rd && !wr) continue;
+      std::vector<uint8_t> seen(F, 0);
+      for (auto& r : sk.rects)
+        for (int64_t z = r.z0; z < r.z1; ++z) seen[z] = 1;
+      for (int64_t z = 0; z < F; ++z)
+        if (seen[z]) {
+          users[z].push_back(si);
+          if (wr) writers[z].push_back(si);
+        }
+    }
+    for (int64_t z = R; z < F; ++z)
+      for (int32_t w : writers[z])
+        for (int32_t u : users[z - R]) {
+          if (u == w) return fail(KTILER_E_UNTILEABLE, "ring buffer " + std::to_string(bi) + ": one sub-kernel spans frames " +
+                                                           std::to_string(z - R) + " and " + std::to_string(z) + " of a " +
+                                                           std::to_string(R) + "-frame ring");
+          if (m != KTILER_EXEC_GRAPH_DAG && u > w)
+            return fail(KTILER_E_UNTILEABLE, "ring buffer " + std::to_string(bi) + " of " + std::to_string(R) +
+                                                 " frames: frame " + std::to_string(z) + " is written before frame " +
+                                                 std::to_string(z - R) + " is read in this order (a fragment spans >= " +
+                                                 std::to_string(R) + " frames): use a larger ring");
+          if (u > w) return fail(KTILER_E_UNTILEABLE, "ring buffer: a reader of frame z-R follows the writer of z in the order");
+          P->war[w].push_back(u);
+        }
+  }
+  for (auto& v : P->war) {
+    std::sort(v.begin(), v.end());
+    v.erase(std::unique(v.begin(), v.end()), v.end());
+  }
+  return KTILER_OK;
 }
 
 void build_launches(ktiler_plan_s* P) {
@@ -1079,6 +1167,7 @@ std::vector<std::vector<int>> dag_edges(const ktiler_plan_s* P) {
   std::vector<int> last_of_node(g.nodes.size(), -1);
   for (int i = 0; i < nsub; ++i) {
     e[i].assign(S.sub_deps[i].begin(), S.sub_deps[i].end());
+    if (i < (int)P->war.size()) e[i].insert(e[i].end(), P->war[i].begin(), P->war[i].end());  // ring WAR order
     const int prev = last_of_node[S.subs[i].node];
     if (prev >= 0) e[i].push_back(prev);
     const int f = S.subs[i].frag;
@@ -1189,7 +1278,8 @@ bool make_tmap(const kt::Graph& g, const kt::Node& n, CUtensorMap* m, uint32_t* 
   if (bw % 16 || bw / 4 > 256 || bh > 256 || bw * bh != window) return false;
   if (B.d.pitch_bytes % 16 || B.d.frame_stride_bytes % 16) return false;
   const int64_t rowbytes = B.d.width * B.d.elem_bytes;
-  cuuint64_t dims[3] = {(cuuint64_t)((rowbytes + 3) / 4), (cuuint64_t)B.d.height, (cuuint64_t)B.d.frames};
+  cuuint64_t dims[3] = {(cuuint64_t)((rowbytes + 3) / 4), (cuuint64_t)B.d.height,
+                        (cuuint64_t)(B.d.ring_frames ? B.d.ring_frames : B.d.frames)};
   cuuint64_t strides[2] = {(cuuint64_t)B.d.pitch_bytes, (cuuint64_t)B.d.frame_stride_bytes};
   cuuint32_t box[3] = {(cuuint32_t)(bw / 4), (cuuint32_t)bh, 1}, es[3] = {1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, B.d.base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -1851,52 +1941,13 @@ ffn_t flow_variant(int k) {
 }
 int flow_threads(int k) { return k == 5 ? 128 : (k == 2 ? 288 : 160); }
 
-// Automatic roles: every node its own role when the slots allow, the slots shared out in
-// proportion to each node's staged + written bytes (at least one each); otherwise
-// consecutive nodes (topological order) grouped into K roles of balanced bytes.
+// Automatic roles: ONE role serving every node, on K slots per SM.  Measured on 16 x 8K
+// (profiles/r02_flow_sweeps.txt): a CTA that can take any ready tile keeps its warps busy;
+// per-node roles leave the issue-bound nodes (blur, sobel) with a few warps per SM and
+// multi-node roles without the others' tiles stall on their own dependencies.
 void flow_auto_roles(const kt::Graph& g, int K, std::vector<int32_t>& node_role, std::vector<int32_t>& slot_role) {
-  const int nn = (int)g.nodes.size();
-  std::vector<double> wt(nn, 0.0);
-  for (int v = 0; v < nn; ++v) {
-    const kt::Node& n = g.nodes[v];
-    const kt::Access& w = n.acc[n.wacc];
-    const double per = ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) +
-                       (double)w.ax * w.ay * g.bufs[w.buf].d.elem_bytes;
-    wt[v] = per * (double)n.nblocks;
-  }
-  node_role.assign(nn, 0);
-  slot_role.clear();
-  if (nn <= K) {
-    for (int i = 0; i < nn; ++i) node_role[g.topo[i]] = i;
-    std::vector<int> cnt(nn, 1);
-    double tot = 0;
-    for (double x : wt) tot += x;
-    for (int extra = K - nn; extra > 0; --extra) {  // largest weight per slot gets the next slot
-      int best = 0;
-      double bv = -1;
-      for (int i = 0; i < nn; ++i) {
-        const double r = wt[g.topo[i]] / cnt[i];
-        if (r > bv) { bv = r; best = i; }
-      }
-      ++cnt[best];
-    }
-    for (int i = 0; i < nn; ++i)
-      for (int c = 0; c < cnt[i]; ++c) slot_role.push_back(i);
-    (void)tot;
-    return;
-  }
-  // nn > K: contiguous groups, greedy on the running weight
-  double tot = 0;
-  for (double x : wt) tot += x;
-  double acc = 0;
-  int r = 0;
-  for (int i = 0; i < nn; ++i) {
-    const int v = g.topo[i];
-    if (r < K - 1 && acc > 0 && acc + wt[v] / 2 > tot * (r + 1) / K) ++r;
-    acc += wt[v];
-    node_role[v] = r;
-  }
-  for (int i = 0; i < K; ++i) slot_role.push_back(std::min(i, r));
+  node_role.assign(g.nodes.size(), 0);
+  slot_role.assign(K, 0);
 }
 
 ktiler_status setup_flow(ktiler_plan_s* P) {
@@ -1958,7 +2009,7 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
 
   }
   // ---- kernel variant, slots (CTAs) per SM, shared memory per CTA ----
-  int K = P->flow_slot_role.empty() ? 4 : (int)P->flow_slot_role.size();
+  int K = P->flow_slot_role.empty() ? 3 : (int)P->flow_slot_role.size();
   if (K < 2 || K > 5) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: 2..5 slots (CTAs) per SM");
   P->ffn = flow_variant(K);
   P->fthreads = flow_threads(K);
@@ -2014,7 +2065,9 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
   const int64_t nfrag = S.nfrag;
   std::vector<std::vector<int>> by_frag(nfrag, std::vector<int>(nn, -1));
   for (int i = 0; i < nsub; ++i) by_frag[S.subs[i].frag][S.subs[i].node] = i;
-  const int64_t k = P->pol.pipeline_skew > 0 ? P->pol.pipeline_skew : 1;
+  // skew 0 -> 32: consumers 32 fragments behind their producers in the claim order, so
+  // the tiles a CTA claims are mostly ready (measured best, profiles/r02_flow_sweeps.txt)
+  const int64_t k = P->pol.pipeline_skew > 0 ? P->pol.pipeline_skew : 32;
   P->skew = k;
   // run-ahead window: a source tile of fragment f waits for the leaf tiles of fragments
   // <= f - W; W > dmax * k keeps every window dependency earlier in the global order
@@ -2094,9 +2147,9 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
     fp.role_nslots[r] = rslots[r];
   }
   fp.nslots_sm = K;
-  fp.batch = 4;
+  fp.batch = 1;  // measured best (profiles/r02_flow_sweeps.txt): claim one ticket at a time
   if (const char* ev = getenv("KTILER_FLOW_BATCH")) fp.batch = std::min(32, std::max(1, atoi(ev)));
-  fp.pending = 16;
+  fp.pending = 2;
   if (const char* ev = getenv("KTILER_FLOW_PENDING")) fp.pending = std::min(32, std::max(1, atoi(ev)));
   fp.pending = std::max(fp.pending, fp.batch);
   fp.tb = ktflow::FTrace{P->tb.rec, P->tb.n, P->tb.cap};
@@ -2175,6 +2228,11 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
       return s;
     }
     kt::compute_discards(P->g, P->s);
+    s = ring_analysis(P);
+    if (s) {
+      delete P;
+      return s;
+    }
     build_launches(P);
     if (pol->exec_mode == KTILER_EXEC_GRAPH_DAG || pol->exec_mode == KTILER_EXEC_GRAPH_WAVE) fold_dag_discards(P);
   } catch (const std::bad_alloc&) {
@@ -2421,6 +2479,7 @@ ktiler_status ktiler_execute_host(ktiler_plan_t p, const ktiler_host_copy* in, i
     const kt::Buffer& b = p->g.bufs[c.buf_id];
     int64_t f0 = c.frame0, nf = c.frames ? c.frames : b.d.frames - f0;
     if (f0 < 0 || f0 + nf > b.d.frames || !c.host) return fail(KTILER_E_INVALID, "host copy frame range");
+    if (b.d.ring_frames) return fail(KTILER_E_INVALID, "host copies of a ring buffer (its frames are overwritten)");
     const int64_t rowb = b.d.width * b.d.elem_bytes;
     for (int64_t z = f0; z < f0 + nf; ++z) {
       char* dev = (char*)b.d.base + z * b.d.frame_stride_bytes;

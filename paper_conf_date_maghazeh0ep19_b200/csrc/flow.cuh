@@ -217,7 +217,7 @@ __device__ __forceinline__ unsigned flow_ready(const FParams& p, uint64_t mine, 
 __device__ __forceinline__ void flow_consumer_discard(const FNode& nd, const ktd::Tile& t, int nt, int tid) {
   const int64_t eb = nd.op == 2 ? 2 : 4;
   const int64_t y0 = nd.op == 2 ? 2 * t.y0 : t.y0, nrows = nd.op == 2 ? 2 * (t.y1 - t.y0) : t.y1 - t.y0;
-  const uint8_t* base = nd.in.p + t.z * nd.in.fstride;
+  const uint8_t* base = nd.in.p + ktd::zoff(nd.in, t.z);
   const int64_t b0 = eb * t.x0, b1 = eb * t.x1;
   const int64_t first = ((int64_t)(uintptr_t)(base + y0 * nd.in.pitch + b0) + 127) >> 7;
   const int64_t last = ((int64_t)(uintptr_t)(base + y0 * nd.in.pitch + b1)) >> 7;

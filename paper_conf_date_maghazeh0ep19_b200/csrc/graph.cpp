@@ -236,10 +236,15 @@ ktiler_status ktiler_add_buffer(ktiler_graph_t g, const ktiler_buffer_desc* d, i
   if (b.frame_stride_bytes == 0) b.frame_stride_bytes = b.height * b.pitch_bytes;
   if (b.frame_stride_bytes < b.height * b.pitch_bytes || (b.frame_stride_bytes & 15))
     return fail(KTILER_E_INVALID, "frame_stride_bytes must be >= height*pitch_bytes and a multiple of 16");
+  if (b.ring_frames < 0 || b.ring_frames >= b.frames) b.ring_frames = b.ring_frames < 0 ? -1 : 0;
+  if (b.ring_frames < 0) return fail(KTILER_E_INVALID, "ring_frames must be >= 0");
+  if (b.ring_frames && !(b.flags & KTILER_BUF_INTERNAL))
+    return fail(KTILER_E_INVALID, "a ring buffer (ring_frames > 0) must be INTERNAL: its frames are overwritten");
   Buffer nb;
   nb.d = b;
   nb.addr = (uint64_t)b.base;
-  nb.span = (b.frames - 1) * b.frame_stride_bytes + (b.height - 1) * b.pitch_bytes + b.width * b.elem_bytes;
+  const int64_t slots = b.ring_frames ? b.ring_frames : b.frames;
+  nb.span = (slots - 1) * b.frame_stride_bytes + (b.height - 1) * b.pitch_bytes + b.width * b.elem_bytes;
   nb.line0 = (int64_t)(nb.addr >> 7);
   nb.nlines = (int64_t)((nb.addr + nb.span - 1) >> 7) - nb.line0 + 1;
   for (size_t i = 0; i < g->g.bufs.size(); ++i) {

@@ -33,7 +33,13 @@ namespace ktd {
 struct DBuf {
   uint8_t* p;
   int64_t W, H, pitch, fstride;
+  int32_t ring;  // 0, or a WAR-aware ring of `ring` frames: frame z lives in slot z mod ring
+  int32_t pad;
 };
+// byte offset of frame z in b
+__host__ __device__ __forceinline__ int64_t zoff(const DBuf& b, int64_t z) {
+  return (b.ring ? (int64_t)((uint32_t)z % (uint32_t)b.ring) : z) * b.fstride;
+}
 
 // ---------------------------------------------------------------------------------
 // memory helpers
@@ -63,7 +69,7 @@ __device__ __forceinline__ void discard_line(const void* p) {
 __device__ __forceinline__ int64_t clampi(int64_t v, int64_t lo, int64_t hi) { return v < lo ? lo : (v > hi ? hi : v); }
 __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t s) { return __byte_perm(a, b, s); }
 __device__ __forceinline__ const uint8_t* row_ptr(const DBuf& b, int64_t z, int64_t y) {
-  return b.p + z * b.fstride + y * b.pitch;
+  return b.p + zoff(b, z) + y * b.pitch;
 }
 __device__ __forceinline__ uint4 lds16(const uint8_t* p) { return *reinterpret_cast<const uint4*>(p); }
 __device__ __forceinline__ uint32_t lds4(const uint8_t* p) { return *reinterpret_cast<const uint32_t*>(p); }
@@ -229,7 +235,7 @@ __device__ __forceinline__ void stage_issue_tmap(int op, const CUtensorMap* map,
                                                  const Tile& t, uint8_t* sm, uint64_t* m, bool evict_first = false) {
   const StageGeo g = stage_geo(op, in, t);
   mbar_arrive_expect(m, box_bytes);
-  const int x = (int)(g.xb0 >> 2), y = (int)g.ry0, z = (int)t.z;
+  const int x = (int)(g.xb0 >> 2), y = (int)g.ry0, z = (int)(in.ring ? t.z % in.ring : t.z);
   if (evict_first) {
     const uint64_t pol = policy_evict_first();
     asm volatile(
@@ -358,7 +364,7 @@ __device__ __forceinline__ int rows_per_item(int rows, int nseg, int nt) {
 
 // Output base of a tile (pixel (x0, y0) of frame z) and its "all segments full" flag.
 __device__ __forceinline__ uint8_t* tile_out(const DBuf& out, const Tile& t, int elem) {
-  return out.p + t.z * out.fstride + t.y0 * out.pitch + t.x0 * elem;
+  return out.p + zoff(out, t.z) + t.y0 * out.pitch + t.x0 * elem;
 }
 
 __device__ void gray_compute(const DBuf& out, const Tile& t, const uint8_t* sm, int nt, int tid) {
@@ -692,14 +698,14 @@ __device__ void jacobi_compute(const DBuf& out, const DBuf& coef, const Tile& t,
     const float4 up = *reinterpret_cast<const float4*>(cen - stride + 16);  // row above: 2q, 2q+1
     const float4 dn = *reinterpret_cast<const float4*>(cen + stride + 16);  // row below
     const int64_t y = t.y0 + r, x = px0 + 2 * q;
-    const float4* cp = reinterpret_cast<const float4*>(coef.p + t.z * coef.fstride + y * coef.pitch) + x;
+    const float4* cp = reinterpret_cast<const float4*>(coef.p + zoff(coef, t.z) + y * coef.pitch) + x;
     const float4 c0 = __ldcg(cp), c1 = __ldcg(cp + 1);  // every iteration re-reads them: keep in L2
     // pixel 2q: left 2q-1, right 2q+1;  pixel 2q+1: left 2q, right 2q+2
     const float2 o0 = jacobi_px(make_float2(a.z, a.w), make_float2(b.z, b.w), make_float2(up.x, up.y),
                                 make_float2(dn.x, dn.y), c0, a2);
     const float2 o1 = jacobi_px(make_float2(b.x, b.y), make_float2(c.x, c.y), make_float2(up.z, up.w),
                                 make_float2(dn.z, dn.w), c1, a2);
-    float4* dst = reinterpret_cast<float4*>(out.p + t.z * out.fstride + y * out.pitch) + (x >> 1);
+    float4* dst = reinterpret_cast<float4*>(out.p + zoff(out, t.z) + y * out.pitch) + (x >> 1);
     *dst = make_float4(o0.x, o0.y, o1.x, o1.y);
   }
 }

@@ -21,6 +21,8 @@ inline int64_t floordiv(int64_t a, int64_t b) {  // b > 0
 
 struct Buffer {
   ktiler_buffer_desc d;
+  // byte offset of frame z (a ring buffer keeps frame z in slot z mod ring_frames)
+  int64_t frame_off(int64_t z) const { return (d.ring_frames ? z % d.ring_frames : z) * d.frame_stride_bytes; }
   int64_t span = 0;   // bytes from base to the end of the last frame's last row
   uint64_t addr = 0;  // (uint64_t)base
   int64_t line0 = 0;  // addr >> 7
@@ -135,7 +137,7 @@ void Graph::for_each_line_range(int node, int acc, int64_t bx, int64_t by, int64
   PRect r = access_rect(node, acc, bx, by);
   if (r.empty()) return;
   const int64_t e = b.d.elem_bytes;
-  const uint64_t fb = b.addr + (uint64_t)(bz * b.d.frame_stride_bytes);
+  const uint64_t fb = b.addr + (uint64_t)b.frame_off(bz);
   for (int64_t y = r.y0; y < r.y1; ++y) {
     uint64_t lo = fb + (uint64_t)(y * b.d.pitch_bytes + r.x0 * e);
     uint64_t hi = fb + (uint64_t)(y * b.d.pitch_bytes + r.x1 * e);  // exclusive

@@ -741,7 +741,7 @@ void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_
       const Buffer& B = g.bufs[d.buf];
       for (int64_t z = d.z0; z < d.z1; ++z)
         for (int64_t y = d.y0; y < d.y1; ++y) {
-          uint64_t r = B.addr + (uint64_t)(z * B.d.frame_stride_bytes + y * B.d.pitch_bytes);
+          uint64_t r = B.addr + (uint64_t)(B.frame_off(z) + y * B.d.pitch_bytes);
           int64_t l0 = (int64_t)((r + d.xb0 + 127) >> 7), l1 = (int64_t)((r + d.xb1) >> 7);
           if (l1 > l0) s.discard_lines += l1 - l0;
         }

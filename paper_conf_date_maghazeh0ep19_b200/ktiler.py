@@ -50,7 +50,7 @@ class KtilerError(RuntimeError):
 class BufferDesc(ctypes.Structure):
     _fields_ = [("base", ctypes.c_void_p), ("width", ctypes.c_int64), ("height", ctypes.c_int64),
                 ("frames", ctypes.c_int64), ("pitch_bytes", ctypes.c_int64), ("frame_stride_bytes", ctypes.c_int64),
-                ("elem_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32)]
+                ("elem_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32), ("ring_frames", ctypes.c_int64)]
 
 
 class Access(ctypes.Structure):
@@ -170,7 +170,7 @@ def lib() -> ctypes.CDLL:
         f = getattr(L, name)
         f.argtypes = args
         f.restype = res
-    if L.ktiler_abi_version() != 1:
+    if L.ktiler_abi_version() != 2:
         raise RuntimeError("libktiler ABI version mismatch")
     _LIB = L
     return L
@@ -209,10 +209,11 @@ class Graph:
             pass
 
     def add_buffer(self, base: int, width: int, height: int, elem_bytes: int, frames: int = 1,
-                   pitch_bytes: int | None = None, frame_stride_bytes: int = 0, internal: bool = False) -> int:
+                   pitch_bytes: int | None = None, frame_stride_bytes: int = 0, internal: bool = False,
+                   ring_frames: int = 0) -> int:
         pitch = pitch_bytes if pitch_bytes is not None else width * elem_bytes
         d = BufferDesc(base, width, height, frames, pitch, frame_stride_bytes, elem_bytes,
-                       BUF_INTERNAL if internal else 0)
+                       BUF_INTERNAL if internal else 0, ring_frames)
         out = ctypes.c_int32()
         _check(lib().ktiler_add_buffer(self._h, ctypes.byref(d), ctypes.byref(out)))
         return out.value

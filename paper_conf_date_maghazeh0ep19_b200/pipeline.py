@@ -68,19 +68,24 @@ class _GraphBuilder:
         self.store = _Store(device)
         self.g = K.Graph()
         self.bufs = {}  # name -> (id, W, H, F, elem, pitch)
+        self.slots = {}  # name -> frames of storage (< F for a ring buffer)
         self.nodes = {}
         self.grids = {}
         self.pitch_align = pitch_align
         self.bases = bases or {}
 
-    def buffer(self, name, W, H, F, elem, internal):
+    def buffer(self, name, W, H, F, elem, internal, ring=0):
+        """ring > 0 (internal buffers): storage for `ring` frames, frame z in slot z mod ring
+        (ktiler_buffer_desc.ring_frames)."""
         pitch = _round(W * elem, self.pitch_align)
+        ring = ring if internal and 0 < ring < F else 0
         if name in self.bases:
             addr = self.bases[name]
         else:
-            addr = self.store.alloc(name, F, H, pitch)
-        bid = self.g.add_buffer(addr, W, H, elem, frames=F, pitch_bytes=pitch, internal=internal)
+            addr = self.store.alloc(name, ring or F, H, pitch)
+        bid = self.g.add_buffer(addr, W, H, elem, frames=F, pitch_bytes=pitch, internal=internal, ring_frames=ring)
         self.bufs[name] = (bid, W, H, F, elem, pitch)
+        self.slots[name] = ring or F  # frames of storage (views)
         return bid
 
     def kernel(self, name, op, src, dst, tile, threads, halo=0, scale=1, params=None):
@@ -100,6 +105,7 @@ class _GraphBuilder:
         """torch view [F, H, W(, 3)] of a buffer (device mode only)."""
         import torch
         bid, W, H, F, elem, pitch = self.bufs[name]
+        F = self.slots.get(name, F)
         t = self.store.tensors[name].view(F, H, pitch)[:, :, :W * elem]
         if elem == 3:
             return t.view(F, H, W, 3) if pitch == W * 3 else t.unflatten(2, (W, 3))
@@ -114,7 +120,7 @@ class Pipeline:
     NODE_ORDER = ("gray", "blur", "down", "sobel", "thresh")
 
     def __init__(self, W: int, H: int, frames: int = 1, T: float = 200.0, device="cuda", geometry=None,
-                 internal: bool = True, pitch_align: int = 128, bases=None):
+                 internal: bool = True, pitch_align: int = 128, bases=None, ring_frames: int = 0):
         if W % 2 or H % 2:
             raise ValueError("down2 needs even W and H (SURVEY A3)")
         self.W, self.H, self.F, self.T = W, H, frames, T
@@ -126,10 +132,11 @@ class Pipeline:
         b = _GraphBuilder(device, pitch_align, bases)
         self.b = b
         b.buffer("rgb", W, H, frames, 3, internal=False)
-        b.buffer("gray", W, H, frames, 1, internal=internal)
-        b.buffer("blur", W, H, frames, 1, internal=internal)
-        b.buffer("down", W // 2, H // 2, frames, 1, internal=internal)
-        b.buffer("sob", W // 2, H // 2, frames, 4, internal=internal)
+        # ring_frames > 0: the four intermediates are WAR-aware rings of that many frames
+        b.buffer("gray", W, H, frames, 1, internal=internal, ring=ring_frames)
+        b.buffer("blur", W, H, frames, 1, internal=internal, ring=ring_frames)
+        b.buffer("down", W // 2, H // 2, frames, 1, internal=internal, ring=ring_frames)
+        b.buffer("sob", W // 2, H // 2, frames, 4, internal=internal, ring=ring_frames)
         b.buffer("mask", W // 2, H // 2, frames, 1, internal=False)
 
         def thr(n):

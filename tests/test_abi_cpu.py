@@ -28,7 +28,7 @@ def test_exports_every_header_symbol(K):
     for n in names:
         assert hasattr(lib, n), n
     assert set(K.EXPORTS) <= set(names)
-    assert lib.ktiler_abi_version() == 1
+    assert lib.ktiler_abi_version() == 2
     assert lib.ktiler_status_str(3).decode() == "KTILER_E_UNTILEABLE"
 
 
@@ -339,3 +339,57 @@ def test_flow_roles_abi(K):
     with pytest.raises(K.KtilerError) as e:
         dag.set_flow_roles([0] * 5, [0, 0])
     assert e.value.status == K.E_STATE
+
+
+def _frames_of(sk):
+    return {z for (x0, y0, z0, x1, y1, z1) in sk["rects"] for z in range(z0, z1)}
+
+
+@pytest.mark.parametrize("ring", [1, 2, 3])
+def test_ring_buffers_war_order(K, ring):
+    """Ring intermediates (ktiler_buffer_desc.ring_frames): the total
+    order of an accepted plan puts every read of frame z - R before every write of frame z
+    (write-after-read, the hazard PAPER.md:193's RAW model lacks); a plan whose fragments
+    span R frames or more is refused (KTILER_E_UNTILEABLE) instead of racing."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 64, 32, 6
+    geo = SMALL
+    p = Pipeline(W, H, F, device=None, geometry=geo, internal=True, ring_frames=ring)
+    names = ("gray", "blur", "down", "sobel", "thresh")
+    reads = {1: "gray", 2: "blur", 3: "down", 4: "sob"}   # node -> ring buffer it reads
+    writes = {0: "gray", 1: "blur", 2: "down", 3: "sob"}  # node -> ring buffer it writes
+    accepted = 0
+    for budget in (16000, 24000, 40000):
+        try:
+            plan = p.plan(budget, kind="budget", exec_mode="graph")
+        except K.KtilerError as e:
+            assert e.status == K.E_UNTILEABLE
+            continue
+        accepted += 1
+        subs = plan.subkernels()
+        for buf in ("gray", "blur", "down", "sob"):
+            last_read, first_write = {}, {}
+            for i, sk in enumerate(subs):
+                for z in _frames_of(sk):
+                    if reads.get(sk["node"]) == buf:
+                        last_read[z] = i
+                    if writes.get(sk["node"]) == buf:
+                        first_write.setdefault(z, i)
+            for z in range(ring, F):
+                assert first_write[z] > last_read[z - ring], (buf, z, budget)
+    assert accepted >= 2
+    # a whole-batch fragment (budget = infinity) spans every frame: a ring must refuse it
+    with pytest.raises(K.KtilerError) as e:
+        p.plan(0 + (1 << 40), kind="budget", exec_mode="graph")
+    assert e.value.status == K.E_UNTILEABLE
+    with pytest.raises(K.KtilerError) as e:  # executors without WAR support
+        p.plan(6000, kind="budget", exec_mode="chain")
+    assert e.value.status in (K.E_UNSUPPORTED, K.E_UNTILEABLE)
+
+
+def test_ring_buffer_validation(K):
+    from paper_conf_date_maghazeh0ep19_b200 import ktiler as KK
+    g = KK.Graph()
+    with pytest.raises(KK.KtilerError):  # a ring must be INTERNAL
+        g.add_buffer(1 << 20, 64, 32, 1, frames=4, ring_frames=2)
+    g.add_buffer(1 << 20, 64, 32, 1, frames=4, internal=True, ring_frames=2)

@@ -368,3 +368,31 @@ def test_alg1_calibrated_plan():
         p.run()
         torch.cuda.synchronize()
         assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(rgb, T=40.0)["mask"])
+
+
+@pytest.mark.parametrize("ring", [1, 2, 3])
+@pytest.mark.parametrize("mode,pol", [("stream", dict()), ("graph", dict(discard=True)),
+                                      ("dag", dict(window=2, consumer_discard=True)),
+                                      ("dag", dict(window=3, resident_budget=True))],
+                         ids=["stream", "graph-discard", "dag-w2-cd", "dag-w3"])
+def test_ring_intermediates(ring, mode, pol):
+    """§8(f) f4: the four intermediates as WAR-aware rings of `ring` frames (frame z in slot
+    z mod ring).  The executors order every write of frame z after every read of frame
+    z - ring (GRAPH_DAG: WAR edges; total orders: checked at plan time), so the whole batch
+    — 6 frames through 1..3 frames of intermediate storage — equals the oracle, over
+    repeated executes with alternating inputs."""
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 512, 128, 6
+    a, b = synth.scene(3, W, H, F), synth.uniform(4, W, H, F)
+    p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL, ring_frames=ring)
+    for k in ("gray", "blur", "down", "sob"):
+        assert p.view(k).shape[0] == ring  # the storage really is a ring
+    # 4 of a frame's 8 leaf block-rows per fragment: fragments never straddle two frames
+    plan = p.plan(1 << 20, kind="rows", rows=4, exec_mode=mode, **pol)
+    assert plan.num_fragments() == 2 * F
+    for it in range(3):
+        x = a if it % 2 == 0 else b
+        p.view("rgb").copy_(torch.from_numpy(x))
+        p.run()
+        torch.cuda.synchronize()
+        assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(x, T=40.0)["mask"]), (ring, mode, it)

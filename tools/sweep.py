@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--configs", default="default", help="default | json list of plan kwargs")
     ap.add_argument("--geom", default="", help='json {op: [tile_w, tile_h, threads]} overriding B200_GEOMETRY')
     ap.add_argument("--check", action="store_true", help="compare every config's mask with the untiled graph's")
+    ap.add_argument("--ring", type=int, default=0, help="intermediates as rings of this many frames (f4)")
     args = ap.parse_args()
     import torch
 
@@ -35,7 +36,7 @@ def main():
         from paper_conf_date_maghazeh0ep19_b200.pipeline import B200_GEOMETRY
         geom = dict(B200_GEOMETRY)
         geom.update({k: tuple(v) for k, v in json.loads(args.geom).items()})
-    p = Pipeline(args.W, args.H, args.F, internal=True, geometry=geom)
+    p = Pipeline(args.W, args.H, args.F, internal=True, geometry=geom, ring_frames=args.ring)
     s = torch.cuda.current_stream()
     G.fill("scene", 1234, p.view("rgb").data_ptr(), args.W * 3, args.W * 3 * args.H, args.W, args.H, F=args.F,
            stream=s.cuda_stream)
@@ -52,11 +53,14 @@ def main():
     pix = args.W * args.H * args.F
     ref = None
     if args.check:
-        pl = p.b.g.plan(0, kind="none", exec_mode="graph")
+        ref_pipe = Pipeline(args.W, args.H, args.F, internal=True, geometry=geom) if args.ring else p
+        if args.ring:
+            ref_pipe.view("rgb").copy_(p.view("rgb"))
+        pl = ref_pipe.b.g.plan(0, kind="none", exec_mode="graph")
         pl.execute(s.cuda_stream)
         torch.cuda.synchronize()
-        ref = p.view("mask").clone()
-        del pl
+        ref = ref_pipe.view("mask").clone()
+        del pl, ref_pipe
     for c in cfgs:
         try:
             c = dict(c)
