@@ -550,6 +550,18 @@ def main():
                            "roofline_frac": 9.75 * pix / (ms_un / 1000) / 1e9 / peak,
                            "algorithmic_bytes": "9.75 B/px (every intermediate written and read once)"}
         del un
+    if not args.no_untiled and sp is None and not args.ring_frames and args.mode != "flow":
+        # the persistent executor driven by per-tile dependency flags (north star's variant,
+        # KTILER_EXEC_FLOW, its measured-best defaults) on the same batch, for comparison
+        try:
+            fl = p.b.g.plan(0, kind="rows", rows=1, exec_mode="flow", consumer_discard=True)
+            ms_fl = timed(lambda: fl.execute(s), max(3, args.steps // 4), 2)
+            line["flow"] = {"value": pix / (ms_fl / 1000) / 1e6, "ms_per_step": ms_fl,
+                            "vs_untiled": line["untiled"]["ms_per_step"] / ms_fl,
+                            "policy": "rows=1 fragments, 3 CTAs/SM one role, skew 32, consumer discard"}
+            del fl
+        except Exception as e:  # diagnostics only
+            line["flow"] = {"error": str(e)}
     if not args.no_trace and rank == 0:
         try:
             tiled_sh, tiled_span, per_node = trace_shares(p, pol) if args.mode != "persistent" else (None, None, None)

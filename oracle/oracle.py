@@ -21,8 +21,11 @@ Contents (ids O-n):
   by step in the paper's order and notation, with readings A11–A19.
 * O-11 ``validate_schedule``: partition, dependency order
   (PAPER.md:171, 271), cache constraint.
-* O-12 ``lru_dram_bytes``: fully-associative LRU line model (expectation only,
-  not a parity target — "parity unpinned" for anything it predicts).
+* O-12 ``lru_dram_bytes``: fully-associative LRU line model, write-back,
+  write-allocate, optional discard; pinned to hand-worked traces (every read miss,
+  dirty eviction and dirty tail counted by hand, tests/test_oracle_schedule.py).  What
+  it predicts for a real B200 (whose L2 is neither fully associative nor LRU) is an
+  expectation, not a parity claim.
 * O-13 ``application_tiling``: Alg. 1 with performance tables.
 * O-14 ``hs_jacobi``: K Horn–Schunck Jacobi iterations, the paper's JI nodes
   (SURVEY §8(f) f2), in f32 (the GPU's exact operation order) or f64.

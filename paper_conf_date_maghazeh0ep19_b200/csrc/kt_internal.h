@@ -190,6 +190,7 @@ struct Schedule {
 ktiler_status halo_exchange(ktiler_comm_s* c, int32_t rank, int32_t halo_rows, void* stream);
 
 ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out);
+ktiler_status build_schedule_core(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out);
 void compute_discards(const Graph& g, Schedule& s, std::vector<int32_t>* sub_of_block = nullptr);
 
 }  // namespace kt

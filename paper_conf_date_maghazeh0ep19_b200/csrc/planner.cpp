@@ -536,7 +536,80 @@ static ktiler_status alg1(Graph& g, int64_t budget_lines, double thld, bool resi
   return KTILER_OK;
 }
 
+// KTILER_PF_MULTIRATE: cheap nodes (output pixels <= 1/4 of the largest node's, closed
+// under "all consumers are cheap too") get one sub-kernel per two fragments: the one of
+// fragment 2k is merged into that of fragment 2k+1 (emitted at 2k+1's place, in the same
+// topological position).  Only consumers move later, so every RAW dependency still points
+// to an earlier sub-kernel.  sub_deps / discards are derived afterwards.
+static void multirate(const Graph& g, Schedule& s) {
+  const int nn = (int)g.nodes.size();
+  std::vector<double> pix(nn, 0.0);
+  double maxpix = 0;
+  for (int v = 0; v < nn; ++v) {
+    const Node& n = g.nodes[v];
+    const Buffer& b = g.bufs[n.acc[n.wacc].buf];
+    pix[v] = (double)b.d.width * b.d.height * b.d.frames;
+    maxpix = std::max(maxpix, pix[v]);
+  }
+  std::vector<uint8_t> cheap(nn, 0);
+  for (int v = 0; v < nn; ++v) cheap[v] = 4.0 * pix[v] <= maxpix;
+  for (bool changed = true; changed;) {  // close downward
+    changed = false;
+    for (int v = 0; v < nn; ++v)
+      if (cheap[v])
+        for (const Chan& c : g.out_ch[v])
+          if (!cheap[c.v]) {
+            cheap[v] = 0;
+            changed = true;
+          }
+  }
+  bool any = false;
+  for (int v = 0; v < nn; ++v) any |= cheap[v] != 0;
+  if (!any || s.nfrag < 2) return;
+  std::vector<SubKernel> out;
+  std::vector<int> pending(nn, -1);  // index into s.subs of a deferred sub-kernel
+  std::vector<SubKernel>& in = s.subs;
+  size_t i = 0;
+  while (i < in.size()) {
+    const int32_t f = in[i].frag;
+    size_t j = i;
+    while (j < in.size() && in[j].frag == f) ++j;
+    const bool last_frag = j == in.size();
+    for (size_t k = i; k < j; ++k) {
+      const int v = in[k].node;
+      if (!cheap[v]) {
+        out.push_back(in[k]);
+        continue;
+      }
+      if (pending[v] < 0 && (f % 2 == 0) && !last_frag) {
+        pending[v] = (int)k;  // defer to the next odd fragment
+        continue;
+      }
+      SubKernel m = in[k];
+      if (pending[v] >= 0) {
+        const SubKernel& p = in[pending[v]];
+        m.rects.insert(m.rects.begin(), p.rects.begin(), p.rects.end());
+        m.nblocks += p.nblocks;
+        m.footprint = std::max(m.footprint, p.footprint);
+        pending[v] = -1;
+      }
+      out.push_back(std::move(m));
+    }
+    i = j;
+  }
+  for (int v = 0; v < nn; ++v)  // a deferred sub-kernel with no later fragment of its node
+    if (pending[v] >= 0) out.push_back(in[pending[v]]);
+  s.subs.swap(out);
+}
+
 ktiler_status build_schedule(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out) {
+  ktiler_status st0 = build_schedule_core(g, cache_bytes, pol, out);
+  if (st0 || !(pol.flags & KTILER_PF_MULTIRATE) || pol.kind == KTILER_FRAG_NONE) return st0;
+  multirate(g, out);
+  return KTILER_OK;
+}
+
+ktiler_status build_schedule_core(Graph& g, int64_t cache_bytes, const ktiler_fragment_policy& pol, Schedule& out) {
   ktiler_status s = g.finalize();
   if (s) return s;
   out = Schedule();

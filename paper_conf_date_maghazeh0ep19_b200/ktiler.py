@@ -22,6 +22,7 @@ FRAG_BUDGET, FRAG_ROWS, FRAG_BALANCED, FRAG_NONE, FRAG_ALG1, FRAG_CHAIN = range(
 EXEC_STREAM, EXEC_GRAPH, EXEC_GRAPH_PERSIST_L2, EXEC_PERSISTENT, EXEC_GRAPH_DAG, EXEC_GRAPH_CHAIN, EXEC_GRAPH_WAVE, \
     EXEC_FLOW = range(8)
 PF_DISCARD_DEAD, PF_PDL, PF_FORCE_MINIMAL, PF_RESIDENT_BUDGET, PF_CONSUMER_DISCARD, PF_HALO_DISCARD = 1, 2, 4, 8, 16, 32
+PF_MULTIRATE = 64
 
 EXEC_MODES = {"stream": EXEC_STREAM, "graph": EXEC_GRAPH, "persist_l2": EXEC_GRAPH_PERSIST_L2,
               "persistent": EXEC_PERSISTENT, "dag": EXEC_GRAPH_DAG, "chain": EXEC_GRAPH_CHAIN,
@@ -279,12 +280,13 @@ class Graph:
     def plan(self, cache_bytes: int = 0, kind: str | int = "budget", l2_fraction: float = 1.0, rows: int = 1,
              exec_mode: str | int = "graph", discard: bool = False, pdl: bool = False, force_minimal: bool = False,
              persistent_ctas: int = 0, skew: int = 0, window: int = 0, resident_budget: bool = False,
-             alg1_thld: float = 0.0, consumer_discard: bool = False, halo_discard: bool = False) -> "Plan":
+             alg1_thld: float = 0.0, consumer_discard: bool = False, halo_discard: bool = False,
+             multirate: bool = False) -> "Plan":
         k = FRAG_KINDS[kind] if isinstance(kind, str) else kind
         m = EXEC_MODES[exec_mode] if isinstance(exec_mode, str) else exec_mode
         flags = (PF_DISCARD_DEAD if discard else 0) | (PF_PDL if pdl else 0) | (PF_FORCE_MINIMAL if force_minimal else 0) \
             | (PF_RESIDENT_BUDGET if resident_budget else 0) | (PF_CONSUMER_DISCARD if consumer_discard else 0) \
-            | (PF_HALO_DISCARD if halo_discard else 0)
+            | (PF_HALO_DISCARD if halo_discard else 0) | (PF_MULTIRATE if multirate else 0)
         pol = Policy(k, l2_fraction, rows, m, flags, persistent_ctas, skew, window, alg1_thld)
         h = ctypes.c_void_p()
         _check(lib().ktiler_plan(self._h, cache_bytes, ctypes.byref(pol), ctypes.byref(h)))

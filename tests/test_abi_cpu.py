@@ -393,3 +393,26 @@ def test_ring_buffer_validation(K):
     with pytest.raises(KK.KtilerError):  # a ring must be INTERNAL
         g.add_buffer(1 << 20, 64, 32, 1, frames=4, ring_frames=2)
     g.add_buffer(1 << 20, 64, 32, 1, frames=4, internal=True, ring_frames=2)
+
+
+@pytest.mark.parametrize("W,H,F,geo", GEOS[:2], ids=lambda v: str(v) if not isinstance(v, dict) else "")
+def test_multirate_schedule_valid(K, W, H, F, geo):
+    """KTILER_PF_MULTIRATE: the cheap half-resolution nodes (down2, sobel3, thresh: 1/4 of
+    gray's pixels, all consumers cheap) run one sub-kernel per two fragments; the schedule
+    is still a partition whose order respects every traced RAW dependency (O-11), and the
+    expensive nodes keep one sub-kernel per fragment."""
+    og, p = _pipe_pair(W, H, F, geo)
+    tr = O.trace(og)
+    base = p.plan(1 << 20, kind="rows", rows=1, exec_mode="stream")
+    mr = p.plan(1 << 20, kind="rows", rows=1, exec_mode="stream", multirate=True)
+    subs0, subs1 = _blocks_by_sub(base), _blocks_by_sub(mr)
+    nfrag = base.num_fragments()
+    assert nfrag >= 3
+    assert not O.validate_schedule(og, tr, [(n, b) for n, b, _ in subs1])
+    for v in range(5):
+        n0 = sum(1 for n, _, _ in subs0 if n == v)
+        n1 = sum(1 for n, _, _ in subs1 if n == v)
+        if v < 2:
+            assert n1 == n0
+        else:
+            assert n1 == -(-n0 // 2)

@@ -396,3 +396,19 @@ def test_ring_intermediates(ring, mode, pol):
         p.run()
         torch.cuda.synchronize()
         assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(x, T=40.0)["mask"]), (ring, mode, it)
+
+
+@pytest.mark.parametrize("mode,pol", [("dag", dict(kind="budget", window=2, resident_budget=True, consumer_discard=True)),
+                                      ("graph", dict(kind="budget", discard=True)),
+                                      ("flow", dict(kind="rows", rows=1, consumer_discard=True))],
+                         ids=["dag", "graph-discard", "flow"])
+def test_multirate_bit_exact(mode, pol):
+    """KTILER_PF_MULTIRATE (down2 / sobel3 / thresh: one sub-kernel per two fragments) in
+    the bench's executor and two others: bit-exact vs the oracle."""
+    rgb = synth.scene(12, 1040, 256, 2)
+    pol = dict(pol)
+    kind = pol.pop("kind")
+    out, plan = _run(1040, 256, 2, rgb, T=40.0, cache_bytes=200 * 1024, internal=True, kind=kind, exec_mode=mode,
+                     multirate=True, **pol)
+    assert plan.num_fragments() > 2
+    assert np.array_equal(out["mask"], O.pipeline(rgb, T=40.0)["mask"])
