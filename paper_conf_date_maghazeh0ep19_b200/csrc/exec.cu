@@ -2248,6 +2248,41 @@ ktiler_status ktiler_plan(ktiler_graph_t gh, size_t cache_bytes, const ktiler_fr
 
 void ktiler_plan_destroy(ktiler_plan_t p) { delete p; }
 
+ktiler_status ktiler_plan_reorder(ktiler_plan_t p, const int64_t* order, int64_t n) {
+  if (!p || !order) return fail(KTILER_E_INVALID, "NULL argument");
+  if (p->executed || p->device >= 0) return fail(KTILER_E_STATE, "reorder before the first execute");
+  kt::Schedule& S = p->s;
+  const int64_t nsub = (int64_t)S.subs.size();
+  if (n != nsub) return fail(KTILER_E_INVALID, "order must list every sub-kernel once");
+  std::vector<int64_t> pos(nsub, -1);
+  for (int64_t k = 0; k < n; ++k) {
+    if (order[k] < 0 || order[k] >= nsub || pos[order[k]] >= 0) return fail(KTILER_E_INVALID, "order is not a permutation");
+    pos[order[k]] = k;
+  }
+  // a valid schedule: every sub-kernel after all sub-kernels it depends on
+  for (int64_t i = 0; i < nsub; ++i)
+    for (int32_t d : S.sub_deps[i])
+      if (pos[d] >= pos[i])
+        return fail(KTILER_E_INVALID, "order puts sub-kernel " + std::to_string(i) + " before sub-kernel " +
+                                          std::to_string(d) + " it depends on (PAPER.md:271)");
+  std::vector<kt::SubKernel> subs(nsub);
+  for (int64_t k = 0; k < n; ++k) subs[k] = S.subs[order[k]];
+  S.subs.swap(subs);
+  // everything derived from the order: sub-kernel deps, last readers / discard lists, ring
+  // WAR order, launches
+  S.discards.clear();
+  S.discard_lines = 0;
+  kt::compute_discards(p->g, S);
+  ktiler_status st = ring_analysis(p);
+  if (st) return st;
+  p->launches.clear();
+  p->dag_disc.clear();
+  build_launches(p);
+  if (p->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || p->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE) fold_dag_discards(p);
+  kt::clear_error();
+  return KTILER_OK;
+}
+
 ktiler_status ktiler_plan_attach_halo(ktiler_plan_t p, ktiler_comm_t c, int32_t rank, int32_t halo_rows) {
   if (!p || !c || rank < 0 || halo_rows < 0) return fail(KTILER_E_INVALID, "bad argument");
   if (p->executed || p->device >= 0) return fail(KTILER_E_STATE, "attach the halo exchange before the first execute");

@@ -115,7 +115,7 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint",
            "ktiler_plan_set_flow_roles", "ktiler_comm_unique_id", "ktiler_comm_init_nccl",
            "ktiler_comm_init_loopback", "ktiler_comm_destroy", "ktiler_comm_register_strip", "ktiler_halo_exchange",
-           "ktiler_plan_attach_halo"]
+           "ktiler_plan_attach_halo", "ktiler_plan_reorder"]
 
 _LIB = None
 
@@ -166,6 +166,7 @@ def lib() -> ctypes.CDLL:
         "ktiler_comm_register_strip": ([vp, i32, P(Strip)], st),
         "ktiler_halo_exchange": ([vp, i32, i32, vp], st),
         "ktiler_plan_attach_halo": ([vp, vp, i32, i32], st),
+        "ktiler_plan_reorder": ([vp, P(i64), i64], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -388,6 +389,12 @@ class Plan:
         nr, sr = list(node_role), list(slot_role)
         _check(lib().ktiler_plan_set_flow_roles(self._h, (ctypes.c_int32 * max(1, len(nr)))(*nr), len(nr),
                                                 (ctypes.c_int32 * max(1, len(sr)))(*sr), len(sr)))
+
+    def reorder(self, order) -> None:
+        """Run the sub-kernels in another dependency-respecting total order
+        (include/ktiler.h ktiler_plan_reorder); order[k] = current index of the k-th."""
+        o = list(order)
+        _check(lib().ktiler_plan_reorder(self._h, (ctypes.c_int64 * max(1, len(o)))(*o), len(o)))
 
     def attach_halo(self, comm: "Comm", rank: int, halo_rows: int) -> None:
         """Run rank's strip exchange first in every execute, inside the plan's CUDA graph

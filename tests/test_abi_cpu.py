@@ -416,3 +416,73 @@ def test_multirate_schedule_valid(K, W, H, F, geo):
             assert n1 == n0
         else:
             assert n1 == -(-n0 // 2)
+
+
+def _sub_deps(graph, subs):
+    """sub-kernel -> set of sub-kernels it depends on, from the library's block deps."""
+    owner = {}
+    for i, sk in enumerate(subs):
+        for (x0, y0, z0, x1, y1, z1) in sk["rects"]:
+            for z in range(z0, z1):
+                for y in range(y0, y1):
+                    for x in range(x0, x1):
+                        owner[(sk["node"], x, y, z)] = i
+    deps = []
+    for i, sk in enumerate(subs):
+        d = set()
+        for (x0, y0, z0, x1, y1, z1) in sk["rects"]:
+            for z in range(z0, z1):
+                for y in range(y0, y1):
+                    for x in range(x0, x1):
+                        for (u, px, py, pz) in graph.block_deps(sk["node"], x, y, z):
+                            d.add(owner[(u, px, py, pz)])
+        d.discard(i)
+        deps.append(d)
+    return deps
+
+
+def random_topo_orders(deps, k, seed):
+    import random
+    rnd = random.Random(seed)
+    n = len(deps)
+    succ = [[] for _ in range(n)]
+    for i, d in enumerate(deps):
+        for j in d:
+            succ[j].append(i)
+    out = []
+    for _ in range(k):
+        indeg = [len(d) for d in deps]
+        ready = [i for i in range(n) if indeg[i] == 0]
+        order = []
+        while ready:
+            i = ready.pop(rnd.randrange(len(ready)))
+            order.append(i)
+            for s in succ[i]:
+                indeg[s] -= 1
+                if indeg[s] == 0:
+                    ready.append(s)
+        out.append(order)
+    return out
+
+
+def test_plan_reorder_validation(K):
+    """ktiler_plan_reorder: any dependency-respecting order is accepted (and becomes the
+    plan's order), an order that runs a consumer before its producer is refused."""
+    og, p = _pipe_pair(64, 96, 2, SMALL)
+    plan = p.plan(20000, kind="budget", exec_mode="stream")
+    subs = plan.subkernels()
+    deps = _sub_deps(p.graph, subs)
+    order = random_topo_orders(deps, 1, 5)[0]
+    plan.reorder(order)
+    got = plan.subkernels()
+    assert [(s["node"], s["rects"]) for s in got] == [(subs[i]["node"], subs[i]["rects"]) for i in order]
+    plan2 = p.plan(20000, kind="budget", exec_mode="stream")
+    bad = list(range(len(subs)))
+    i = next(i for i in range(len(subs)) if deps[i])
+    j = min(deps[i])
+    bad[i], bad[j] = bad[j], bad[i]  # consumer i now runs before its producer j
+    with pytest.raises(K.KtilerError) as e:
+        plan2.reorder(bad)
+    assert e.value.status == K.E_INVALID
+    with pytest.raises(K.KtilerError):
+        plan2.reorder([0] * len(subs))  # not a permutation

@@ -7,6 +7,8 @@ Two tile geometries: the B200 geometry bench.py uses (pipeline.B200_GEOMETRY: 51
 256x32 tiles) and a SMALL geometry whose tiles are small enough that images of a few
 hundred pixels split into tens of fragments, so tiling, fragment edges, ragged Alg. 2
 fragments and discards are exercised at sizes the oracle finishes in seconds."""
+import os
+
 import numpy as np
 import pytest
 
@@ -412,3 +414,31 @@ def test_multirate_bit_exact(mode, pol):
                      multirate=True, **pol)
     assert plan.num_fragments() > 2
     assert np.array_equal(out["mask"], O.pipeline(rgb, T=40.0)["mask"])
+
+
+@pytest.mark.parametrize("mode,discard", [("stream", True), ("graph", True), ("dag", False)])
+def test_random_linear_extensions(mode, discard):
+    """P10 on the GPU: random dependency-respecting total orders of the plan's
+    sub-kernels (ktiler_plan_reorder; last readers and discard lists re-derived per order),
+    replayed on poisoned intermediates, all give the oracle's result — including with
+    dead-line discards, where a wrong last reader would drop lines still to be read."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from test_abi_cpu import _sub_deps, random_topo_orders
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 640, 160, 2
+    rgb = synth.scene(21, W, H, F)
+    ref = O.pipeline(rgb, T=40.0)
+    p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
+    p.view("rgb").copy_(torch.from_numpy(rgb))
+    subs = p.plan(150 * 1024, kind="budget", exec_mode=mode, discard=discard).subkernels()
+    assert len(subs) > 20
+    deps = _sub_deps(p.graph, subs)
+    for order in random_topo_orders(deps, 6, seed=7):
+        for k in KEYS:
+            p.b.store.tensors[k].fill_(0xA5)
+        plan = p.plan(150 * 1024, kind="budget", exec_mode=mode, discard=discard)  # same shapes -> same plan
+        plan.reorder(order)
+        p.run()
+        torch.cuda.synchronize()
+        assert np.array_equal(p.view("mask").cpu().numpy(), ref["mask"]), order[:12]
