@@ -665,7 +665,7 @@ def main():
                        "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                        "path": (e2e_path or "ktiler_execute_host (pinned host rgb -> device -> plan -> host mask)")
                        if sp is None else "pinned host rows -> device, halo exchange, ktiler_execute, mask -> host"}
-    if rank == 0 and world == 1 and not args.no_ncu and sp is None:
+    if rank == 0 and world == 1 and not args.no_ncu:  # (a one-rank strip is the whole image)
         # DRAM bytes and L2 hit rate of the tiled step and of the untiled one, measured by
         # ncu on this run's exact configuration (the metric's "DRAM bytes & L2 hit rate")
         if args.ring_frames:  # the untiled schedule needs full-batch intermediates

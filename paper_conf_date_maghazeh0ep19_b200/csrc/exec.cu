@@ -33,6 +33,7 @@ namespace {
 
 using ktd::DBuf;
 constexpr int MAXR = 4, MAXD = 8;
+constexpr int KMAXST = 4;  // staging ring depth of the op kernels (KParams::nstage)
 constexpr int PCOMP_WARPS = 4;  // compute warps per persistent CTA (+ producer + publisher warp)
 constexpr int PCOMP_THREADS = 32 * PCOMP_WARPS;
 constexpr int PSTAGES_MAX = 12;   // staging ring depth (slots that fit the CTA's share of smem)
@@ -91,7 +92,9 @@ struct KParams {
   unsigned int* hcnt;       // [frames][pgy][pgx] readers so far (reset to 0 by the last one)
   const uint8_t* hneed;     // [pgy][pgx] consumer blocks reading each producer block
   int32_t nrect, ndisc, pdl;
-  int64_t stage_bytes;  // one of the two staging buffers
+  int64_t stage_bytes;  // one staging buffer (slot) of the ring
+  int32_t nstage;       // ring depth (2..KMAXST)
+  int32_t pad_ns;
   LRect r[MAXR];
   int64_t rpre[MAXR + 1];
   DRect d[MAXD];
@@ -270,7 +273,10 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
   }
 }
 
-template <int OP, bool SCALAR>
+// NST: staging ring depth; 2 (compile time, the default code path) or 0 = p.nstage at run
+// time (KTILER_STAGES variants of the L2-fed consumers, instantiated for down2 / sobel3 /
+// thresh only)
+template <int OP, bool SCALAR, int NST = 2>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ unsigned int s_epoch;
@@ -304,15 +310,16 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       }
     }
   } else {
-    // Grid-stride over the launch's tiles with two shared buffers: the TMA bulk copies of
-    // tile i+2 stream in while tile i+1 computes.
+    // Grid-stride over the launch's tiles with a ring of S = p.nstage shared buffers (2 by
+    // default; deeper for L2-fed sub-kernels, KTILER_STAGES): the TMA copies of the next
+    // S - 1 tiles stream in while one computes.
     extern __shared__ __align__(128) uint8_t ktsm[];
-    __shared__ __align__(8) uint64_t mbar[2];
-    __shared__ ktd::Tile s_tile[2];  // decoded once by warp 0, read by all after the mbarrier
-    __shared__ uint64_t s_tw[2];     // trace (chain): producers ready
+    __shared__ __align__(8) uint64_t mbar[KMAXST];
+    __shared__ ktd::Tile s_tile[KMAXST];  // decoded once by warp 0, read by all after the mbarrier
+    __shared__ uint64_t s_tw[KMAXST];     // trace (chain): producers ready
+    const int S = NST ? NST : (p.nstage < 2 ? 2 : (p.nstage > KMAXST ? KMAXST : p.nstage));
     if (tid == 0) {
-      ktd::mbar_init(&mbar[0], 1);
-      ktd::mbar_init(&mbar[1], 1);
+      for (int j = 0; j < S; ++j) ktd::mbar_init(&mbar[j], 1);
       ktd::fence_proxy_async();
     }
     __syncthreads();
@@ -325,7 +332,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
         ktd::fence_proxy_async();
         if (p.tb.rec && tid == 0) s_tw[slot] = gtimer();
       }
-      uint8_t* dst = ktsm + (slot ? p.stage_bytes : 0);
+      uint8_t* dst = ktsm + slot * p.stage_bytes;
       if (p.use_tmap) {
         if (tid == 0) {
           s_tile[slot] = t;
@@ -336,16 +343,13 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
         ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
       }
     };
-    if (i0 < ntiles && tid < 32) {
-      issue(i0, 0);
-      if (i0 + gridDim.x < ntiles) issue(i0 + gridDim.x, 1);
-    }
-    unsigned ph = 0;
-    int b = 0;
-    for (int64_t i = i0; i < ntiles; i += gridDim.x, b ^= 1) {
-      uint8_t* buf = ktsm + (b ? p.stage_bytes : 0);
-      ktd::mbar_wait(&mbar[b], (ph >> b) & 1u);
-      ph ^= 1u << b;
+    if (tid < 32)
+      for (int j = 0; j < S && i0 + j * (int64_t)gridDim.x < ntiles; ++j) issue(i0 + j * (int64_t)gridDim.x, j);
+    int b = 0;          // slot of the current tile
+    unsigned par = 0;   // its mbarrier phase parity (flips each time the ring wraps)
+    for (int64_t i = i0; i < ntiles; i += gridDim.x) {
+      uint8_t* buf = ktsm + b * p.stage_bytes;
+      ktd::mbar_wait(&mbar[b], par);
       const ktd::Tile t = s_tile[b];
       if constexpr (OP == 2 || OP == 4) {
         if (p.cdisc) consumer_discard<OP>(p, t, nt, tid);
@@ -359,7 +363,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
         __syncthreads();
       }
       ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid, &p.aux, p.taps, p.radius);
-      const int64_t nx = i + 2 * (int64_t)gridDim.x;
+      const int64_t nx = i + (int64_t)S * gridDim.x;
       if (p.chain) {
         __syncthreads();  // tile written (and buffer b consumed)
         if (tid == 0) {
@@ -376,6 +380,10 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       if (nx < ntiles && tid < 32) {
         ktd::fence_proxy_async();
         issue(nx, b);
+      }
+      if (++b == S) {
+        b = 0;
+        par ^= 1u;
       }
     }
   }
@@ -808,6 +816,7 @@ __global__ void disc_cmp_kernel(const uint8_t* cur, const uint8_t* ref, const ui
 // host side
 // ------------------------------------------------------------------------------------
 typedef void (*kfn_t)(KParams);
+kfn_t deep_kernel(int op);
 
 kfn_t vec_kernel(int op) {
   switch (op) {
@@ -1101,7 +1110,16 @@ void build_launches(ktiler_plan_s* P) {
         }
         L.block = dim3(n.block[0], n.block[1], n.block[2]);
         L.kp.stage_bytes = n.scalar ? 0 : (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127;
+        L.kp.nstage = 2;
         L.smem = (int)(2 * L.kp.stage_bytes);
+        // KTILER_STAGES=S (experiment): sub-kernels of a tiled plan whose input is
+        // an intermediate (L2-resident) run one resident wave of CTAs that grid-stride over
+        // their tiles through an S-deep staging ring instead of one tile per CTA
+        static const int stages_env = getenv("KTILER_STAGES") ? atoi(getenv("KTILER_STAGES")) : 0;
+        if (stages_env > 2 && !n.scalar && P->s.nfrag > 1 && deep_kernel(n.op) && g.written_by_node(r.buf)) {
+          L.kp.nstage = std::min(stages_env, KMAXST);
+          L.smem = (int)(L.kp.nstage * L.kp.stage_bytes);
+        }
         P->launches.push_back(L);
       }
     }
@@ -1293,19 +1311,35 @@ ktiler_status cuda_fail(cudaError_t e, const char* what) {
   return fail(KTILER_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
+kfn_t deep_kernel(int op) {  // runtime ring depth (KParams::nstage > 2)
+  switch (op) {
+    case 2: return op_kernel<2, false, 0>;
+    case 3: return op_kernel<3, false, 0>;
+    case 4: return op_kernel<4, false, 0>;
+    default: return nullptr;
+  }
+}
 kfn_t launch_fn(const Launch& L) {
+  if (L.node >= 0 && !L.n->scalar && L.kp.nstage > 2 && deep_kernel(L.n->op)) return deep_kernel(L.n->op);
   return L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
 }
 
 // Dynamic-smem attribute + grid of one launch: the vector kernels grid-stride over their
 // tiles with as many CTAs as fit the device at once.
 ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_out) {
-  // static + dynamic may pass the 48 KB default; the attribute is per function, so it is
-  // always set to the two-buffer maximum (a one-buffer launch of the same kernel uses less)
-  const int smem_max = std::max(L.smem, (int)(2 * L.kp.stage_bytes));
-  if (L.resident == 0 && smem_max > 32 * 1024) {
-    cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_max);
-    if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
+  // static + dynamic may pass the 48 KB default.  The attribute is a per-function MAXIMUM
+  // (occupancy follows each launch's own size), so it is raised once to the device's
+  // opt-in limit: launches of one kernel with different ring depths never undercut it
+  if (L.resident == 0) {
+    cudaFuncAttributes fa{};
+    cudaFuncGetAttributes(&fa, (const void*)fn);
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, P->device);
+    const int want = optin - (int)fa.sharedSizeBytes;
+    if (fa.maxDynamicSharedSizeBytes < want) {
+      cudaError_t ea = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, want);
+      if (ea != cudaSuccess) return cuda_fail(ea, "cudaFuncSetAttribute (dynamic smem)");
+    }
   }
   if (L.resident == 0) {
     int nsm = 0, occ = 0;
@@ -1314,6 +1348,12 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
     L.resident = (int64_t)std::max(1, nsm) * std::max(1, occ);
   }
   int64_t grid = std::max<int64_t>(L.blocks, 1);
+  // deep staging ring (KTILER_STAGES, set at plan time): one resident wave of CTAs that
+  // grid-stride over the sub-kernel's tiles
+  if (L.kp.nstage > 2) {
+    *grid_out = std::min<int64_t>(grid, L.resident);
+    return KTILER_OK;
+  }
   // grid-stride CTAs (x tiles_per_cta) in stream/graph modes; in GRAPH_DAG one CTA per
   // tile by default, so concurrent sub-kernels interleave at tile granularity
   static const int tpc_env = getenv("KTILER_TILES_PER_CTA") ? atoi(getenv("KTILER_TILES_PER_CTA")) : -1;

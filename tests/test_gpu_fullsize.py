@@ -96,3 +96,30 @@ def test_giant_image_bench_config(W):
     p.b.store.tensors["mask"].fill_(0xA5)
     _run(p, kind="none", exec_mode="graph", discard=False)
     assert torch.equal(tiled, p.view("mask")[0]), "tiled != untiled"
+
+
+@pytest.mark.parametrize("name,pol,ring", [
+    ("flow", dict(kind="rows", rows=1, exec_mode="flow", consumer_discard=True), 0),
+    ("dag-ring4", dict(kind="budget", l2_fraction=0.85, exec_mode="dag", window=2, resident_budget=True,
+                       consumer_discard=True), 4),
+    ("dag-multirate", dict(kind="budget", l2_fraction=0.6, exec_mode="dag", window=3, resident_budget=True,
+                           consumer_discard=True, multirate=True), 0)])
+def test_batch64_8k_other_executors(name, pol, ring):
+    """The round-2 variants at BASELINE configs[3]'s full size, as measured in DESIGN §6.6-6.8:
+    the FLOW executor, ring intermediates (4 frames of storage for 64 frames) and multi-rate
+    fragments.  One sampled frame against the oracle; every frame against the untiled mask."""
+    from inputs import gpu as G
+    from paper_conf_date_maghazeh0ep19_b200 import Pipeline
+    W, H, F = 7680, 4320, 64
+    p = Pipeline(W, H, F, T=200.0, internal=True, ring_frames=ring)
+    G.fill("scene", SEED, p.view("rgb").data_ptr(), W * 3, W * 3 * H, W, H, F=F,
+           stream=torch.cuda.current_stream().cuda_stream)
+    p.b.store.tensors["mask"].fill_(0xA5)
+    plan = _run(p, **pol)
+    assert plan.num_fragments() > 1
+    got = p.view("mask").clone()
+    ref = O.pipeline(synth.scene_rows(SEED + 50, W, H, 0, H)[None])["mask"][0]
+    assert np.array_equal(got[50].cpu().numpy(), ref)
+    u = _pipeline(W, H, F)
+    _run(u, kind="none", exec_mode="graph", discard=False)
+    assert torch.equal(got, u.view("mask")), f"{name}: tiled != untiled on some frame"
