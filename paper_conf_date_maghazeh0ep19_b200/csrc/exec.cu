@@ -2049,7 +2049,24 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
 
   }
   // ---- kernel variant, slots (CTAs) per SM, shared memory per CTA ----
-  int K = P->flow_slot_role.empty() ? 3 : (int)P->flow_slot_role.size();
+  int K = (int)P->flow_slot_role.size();
+  if (P->flow_slot_role.empty()) {
+    // automatic: as many CTAs per SM as leave room for two staging slots of the largest
+    // tile each (more compute warps per SM; 3 for the shipped geometry's 37 KB blur tiles)
+    int maxst = 128;
+    for (auto& n : g.nodes) {
+      const kt::Access& w = n.acc[n.wacc];
+      maxst = std::max(maxst, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
+    }
+    int smem_sm0 = 0;
+    cudaDeviceGetAttribute(&smem_sm0, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
+    K = 2;
+    for (int k = 5; k >= 3; --k)
+      if (smem_sm0 / k - 1024 - 1024 >= 2 * maxst) {
+        K = k;
+        break;
+      }
+  }
   if (K < 2 || K > 5) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: 2..5 slots (CTAs) per SM");
   P->ffn = flow_variant(K);
   P->fthreads = flow_threads(K);
