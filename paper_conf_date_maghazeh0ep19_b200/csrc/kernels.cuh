@@ -564,43 +564,45 @@ __device__ __forceinline__ float2 mag2(uint32_t gx, uint32_t gy) {
 // three register sets, the row loop unrolled by 3 (static slot indices).
 __device__ __forceinline__ void sobel_row(const SobelRow& T, const SobelRow& M, const SobelRow& B, uint8_t* drow,
                                           bool seg_full, int64_t x0, int64_t W) {
-  // column smoothing S = top + 2 mid + bot, difference D = bot - top + 255 (per lane)
-  uint32_t SE[6], SO[6], DE[6], DO[6];
-#pragma unroll
-  for (int q = 0; q < 6; ++q) {
-    if (q >= 1) {
-      SE[q] = T.e[q] + B.e[q] + 2u * M.e[q];
-      DE[q] = B.e[q] + 0x00FF00FFu - T.e[q];
-    }
-    if (q <= 4) {
-      SO[q] = T.o[q] + B.o[q] + 2u * M.o[q];
-      DO[q] = B.o[q] + 0x00FF00FFu - T.o[q];
-    }
-  }
   float* dst = reinterpret_cast<float*>(drow);
-  uint32_t o[16];  // columns x .. x+15
+  // Two halves of 8 columns (window words q = 1, 2 and q = 3, 4), each stored as soon as it
+  // is done: at most 8 results and the column sums of words q-1 .. q+1 are live at once
+  // (register pressure: 4 sobel CTAs per SM at 128 registers before).
 #pragma unroll
-  for (int q = 1; q <= 4; ++q) {
-    const uint32_t gxe = SO[q] + 0x03FC03FCu - prmt(SO[q - 1], SO[q], 0x5432);
-    const uint32_t gye = prmt(DO[q - 1], DO[q], 0x5432) + 2u * DE[q] + DO[q];
-    const uint32_t gxo = prmt(SE[q], SE[q + 1], 0x5432) + 0x03FC03FCu - SE[q];
-    const uint32_t gyo = DE[q] + 2u * DO[q] + prmt(DE[q], DE[q + 1], 0x5432);
-    const float2 ev = mag2(gxe, gye);  // columns c, c+2 (c = x + 4q - 4)
-    const float2 od = mag2(gxo, gyo);  // columns c+1, c+3
-    o[4 * q - 4] = __float_as_uint(ev.x);
-    o[4 * q - 3] = __float_as_uint(od.x);
-    o[4 * q - 2] = __float_as_uint(ev.y);
-    o[4 * q - 1] = __float_as_uint(od.y);
-  }
-  if (seg_full) {
-    // two 256-bit stores: each covers whole 32-B sectors (16-B stores at a 64-B lane stride
-    // would write every sector in two halves, doubling the L2 write requests)
-    st32(dst, o);
-    st32(dst + 8, o + 8);
-  } else {
+  for (int half = 0; half < 2; ++half) {
+    uint32_t o[8];  // columns x + 8*half .. x + 8*half + 7
 #pragma unroll
-    for (int k = 0; k < 16; ++k)
-      if (x0 + k < W) dst[k] = __uint_as_float(o[k]);
+    for (int qq = 0; qq < 2; ++qq) {
+      const int q = 1 + 2 * half + qq;
+      // column smoothing S = top + 2 mid + bot, difference D = bot - top + 255 (per lane)
+      const uint32_t SOm = T.o[q - 1] + B.o[q - 1] + 2u * M.o[q - 1];
+      const uint32_t SOq = T.o[q] + B.o[q] + 2u * M.o[q];
+      const uint32_t SEq = T.e[q] + B.e[q] + 2u * M.e[q];
+      const uint32_t SEp = T.e[q + 1] + B.e[q + 1] + 2u * M.e[q + 1];
+      const uint32_t DOm = B.o[q - 1] + 0x00FF00FFu - T.o[q - 1];
+      const uint32_t DOq = B.o[q] + 0x00FF00FFu - T.o[q];
+      const uint32_t DEq = B.e[q] + 0x00FF00FFu - T.e[q];
+      const uint32_t DEp = B.e[q + 1] + 0x00FF00FFu - T.e[q + 1];
+      const uint32_t gxe = SOq + 0x03FC03FCu - prmt(SOm, SOq, 0x5432);
+      const uint32_t gye = prmt(DOm, DOq, 0x5432) + 2u * DEq + DOq;
+      const uint32_t gxo = prmt(SEq, SEp, 0x5432) + 0x03FC03FCu - SEq;
+      const uint32_t gyo = DEq + 2u * DOq + prmt(DEq, DEp, 0x5432);
+      const float2 ev = mag2(gxe, gye);  // columns c, c+2 (c = x + 4q - 4)
+      const float2 od = mag2(gxo, gyo);  // columns c+1, c+3
+      o[4 * qq + 0] = __float_as_uint(ev.x);
+      o[4 * qq + 1] = __float_as_uint(od.x);
+      o[4 * qq + 2] = __float_as_uint(ev.y);
+      o[4 * qq + 3] = __float_as_uint(od.y);
+    }
+    if (seg_full) {
+      // one 256-bit store per 8 columns: whole 32-B sectors (16-B stores at a 64-B lane
+      // stride would write every sector in two halves, doubling the L2 write requests)
+      st32(dst + 8 * half, o);
+    } else {
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+        if (x0 + 8 * half + k < W) dst[8 * half + k] = __uint_as_float(o[k]);
+    }
   }
 }
 
