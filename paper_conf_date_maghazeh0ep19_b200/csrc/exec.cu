@@ -1996,12 +1996,12 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
   const kt::Schedule& S = P->s;
   const int nn = (int)g.nodes.size();
   const int nsub = (int)S.subs.size();
-  if (nn > FMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: at most 32 nodes");
+  if (nn > FMAX_NODES) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: at most 1024 nodes");
   for (auto& n : g.nodes) {
-    if (n.op < KTILER_OP_GRAY || n.op > KTILER_OP_THRESH || n.scalar)
-      return fail(KTILER_E_UNSUPPORTED, "FLOW mode runs the vector image-pipeline built-ins (GRAY..THRESH) only");
-    if (n.gx() > 4096 || n.gy() > 4096 || n.gz() > 4096)
-      return fail(KTILER_E_UNSUPPORTED, "FLOW mode: grid exceeds the ticket (4096 blocks per axis and frames)");
+    if (n.op == KTILER_OP_CUSTOM || n.scalar)
+      return fail(KTILER_E_UNSUPPORTED, "FLOW mode runs the vector built-ins only (no OP_CUSTOM, no one-thread-per-pixel)");
+    if (n.gx() > FLOW_BXY_MAX + 1 || n.gy() > FLOW_BXY_MAX + 1 || n.gz() > FLOW_BZ_MAX + 1)
+      return fail(KTILER_E_UNSUPPORTED, "FLOW mode: grid exceeds the ticket (4096 blocks per axis, 256 frames)");
   }
   // ---- node table ----
   std::vector<int64_t> flag0(nn);
@@ -2021,6 +2021,9 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
     if (!make_tmap(g, n, &q.tmap, &q.box_bytes)) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: input tile map unavailable");
     q.in = dbuf(g.bufs[r.buf]);
     q.out = dbuf(g.bufs[w.buf]);
+    if (n.racc2 >= 0) q.aux = dbuf(g.bufs[n.acc[n.racc2].buf]);
+    q.radius = n.radius;
+    for (int k = 0; k < 9; ++k) q.taps[k] = n.taps[k];
     q.flag0 = flag0[v];
     q.op = n.op;
     q.tw = (int32_t)w.ax;

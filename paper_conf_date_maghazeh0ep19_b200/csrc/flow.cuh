@@ -40,13 +40,16 @@ namespace ktflow {
 using ktd::DBuf;
 
 constexpr int FSLOTS_MAX = 8;
-constexpr int FMAX_NODES = 32;
+constexpr int FMAX_NODES = 1024;
 constexpr int FMAX_ROLES = 16;
 constexpr int FMAX_SLOTS = 16;
 
 struct FNode {
   CUtensorMap tmap;  // input tile map (tensor TMA)
   DBuf in, out;
+  DBuf aux;          // KTILER_OP_JACOBI: the coefficient buffer (a graph input)
+  float taps[9];     // KTILER_OP_GAUSS_F32: f32 weights, taps[k + radius]
+  int32_t radius;
   int64_t flag0;     // this node's first tile flag
   int64_t pflag0;    // its producer node's first tile flag
   uint32_t box_bytes;
@@ -104,12 +107,18 @@ struct FParams {
   FTrace tb;                  // rec == NULL: tracing off
 };
 
-// Ticket: node (5) | window (23: leaf tiles that must be complete first) | bz (12) |
+// Ticket: node (10) | window (22: leaf tiles that must be complete first) | bz (8) |
 // by (12) | bx (12).
 __host__ __device__ inline uint64_t flow_ticket(uint64_t node, uint64_t wait, uint64_t bx, uint64_t by, uint64_t bz) {
-  return (node << 59) | (wait << 36) | (bz << 24) | (by << 12) | bx;
+  return (node << 54) | (wait << 32) | (bz << 24) | (by << 12) | bx;
 }
-constexpr uint64_t FLOW_WAIT_MAX = (1ull << 23) - 1;
+constexpr uint64_t FLOW_WAIT_MAX = (1ull << 22) - 1;
+constexpr int FLOW_BZ_MAX = 255, FLOW_BXY_MAX = 4095;
+__host__ __device__ __forceinline__ int fl_node(uint64_t d) { return (int)(d >> 54); }
+__host__ __device__ __forceinline__ unsigned fl_waitv(uint64_t d) { return (unsigned)((d >> 32) & FLOW_WAIT_MAX); }
+__host__ __device__ __forceinline__ int fl_bx(uint64_t d) { return (int)(d & 0xFFF); }
+__host__ __device__ __forceinline__ int fl_by(uint64_t d) { return (int)((d >> 12) & 0xFFF); }
+__host__ __device__ __forceinline__ int fl_bz(uint64_t d) { return (int)((d >> 24) & 0xFF); }
 constexpr uint64_t FLOW_STOP = ~0ull;
 
 __device__ __forceinline__ unsigned int fl_acquire(const unsigned int* p) {
@@ -144,7 +153,7 @@ __device__ __forceinline__ void fl_spin(uint64_t& n, uint64_t limit) {
 }
 
 __device__ __forceinline__ ktd::Tile flow_tile(const FNode& nd, uint64_t d) {
-  const int bx = (int)(d & 0xFFF), by = (int)((d >> 12) & 0xFFF), bz = (int)((d >> 24) & 0xFFF);
+  const int bx = fl_bx(d), by = fl_by(d), bz = fl_bz(d);
   ktd::Tile t;
   t.z = bz;
   t.x0 = (int64_t)nd.tw * bx;
@@ -161,7 +170,7 @@ struct PRange {
   int px0, py0, pw, n;
 };
 __device__ __forceinline__ PRange flow_prange(const FNode& nd, uint64_t d) {
-  const int bx = (int)(d & 0xFFF), by = (int)((d >> 12) & 0xFFF);
+  const int bx = fl_bx(d), by = fl_by(d);
   const int rx0 = max(0, nd.rax * bx + nd.rox - nd.rhl), rx1 = min((int)nd.in.W, nd.rax * (bx + 1) + nd.rox + nd.rhr);
   const int ry0 = max(0, nd.ray * by + nd.roy - nd.rht), ry1 = min((int)nd.in.H, nd.ray * (by + 1) + nd.roy + nd.rhb);
   const int px0 = rx0 / nd.wax, px1 = min(nd.pgx, (rx1 + nd.wax - 1) / nd.wax);
@@ -182,7 +191,7 @@ __device__ __forceinline__ unsigned flow_ready(const FParams& p, uint64_t mine, 
                                                int lane) {
   unsigned bad = 0;
   // window (source tiles): one load, compared with every pending tile's requirement
-  const unsigned wait = ((left >> lane) & 1u) ? (unsigned)((mine >> 36) & FLOW_WAIT_MAX) : 0u;
+  const unsigned wait = ((left >> lane) & 1u) ? fl_waitv(mine) : 0u;
   if (__any_sync(0xFFFFFFFFu, wait != 0u)) {
     unsigned done = 0;
     if (lane == 0) done = fl_relaxed(&p.ctrl->leaf_done);
@@ -193,9 +202,9 @@ __device__ __forceinline__ unsigned flow_ready(const FParams& p, uint64_t mine, 
   for (unsigned m = left; m; m &= m - 1) {
     const int j = __ffs(m) - 1;
     const uint64_t d = __shfl_sync(0xFFFFFFFFu, mine, j);
-    const FNode& nd = p.nodes[d >> 59];
+    const FNode& nd = p.nodes[fl_node(d)];
     const PRange r = flow_prange(nd, d);
-    const int bz = (int)((d >> 24) & 0xFFF);
+    const int bz = fl_bz(d);
     for (int i = lane; i < r.n; i += 32) {
       const int dy = i / r.pw;
       const unsigned int* f = p.flags + nd.pflag0 + ((int64_t)bz * nd.pgy + r.py0 + dy) * nd.pgx + r.px0 + (i - dy * r.pw);
@@ -331,7 +340,7 @@ __global__ void __launch_bounds__(32 * (NW + 1), MINB) flow_kernel(const __grid_
             rdy &= ~(1u << j);
             const uint64_t d = __shfl_sync(0xFFFFFFFFu, mine, j);
             if (lane == 0) {
-              const FNode& nd = p.nodes[d >> 59];
+              const FNode& nd = p.nodes[fl_node(d)];
               const int s = k_iss % S;
               const ktd::Tile tl = flow_tile(nd, d);
               s_tile[s] = tl;
@@ -369,7 +378,7 @@ __global__ void __launch_bounds__(32 * (NW + 1), MINB) flow_kernel(const __grid_
       const uint64_t tc0 = p.tb.rec ? fl_timer() : 0;
       const uint64_t d = s_desc[s];
       if (d == FLOW_STOP) break;
-      const FNode& nd = p.nodes[d >> 59];
+      const FNode& nd = p.nodes[fl_node(d)];
       const ktd::Tile t = s_tile[s];
       const uint8_t* buf = fsm + s * stage_bytes;
       if (nd.cdisc) flow_consumer_discard(nd, t, NC, tid);
@@ -377,7 +386,7 @@ __global__ void __launch_bounds__(32 * (NW + 1), MINB) flow_kernel(const __grid_
         ktd::stage_fix(nd.op, nd.in, t, const_cast<uint8_t*>(buf), NC, tid, 2);
         fl_bar(1, NC);
       }
-      ktd::compute_tile(nd.op, nd.out, t, buf, nd.T, NC, tid);
+      ktd::compute_tile(nd.op, nd.out, t, buf, nd.T, NC, tid, &nd.aux, nd.taps, nd.radius);
       if (p.tb.rec && tid == 0) fl_trace(p.tb, d, 6, tc0, fl_timer());
       fl_arrive(&s_done[s]);  // release (CTA scope) after this thread's tile stores
       if (warp == k % NW) {   // this warp publishes tile k

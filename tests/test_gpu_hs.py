@@ -83,3 +83,17 @@ def test_paper_shape_500_iterations():
     assert len(plan.clusters()) == K // 4
     ref = O.hs_jacobi(coef, s0, 0.5, K)
     assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("K,W,H,pol", [(8, 256, 160, dict(kind="none")), (8, 256, 160, dict(kind="rows", rows=2)),
+                                       (500, 1024, 1024, dict(kind="none"))],
+                         ids=["k8-one-fragment", "k8-rows2", "k500-1024"])
+def test_jacobi_chain_flow(K, W, H, pol):
+    """The JI chain under the persistent per-tile-flag executor (FLOW): a tile of iteration
+    k+1 starts as soon as the iteration-k tiles covering its 1-pixel halo are published —
+    a wavefront across iterations with no launch per iteration (the paper's inter-launch
+    gap, removed inside one launch).  Bit-exact vs O-14."""
+    got, plan, coef, s0, _ = _run(W, H, 1, K, 0.5, 99 + K, internal=True, exec_mode="flow", consumer_discard=True,
+                                  **dict(pol))
+    assert plan.stats()["n_launches"] == 1
+    assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 0.5, K).view(np.uint32))

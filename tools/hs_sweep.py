@@ -20,6 +20,7 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--workloads", default="1024x1024x500,7680x4320x40")
     ap.add_argument("--configs", default="")
+    ap.add_argument("--tile", default="64x16", help="JI tile (pixels) WxH")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -31,7 +32,8 @@ def main():
     s = torch.cuda.current_stream()
     for wl in args.workloads.split(","):
         W, H, K = (int(v) for v in wl.split("x"))
-        h = HSJacobi(W, H, K, a2=1.0, internal=True)
+        tw, th = (int(v) for v in args.tile.split("x"))
+        h = HSJacobi(W, H, K, a2=1.0, internal=True, tile=(tw, th))
         coef, s0 = synth.hs_fields(1234, W, H, 1)
         h.set("coef", coef)
         h.set("s0", s0)
@@ -58,7 +60,7 @@ def main():
                     ts.append(e0.elapsed_time(e1))
                 ms = statistics.median(ts)
                 st = pl.stats()
-                print(json.dumps({"workload": wl, "cfg": cfg, "ms": round(ms, 4), "Mpix_iter_per_s": round(W * H * K / ms / 1e3, 1),
+                print(json.dumps({"workload": wl, "tile": args.tile, "cfg": cfg, "ms": round(ms, 4), "Mpix_iter_per_s": round(W * H * K / ms / 1e3, 1),
                                   "fragments": st["n_fragments"], "launches": st["n_launches"]}), flush=True)
                 del pl
             except Exception as e:
