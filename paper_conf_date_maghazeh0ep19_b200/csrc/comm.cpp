@@ -230,6 +230,22 @@ ktiler_status ktiler_comm_register_strip(ktiler_comm_t c, int32_t rank, const kt
   return KTILER_OK;
 }
 
+ktiler_status ktiler_comm_check(ktiler_comm_t c) {
+  if (!c) return fail(KTILER_E_INVALID, "NULL comm");
+  if (c->kind != KTILER_COMM_NCCL || !c->nc) {
+    kt::clear_error();
+    return KTILER_OK;
+  }
+  const NcclApi& a = nccl();
+  if (!a.CommGetAsyncError) return fail(KTILER_E_UNSUPPORTED, "ncclCommGetAsyncError not available");
+  ncclResult_t r = ncclSuccess;
+  const ncclResult_t q = a.CommGetAsyncError(c->nc, &r);
+  if (q != ncclSuccess) return nccl_fail(q, "ncclCommGetAsyncError");
+  if (r != ncclSuccess && r != ncclInProgress) return nccl_fail(r, "NCCL communicator (asynchronous error)");
+  kt::clear_error();
+  return KTILER_OK;
+}
+
 ktiler_status ktiler_halo_exchange(ktiler_comm_t c, int32_t rank, int32_t halo_rows, void* stream) {
   ktiler_status s = kt::halo_exchange(c, rank, halo_rows, stream);
   if (!s) kt::clear_error();

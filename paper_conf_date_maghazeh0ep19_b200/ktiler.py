@@ -115,7 +115,7 @@ EXPORTS = ["ktiler_status_str", "ktiler_last_error", "ktiler_abi_version", "ktil
            "ktiler_plan_get_cluster", "ktiler_set_perf_table", "ktiler_calibrate", "ktiler_discover_footprint",
            "ktiler_plan_set_flow_roles", "ktiler_comm_unique_id", "ktiler_comm_init_nccl",
            "ktiler_comm_init_loopback", "ktiler_comm_destroy", "ktiler_comm_register_strip", "ktiler_halo_exchange",
-           "ktiler_plan_attach_halo", "ktiler_plan_reorder"]
+           "ktiler_plan_attach_halo", "ktiler_plan_reorder", "ktiler_comm_check"]
 
 _LIB = None
 
@@ -167,6 +167,7 @@ def lib() -> ctypes.CDLL:
         "ktiler_halo_exchange": ([vp, i32, i32, vp], st),
         "ktiler_plan_attach_halo": ([vp, vp, i32, i32], st),
         "ktiler_plan_reorder": ([vp, P(i64), i64], st),
+        "ktiler_comm_check": ([vp], st),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -442,6 +443,10 @@ class Comm:
                        e1: int) -> None:
         st = Strip(base, pitch_bytes, row_bytes, o0, o1, e0, e1)
         _check(lib().ktiler_comm_register_strip(self._h, rank, ctypes.byref(st)))
+
+    def check(self) -> None:
+        """Raise KtilerError if the NCCL communicator hit an asynchronous error."""
+        _check(lib().ktiler_comm_check(self._h))
 
     def exchange(self, rank: int, halo_rows: int, stream: int = 0) -> None:
         _check(lib().ktiler_halo_exchange(self._h, rank, halo_rows, ctypes.c_void_p(stream)))

@@ -318,6 +318,7 @@ def test_comm_abi_host_paths(K):
     plan.attach_halo(c, 0, 4)
     uid = K.comm_unique_id()  # NCCL is loadable here (no GPU needed for the id)
     assert len(uid) == 128
+    c.check()  # failure detection: a loopback comm never has an asynchronous error
     c.close()
 
 

@@ -343,6 +343,7 @@ def test_halo_exchange_nccl_single_rank():
     sp.attach(comm)
     sp.pipe.run()
     torch.cuda.synchronize()
+    comm.check()  # ncclCommGetAsyncError: no asynchronous error
     assert np.array_equal(sp.mask_owned().cpu().numpy(), O.pipeline(full[None], T=45.0)["mask"][0])
 
 
