@@ -65,7 +65,7 @@ def parse(argv=None):
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave", "flow"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=0.85)
+    ap.add_argument("--l2-fraction", type=float, default=1.0)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
     ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
@@ -81,7 +81,9 @@ def parse(argv=None):
                     help="also drop gray / down lines via per-block reader counts (DRAM -62%%, ~15%% slower: A44)")
     ap.add_argument("--no-consumer-discard", action="store_true",
                     help="keep the lines down2 / thresh consume (default: drop them once staged, DESIGN A44)")
-    ap.add_argument("--pdl", action="store_true")
+    ap.add_argument("--pdl", action="store_true", default=True,
+                    help="(default) programmatic-dependent-launch edges from each sub-kernel's producers (DESIGN §6.10)")
+    ap.add_argument("--no-pdl", dest="pdl", action="store_false")
     ap.add_argument("--ctas", type=int, default=0)
     ap.add_argument("--skew", type=int, default=0)
     ap.add_argument("--T", type=float, default=200.0)
@@ -173,7 +175,7 @@ def traffic_for(cfg: dict):
     except Exception:
         return None, None
     for e in d.get("entries", []):
-        if all(e["config"].get(k) == v for k, v in cfg.items()):
+        if all(e["config"].get(k, False if k == "pdl" else None) == v for k, v in cfg.items()):
             return e["dram_bytes_per_step"], e["source"]
     return None, None
 
@@ -516,7 +518,7 @@ def main():
     achieved = comp_bytes / world / (ms / 1000) / 1e9  # per GPU, against one GPU's peak
     tcfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
             "discard": discard, "window": args.window, "resident_budget": resident,
-            "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"]}
+            "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"], "pdl": bool(args.pdl)}
     traffic, traffic_src = traffic_for(tcfg)
     line = {
         "metric": METRIC,
@@ -572,7 +574,13 @@ def main():
         if comm is not None:
             un.attach_halo(comm, rank, SM.HALO_ROWS)
         ms_un = timed(lambda: un.execute(s), max(3, args.steps // 2), 2)
+        unp = pu.b.g.plan(0, kind="none", exec_mode="graph", discard=False, pdl=True)
+        if comm is not None:
+            unp.attach_halo(comm, rank, SM.HALO_ROWS)
+        ms_unp = timed(lambda: unp.execute(s), max(3, args.steps // 2), 2)
+        del unp
         line["untiled"] = {"value": pix / (ms_un / 1000) / 1e6, "ms_per_step": ms_un,
+                           "pdl_ms_per_step": ms_unp, "tiled_speedup_vs_pdl": ms_unp / ms,
                            "tiled_speedup": ms_un / ms,
                            "achieved_gbs": 9.75 * pix / (ms_un / 1000) / 1e9,
                            "roofline_frac": 9.75 * pix / (ms_un / 1000) / 1e9 / peak,
@@ -604,7 +612,7 @@ def main():
                 ach = d["bytes"] / d["launches"] / (d["span_ns"] / d["launches"])  # B/ns = GB/s
                 dtraffic = None
                 try:
-                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02_dominant_traffic.json")))
+                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02b_dominant_traffic.json")))
                     if dom in dt["kernels"] and all(line["config"].get(k) == v for k, v in dt["config"].items()):
                         kd = dt["kernels"][dom]
                         dtraffic = {"bytes": kd["dram_bytes_per_launch_mean"], "source": kd["source"]}

@@ -16,7 +16,7 @@ def test_default_policy_has_measured_traffic():
     pol = bench.policy(args)
     cfg = {"workload": args.workload, "mode": args.mode, "policy": args.kind, "l2_fraction": args.l2_fraction,
            "discard": pol["discard"], "window": args.window, "resident_budget": pol["resident_budget"],
-           "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"]}
+           "consumer_discard": pol["consumer_discard"], "halo_discard": pol["halo_discard"], "pdl": bool(args.pdl)}
     traffic, src = bench.traffic_for(cfg)
     assert traffic and traffic > 0 and src.startswith("profiles/")
     assert bench.l2_ceiling() is not None
