@@ -3,8 +3,9 @@
 #   gpurun_out/${TAG}_bench.json             python bench.py (defaults: the driver's command)
 #   gpurun_out/${TAG}_bench_reference.json   python bench.py --impl reference
 #   gpurun_out/${TAG}_launches_bench.csv     ncu launch list (gpu__time_duration per launch) of a short bench run
-#   gpurun_out/${TAG}_dag_op{0,1}_details.csv ncu --set full of one gray / blur sub-kernel launch of the
+#   gpurun_out/${TAG}_dag_op{0,1}_details.csv ncu --set full of four gray / blur sub-kernel launches of the
 #                                             default DAG plan (shipped geometry), serialised
+#                                             (tools/full_summary.py keeps the largest grid of each)
 #   gpurun_out/${TAG}_dominant_launches.csv  DRAM bytes of every gray sub-kernel launch of one execute
 set -u
 TAG=${1:-r02}
@@ -17,7 +18,7 @@ echo "launches rc=$?"
 C='[{"kind":"budget","l2_fraction":1.0,"exec_mode":"dag","discard":false,"window":2,"resident_budget":true,"consumer_discard":true,"pdl":true}]'
 for K in 0 1; do
   timeout 900 ncu --set full --import-source on --cache-control none --clock-control none --kernel-name-base mangled \
-    -k regex:"op_kernelILi${K}ELb0" --launch-skip 140 -c 1 -f -o gpurun_out/${TAG}_dag_op${K}_full \
+    -k regex:"op_kernelILi${K}ELb0" --launch-skip 120 -c 4 -f -o gpurun_out/${TAG}_dag_op${K}_full \
     python tools/sweep.py --reps 1 --configs "$C" > /dev/null 2>&1
   ncu -i gpurun_out/${TAG}_dag_op${K}_full.ncu-rep --page details --csv > gpurun_out/${TAG}_dag_op${K}_details.csv 2>/dev/null
 done
