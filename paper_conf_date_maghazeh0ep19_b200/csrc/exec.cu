@@ -286,12 +286,18 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     if (p.tb.rec) s_t0 = gtimer();
     if (p.chain) s_epoch = *(volatile const unsigned int*)p.epoch;
   }
-  if (p.chain) {
-    pdl_launch();  // the next sub-kernel may become resident now: it waits on tile flags
-  } else {
+  // PDL (p.pdl): wait for the programmatic producers (griddepcontrol.wait), then let this
+  // launch's dependents be scheduled (p.pdl == 1: right away; 2: only when CTAs exit).  The
+  // vector path sets up its shared-memory ring first, so that part overlaps the wait.
+  auto pdl_enter = [&]() {
     if (p.pdl) pdl_wait();
     if (p.ndisc) do_discards(p);
-    if (p.pdl) pdl_launch();
+    if (p.pdl == 1) pdl_launch();
+  };
+  if (p.chain) {
+    pdl_launch();  // the next sub-kernel may become resident now: it waits on tile flags
+  } else if (SCALAR) {
+    pdl_enter();
   }
   const int64_t ntiles = p.rpre[p.nrect];
   if (SCALAR) {
@@ -323,6 +329,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       ktd::fence_proxy_async();
     }
     __syncthreads();
+    if (!p.chain) pdl_enter();
     const unsigned epoch = s_epoch;
     const int64_t i0 = blockIdx.x;
     auto issue = [&](int64_t i, int slot) {  // warp 0
@@ -1087,7 +1094,9 @@ void build_launches(ktiler_plan_s* P) {
         L.kp.T = n.T;
         L.kp.radius = n.radius;
         for (int k = 0; k <= 2 * n.radius && k < 2 * ktd::GAUSS_H + 1; ++k) L.kp.taps[k] = n.taps[k];
-        L.kp.pdl = pdl;
+        // KTILER_PDL_TRIGGER=exit (experiment): dependents scheduled only as CTAs exit
+        static const bool trig_exit = getenv("KTILER_PDL_TRIGGER") && !strcmp(getenv("KTILER_PDL_TRIGGER"), "exit");
+        L.kp.pdl = pdl ? (trig_exit ? 2 : 1) : 0;
         size_t m = std::min<size_t>(MAXR, sk.rects.size() - c);
         L.kp.nrect = (int32_t)m;
         L.kp.rpre[0] = 0;
