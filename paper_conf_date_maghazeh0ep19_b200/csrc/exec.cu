@@ -1429,6 +1429,9 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   // (full completion + memory flush of every programmatic producer) before reading.
   const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
   static const bool pdl_all = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "all");
+  // KTILER_DAG_PDL_EDGES=chain (experiment): also the edge from the previous sub-kernel of
+  // the same node (not the window edges)
+  static const bool pdl_chain = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "chain");
   auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, const std::vector<uint8_t>& prog,
                       cudaGraphNode_t* node) -> ktiler_status {
     if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
@@ -1486,7 +1489,8 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   for (int i = 0; i < nsub; ++i) {
     std::vector<std::pair<cudaGraphNode_t, uint8_t>> dp;
     for (int d : edges[i]) {
-      const bool prod = pdl_all || std::find(S.sub_deps[i].begin(), S.sub_deps[i].end(), d) != S.sub_deps[i].end();
+      const bool prod = pdl_all || std::find(S.sub_deps[i].begin(), S.sub_deps[i].end(), d) != S.sub_deps[i].end() ||
+                        (pdl_chain && S.subs[d].node == S.subs[i].node);
       for (cudaGraphNode_t n : nodes_of[d]) dp.push_back({n, (uint8_t)(pdl && prod)});
     }
     std::sort(dp.begin(), dp.end());
