@@ -226,6 +226,9 @@ def test_smoke_configuration_is_tileable(K):
     p = Pipeline(520, 198, 2, T=60.0, internal=True, device=None)
     assert p.b.g.plan(800 * 1024, kind="budget", exec_mode="graph", discard=True, pdl=True).num_fragments() > 1
     assert p.b.g.plan(1 << 20, kind="rows", rows=1, exec_mode="persistent", discard=True).num_fragments() > 1
+    assert p.b.g.plan(400 * 1024, kind="budget", exec_mode="dag", window=2, pdl=True, consumer_discard=True,
+                      resident_budget=True).num_fragments() > 1  # the bench's policy shape
+    assert p.b.g.plan(1 << 20, kind="rows", rows=1, exec_mode="flow", consumer_discard=True).num_fragments() > 1
 
 
 def test_gauss_f32_params(K):
