@@ -1432,6 +1432,8 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   // KTILER_DAG_PDL_EDGES=chain (experiment): also the edge from the previous sub-kernel of
   // the same node (not the window edges)
   static const bool pdl_chain = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "chain");
+  // KTILER_DAG_PDL_EDGES=window (experiment): also the run-ahead window edges
+  static const bool pdl_window = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "window");
   auto add_node = [&](Launch& L, const std::vector<cudaGraphNode_t>& deps, const std::vector<uint8_t>& prog,
                       cudaGraphNode_t* node) -> ktiler_status {
     if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
@@ -1490,7 +1492,8 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     std::vector<std::pair<cudaGraphNode_t, uint8_t>> dp;
     for (int d : edges[i]) {
       const bool prod = pdl_all || std::find(S.sub_deps[i].begin(), S.sub_deps[i].end(), d) != S.sub_deps[i].end() ||
-                        (pdl_chain && S.subs[d].node == S.subs[i].node);
+                        (pdl_chain && S.subs[d].node == S.subs[i].node) ||
+                        (pdl_window && S.subs[d].node != S.subs[i].node);
       for (cudaGraphNode_t n : nodes_of[d]) dp.push_back({n, (uint8_t)(pdl && prod)});
     }
     std::sort(dp.begin(), dp.end());
