@@ -1019,10 +1019,17 @@ ktiler_status ring_analysis(ktiler_plan_s* P) {
   return KTILER_OK;
 }
 
+// PF_PDL takes effect only when the plan has several fragments: a one-fragment plan is the
+// untiled chain, where the early-resident consumer CTAs only hold SM slots (4096^2:
+// 52.0 vs 47.3 us, 64 x 8K untiled: 3.22 vs 3.19 ms; profiles/r02_dag_pdl_sweep.txt)
+static bool pdl_on(const ktiler_plan_s* P) {
+  return (P->pol.flags & KTILER_PF_PDL) != 0 && P->s.nfrag > 1;
+}
+
 void build_launches(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
-  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
+  const bool pdl = pdl_on(P);
   // GRAPH_DAG and GRAPH_CHAIN keep each sub-kernel's discard list apart (dag_disc, sub =
   // the list's sub-kernel): DAG makes them graph nodes, CHAIN attaches them to later launches
   const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN ||
@@ -1427,7 +1434,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   // KTILER_DAG_PDL_EDGES=all every kernel edge) are programmatic: the consumer's CTAs may
   // become resident while the producer's last wave drains and wait in griddepcontrol.wait
   // (full completion + memory flush of every programmatic producer) before reading.
-  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
+  const bool pdl = pdl_on(P);
   static const bool pdl_all = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "all");
   // KTILER_DAG_PDL_EDGES=chain (experiment): also the edge from the previous sub-kernel of
   // the same node (not the window edges)
