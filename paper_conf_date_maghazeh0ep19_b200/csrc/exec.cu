@@ -279,6 +279,7 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
 template <int OP, bool SCALAR, int NST = 2>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
+  __shared__ uint64_t s_tr, s_tl;  // trace: producers ready (after PDL wait), first tile staged
   __shared__ unsigned int s_epoch;
   const int nt = blockDim.x * blockDim.y * blockDim.z;
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
@@ -330,6 +331,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     }
     __syncthreads();
     if (!p.chain) pdl_enter();
+    if (p.tb.rec && tid == 0) s_tr = gtimer();
     const unsigned epoch = s_epoch;
     const int64_t i0 = blockIdx.x;
     auto issue = [&](int64_t i, int slot) {  // warp 0
@@ -357,6 +359,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     for (int64_t i = i0; i < ntiles; i += gridDim.x) {
       uint8_t* buf = ktsm + b * p.stage_bytes;
       ktd::mbar_wait(&mbar[b], par);
+      if (p.tb.rec && tid == 0 && i == i0) s_tl = gtimer();
       const ktd::Tile t = s_tile[b];
       if constexpr (OP == 2 || OP == 4) {
         if (p.cdisc) consumer_discard<OP>(p, t, nt, tid);
@@ -406,7 +409,13 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
   }
   if (p.tb.rec) {
     __syncthreads();
-    if (tid == 0) trace_put(p.tb, p.lid, 0, s_t0, gtimer());
+    if (tid == 0) {
+      trace_put(p.tb, p.lid, 0, s_t0, gtimer());
+      if (!SCALAR && !p.chain && blockIdx.x < ntiles) {  // CTA phases: start -> ready -> first tile staged
+        trace_put(p.tb, p.lid, 5, s_t0, s_tr);
+        trace_put(p.tb, p.lid, 6, s_tr, s_tl);
+      }
+    }
   }
 }
 

@@ -81,6 +81,25 @@ def summarise(rec, launches, pix):
                 per_gap[name] = round(float(np.median(gaps[gm])) / 1e3, 2)
         out["node_launch_span_us"] = per_span
         out["node_gap_before_us"] = per_gap
+    # op-kernel CTA phases (kinds 5, 6): start -> producers ready (PDL wait, discards),
+    # ready -> first tile staged (TMA latency), rest = compute + stores + exit
+    k5, k6 = rec[rec["kind"] == 5], rec[rec["kind"] == 6]
+    if len(k5) and len(k6) and len(k0):
+        phases = {}
+        node5 = np.array([launches[i][1] for i in k5["id"]])
+        d5 = k5["t1"].astype(np.int64) - k5["t0"].astype(np.int64)
+        d6 = k6["t1"].astype(np.int64) - k6["t0"].astype(np.int64)
+        node0 = np.array([launches[i][1] for i in k0["id"]])
+        d0 = k0["t1"].astype(np.int64) - k0["t0"].astype(np.int64)
+        for v in sorted(set(node5.tolist())):
+            if not 0 <= v < len(NODES):
+                continue
+            m5, m0 = node5 == v, node0 == v
+            w, l, c = float(d5[m5].mean()), float(d6[m5].mean()), float(d0[m0].mean())
+            phases[NODES[v]] = {"wait_us": round(w / 1e3, 2), "stage_us": round(l / 1e3, 2),
+                                "rest_us": round((c - w - l) / 1e3, 2),
+                                "stage_us_p10_50_90": [round(float(np.percentile(d6[m5], q)) / 1e3, 2) for q in (10, 50, 90)]}
+        out["cta_phases"] = phases
     for kind, name in ((3, "ready_to_computed"), (4, "publish")):
         kk = rec[rec["kind"] == kind]
         if len(kk):
