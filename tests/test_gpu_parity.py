@@ -150,6 +150,7 @@ REPLAY = [("graph", dict(discard=True)), ("persistent", dict(discard=True)), ("c
           # bench.py's executor and its discard variants: the halo-reader counters persist
           # across executes and must reset themselves
           ("dag", dict(window=2, resident_budget=True, consumer_discard=True)),
+          ("dag", dict(window=2, resident_budget=True, consumer_discard=True, pdl=True)),  # bench default
           ("dag", dict(window=2, consumer_discard=True, halo_discard=True)),
           ("dag", dict(window=2, consumer_discard=True, halo_discard=True, discard=True)),
           ("flow", dict(kind="rows", rows=1, consumer_discard=True)),
@@ -164,18 +165,17 @@ def test_replay_is_idempotent(mode, pol):
     W, H, F = 1024, 128, 1
     pol = dict(pol)
     kind = pol.pop("kind", "budget")
-    if True:
-        p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
-        a = synth.uniform(1, W, H, F)
-        b = synth.scene(2, W, H, F)
-        plan = p.plan(100 * 1024, kind=kind, exec_mode=mode, **pol)
-        assert plan.num_fragments() > 1
-        for it in range(6):
-            x = a if it % 2 == 0 else b
-            p.view("rgb").copy_(torch.from_numpy(x))
-            p.run()
-            torch.cuda.synchronize()
-            assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(x, T=40.0)["mask"]), (mode, it)
+    p = Pipeline(W, H, F, T=40.0, internal=True, geometry=SMALL)
+    a = synth.uniform(1, W, H, F)
+    b = synth.scene(2, W, H, F)
+    plan = p.plan(100 * 1024, kind=kind, exec_mode=mode, **pol)
+    assert plan.num_fragments() > 1
+    for it in range(6):
+        x = a if it % 2 == 0 else b
+        p.view("rgb").copy_(torch.from_numpy(x))
+        p.run()
+        torch.cuda.synchronize()
+        assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(x, T=40.0)["mask"]), (mode, it)
 
 
 @pytest.mark.parametrize("geometry", ["paper", "b200"])
