@@ -287,8 +287,13 @@ def test_trace_records(mode):
         tiles = sum(s["n_blocks"] for s in plan.subkernels())
         assert (rec["kind"] == 2).sum() == tiles and (rec["kind"] == 1).sum() == tiles
     else:
-        assert set(rec["kind"].tolist()) == ({0, 3, 4} if mode == "chain" else {0})
+        assert set(rec["kind"].tolist()) == ({0, 3, 4} if mode == "chain" else {0, 5, 6})
         assert set(rec["id"].tolist()) <= set(range(len(plan.launches())))
+        if mode != "chain":  # CTA phases: start -> ready -> staged, one pair per op-kernel CTA
+            k5, k6 = rec[rec["kind"] == 5], rec[rec["kind"] == 6]
+            assert len(k5) == len(k6) > 0 and np.array_equal(np.sort(k6["t0"]), np.sort(k5["t1"]))
+            node_of = np.array([node for (_, node, _) in plan.launches()])
+            assert len(k5) == int((node_of[rec[rec["kind"] == 0]["id"].astype(np.int64)] >= 0).sum())
     assert np.array_equal(p.view("mask").cpu().numpy(), O.pipeline(rgb, T=40.0)["mask"])
     with pytest.raises(Exception):
         plan.trace_enable(16)  # after the first execute
