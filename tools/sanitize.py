@@ -18,6 +18,8 @@ MODES = {
     "graph": dict(kind="budget", discard=True, pdl=True),
     "persist_l2": dict(kind="budget", discard=True),
     "dag": dict(kind="budget", window=2, resident_budget=True, consumer_discard=True, halo_discard=True, discard=True),
+    # the bench default: programmatic (PDL) producer edges, consumer discards
+    "dag_pdl": dict(kind="budget", window=2, resident_budget=True, consumer_discard=True, pdl=True),
     "chain": dict(kind="budget", discard=True, consumer_discard=True),
     "wave": dict(kind="budget", discard=True),
     "persistent": dict(kind="rows", rows=1, discard=True),
@@ -45,7 +47,7 @@ def main(argv):
         geo = None if mode in ("persistent", "flow") else SMALL
         p = Pipeline(W, H, F, T=60.0, internal=True, geometry=geo)
         p.view("rgb").copy_(torch.from_numpy(rgb))
-        plan = p.plan(256 * 1024 if geo else 1 << 20, kind=kind, exec_mode=mode, **pol)
+        plan = p.plan(256 * 1024 if geo else 1 << 20, kind=kind, exec_mode=mode.split("_")[0] if mode != "persist_l2" else mode, **pol)
         for _ in range(2):
             p.run()
         torch.cuda.synchronize()
