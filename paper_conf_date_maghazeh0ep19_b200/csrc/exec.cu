@@ -863,6 +863,7 @@ struct Launch {
   dim3 block;
   int smem = 0;
   int64_t resident = 0;  // CTAs of this kernel that fit the device at once
+  int64_t grid = 0;      // CTAs of the last prepared launch (prep_launch)
   int sub = -1;          // schedule sub-kernel (kernel launches) / discard list (DAG discards)
   std::vector<int32_t> crects;  // OP_CUSTOM rect list
 };
@@ -1028,17 +1029,29 @@ ktiler_status ring_analysis(ktiler_plan_s* P) {
   return KTILER_OK;
 }
 
-// PF_PDL takes effect only when the plan has several fragments: a one-fragment plan is the
-// untiled chain, where the early-resident consumer CTAs only hold SM slots (4096^2:
-// 52.0 vs 47.3 us, 64 x 8K untiled: 3.22 vs 3.19 ms; profiles/r02_dag_pdl_sweep.txt)
-static bool pdl_on(const ktiler_plan_s* P) {
-  return (P->pol.flags & KTILER_PF_PDL) != 0 && P->s.nfrag > 1;
+// PF_PDL edge policy: an edge from launch `prod` is programmatic when several fragments
+// overlap (nfrag > 1: GRAPH_DAG, profiles/r02_dag_pdl_sweep.txt) or when `prod` is a small
+// launch of at most 2 CTAs per SM (a latency-bound chain of small kernels, where the
+// consumer's early CTAs take idle SMs — HS 256^2 / 512^2 x 500 JI, 64 / 256 CTAs: 2.15 /
+// 2.26 vs 2.39 / 2.50 ms, profiles/r02c_hs_pyramid.txt).  In a one-fragment plan larger
+// producers lose (4096^2, 512-2048 CTAs: 52.5-54.5 vs 48-50 us; 64 x 8K untiled: 3.22 vs
+// 3.19 ms).  STREAM launches are host-latency bound, so there every producer edge is
+// programmatic (HS 1024^2 x 500: 3.86 vs 5.12 ms).  KTILER_PDL_ONE_FRAGMENT=1
+// (experiment): every producer edge.
+static bool pdl_edge(const ktiler_plan_s* P, const Launch& prod) {
+  static const bool one = getenv("KTILER_PDL_ONE_FRAGMENT") && atoi(getenv("KTILER_PDL_ONE_FRAGMENT")) != 0;
+  if (!(P->pol.flags & KTILER_PF_PDL) || prod.node < 0 || prod.n->op == KTILER_OP_CUSTOM) return false;
+  if (P->s.nfrag > 1 || one || P->pol.exec_mode == KTILER_EXEC_STREAM) return true;
+  int nsm = 0;
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+  return prod.grid > 0 && prod.grid <= 2 * (int64_t)std::max(nsm, 1);
 }
 
 void build_launches(ktiler_plan_s* P) {
   const kt::Graph& g = P->g;
   const bool disc = (P->pol.flags & KTILER_PF_DISCARD_DEAD) != 0;
-  const bool pdl = pdl_on(P);
+  // griddepcontrol in the kernels is a no-op on a launch without programmatic producers
+  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
   // GRAPH_DAG and GRAPH_CHAIN keep each sub-kernel's discard list apart (dag_disc, sub =
   // the list's sub-kernel): DAG makes them graph nodes, CHAIN attaches them to later launches
   const bool dag = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_CHAIN ||
@@ -1443,7 +1456,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
   // KTILER_DAG_PDL_EDGES=all every kernel edge) are programmatic: the consumer's CTAs may
   // become resident while the producer's last wave drains and wait in griddepcontrol.wait
   // (full completion + memory flush of every programmatic producer) before reading.
-  const bool pdl = pdl_on(P);
+  const bool pdl = (P->pol.flags & KTILER_PF_PDL) != 0;
   static const bool pdl_all = getenv("KTILER_DAG_PDL_EDGES") && !strcmp(getenv("KTILER_DAG_PDL_EDGES"), "all");
   // KTILER_DAG_PDL_EDGES=chain (experiment): also the edge from the previous sub-kernel of
   // the same node (not the window edges)
@@ -1476,6 +1489,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     int64_t grid = 0;
     ktiler_status ps = prep_launch(P, L, fn, &grid);
     if (ps) return ps;
+    L.grid = grid;
     void* args[1] = {&L.kp};
     cudaKernelNodeParams kp = {};
     kp.func = (void*)fn;
@@ -1504,13 +1518,15 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     return KTILER_OK;
   };
   size_t li = 0;
+  std::vector<std::vector<size_t>> launch_of(nsub);  // P->launches index of each node in nodes_of
   for (int i = 0; i < nsub; ++i) {
     std::vector<std::pair<cudaGraphNode_t, uint8_t>> dp;
     for (int d : edges[i]) {
       const bool prod = pdl_all || std::find(S.sub_deps[i].begin(), S.sub_deps[i].end(), d) != S.sub_deps[i].end() ||
                         (pdl_chain && S.subs[d].node == S.subs[i].node) ||
                         (pdl_window && S.subs[d].node != S.subs[i].node);
-      for (cudaGraphNode_t n : nodes_of[d]) dp.push_back({n, (uint8_t)(pdl && prod)});
+      for (size_t k = 0; k < nodes_of[d].size(); ++k)
+        dp.push_back({nodes_of[d][k], (uint8_t)(pdl && prod && pdl_edge(P, P->launches[launch_of[d][k]]))});
     }
     std::sort(dp.begin(), dp.end());
     std::vector<cudaGraphNode_t> deps;
@@ -1531,6 +1547,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
         return st;
       }
       nodes_of[i].push_back(nd);
+      launch_of[i].push_back(li);
     }
   }
   for (Launch& D : P->dag_disc) {
@@ -1550,15 +1567,20 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
 }
 
 ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
+  const Launch* prev = nullptr;  // the previous launch in the stream
   for (auto& L : P->launches) {
     if (L.node >= 0 && L.n->op == KTILER_OP_CUSTOM) {
       L.n->launch(L.n->user, L.crects.data(), (int32_t)(L.crects.size() / 6), (void*)st);
+      prev = &L;
       continue;
     }
     kfn_t fn = launch_fn(L);
     int64_t grid = 0;
     ktiler_status ps = prep_launch(P, L, fn, &grid);
     if (ps) return ps;
+    L.grid = grid;
+    const bool prog = L.kp.pdl && prev && pdl_edge(P, *prev);
+    prev = &L;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = L.block;
@@ -1566,7 +1588,7 @@ ktiler_status enqueue(ktiler_plan_s* P, cudaStream_t st) {
     cfg.stream = st;
     cudaLaunchAttribute attr[2];
     int na = 0;
-    if (L.kp.pdl || L.kp.chain == 1) {
+    if (prog || L.kp.chain == 1) {
       attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
       attr[na].val.programmaticStreamSerializationAllowed = 1;
       ++na;

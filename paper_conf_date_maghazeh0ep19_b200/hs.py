@@ -78,3 +78,44 @@ class HSJacobi:
 
     def run(self, stream: int = 0) -> None:
         self.plan_obj.execute(stream)
+
+
+class HSPyramid:
+    """The tiled part of Fig. 4: HSOpticalFlow's three steps work on
+    frames of 256, 512 and 1024 pixels per side (coarse to fine), each with a chain of 500 JI
+    nodes that starts from a zero vector ("{0}") and reads that step's derivative
+    coefficients.  The steps' other nodes (DS, WP, DV, AD, US: 1.5% of the application's
+    time) are not part of the north star (the SDK code that defines them is
+    not in the paper), so each step's coefficients come from the caller and the steps'
+    chains are independent graphs: one HSJacobi per step, planned by the same policy and
+    executed in Fig. 4's order on one stream.
+
+      steps[0]: (W >> (levels-1)) x (H >> (levels-1)),  ...,  steps[-1]: W x H."""
+
+    def __init__(self, W: int = 1024, H: int = 1024, iters: int = 500, levels: int = 3, frames: int = 1,
+                 a2: float = 1.0, tile=(64, 16), threads: int = 128, device="cuda", internal: bool = True):
+        if W % (2 << (levels - 1)) or H % (1 << (levels - 1)):
+            raise ValueError("HSPyramid needs W divisible by 2^levels and H by 2^(levels-1)")
+        self.levels, self.K = levels, iters
+        self.steps = [HSJacobi(W >> l, H >> l, iters, frames=frames, a2=a2, tile=tile, threads=threads, device=device,
+                               internal=internal) for l in reversed(range(levels))]
+        if device is not None:
+            for h in self.steps:
+                h.b.store.tensors["s0"].zero_()  # Fig. 4: every JI chain starts from {0}
+        self.plans = None
+
+    def set_coef(self, step: int, coef) -> None:
+        """(Ix, Iy, It, unused) of step `step` (0 = coarsest), host f32 [F, H, W, 4]."""
+        self.steps[step].set("coef", coef)
+
+    def get(self, step: int):
+        """The flow increment after the chain of step `step`: host f32 [F, H, W, 2]."""
+        return self.steps[step].get(f"s{self.K}")
+
+    def plan(self, cache_bytes: int = 0, **policy):
+        self.plans = [h.plan(cache_bytes, **policy) for h in self.steps]
+        return self.plans
+
+    def run(self, stream: int = 0) -> None:
+        for p in self.plans:
+            p.execute(stream)

@@ -490,3 +490,17 @@ def test_plan_reorder_validation(K):
     assert e.value.status == K.E_INVALID
     with pytest.raises(K.KtilerError):
         plan2.reorder([0] * len(subs))  # not a permutation
+
+
+def test_hs_pyramid_steps_plan(K):
+    """Fig. 4's three steps (256, 512, 1024 pixels per side, 500 JI nodes
+    each) plan on the host: one JI chain per step, coarse to fine, each tiled across
+    iterations by FRAG_CHAIN clusters of 4 nodes (the measured HS policy)."""
+    from paper_conf_date_maghazeh0ep19_b200.hs import HSPyramid
+    hp = HSPyramid(1024, 1024, 500, device=None)
+    assert [(h.W, h.H, h.K) for h in hp.steps] == [(256, 256, 500), (512, 512, 500), (1024, 1024, 500)]
+    plans = hp.plan(126 << 20, kind="chain", rows=4, l2_fraction=0.5, exec_mode="dag")
+    assert [len(p.clusters()) for p in plans] == [125, 125, 125]
+    assert all(p.num_fragments() >= 125 for p in plans)
+    with pytest.raises(ValueError):
+        HSPyramid(1020, 1024, 8, device=None)

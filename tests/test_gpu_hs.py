@@ -97,3 +97,26 @@ def test_jacobi_chain_flow(K, W, H, pol):
                                   **dict(pol))
     assert plan.stats()["n_launches"] == 1
     assert np.array_equal(got.view(np.uint32), O.hs_jacobi(coef, s0, 0.5, K).view(np.uint32))
+
+
+def test_pyramid_fig4_steps():
+    """Fig. 4's tiled nodes end to end: the three steps' JI chains (256,
+    512, 1024 pixels per side, 500 iterations each, every chain starting from {0}) executed
+    in order by HSPyramid under the measured HS policy; each step's result bit-exact vs the
+    f32 oracle O-14."""
+    from paper_conf_date_maghazeh0ep19_b200.hs import HSPyramid
+    K = 500
+    hp = HSPyramid(1024, 1024, K, a2=0.5)
+    coefs = []
+    for i, h in enumerate(hp.steps):
+        coef, _ = synth.hs_fields(700 + i, h.W, h.H, 1)
+        hp.set_coef(i, coef)
+        coefs.append(coef)
+        h.b.store.tensors[f"s{K}"].fill_(0xFF)  # NaN poison
+    hp.plan(0, kind="chain", rows=4, l2_fraction=0.5, exec_mode="dag")
+    hp.run()
+    torch.cuda.synchronize()
+    for i, h in enumerate(hp.steps):
+        zero = np.zeros((1, h.H, h.W, 2), np.float32)
+        ref = O.hs_jacobi(coefs[i], zero, 0.5, K)
+        assert np.array_equal(hp.get(i).view(np.uint32), ref.view(np.uint32)), i

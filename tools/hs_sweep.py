@@ -21,7 +21,11 @@ def main():
     ap.add_argument("--workloads", default="1024x1024x500,7680x4320x40")
     ap.add_argument("--configs", default="")
     ap.add_argument("--tile", default="64x16", help="JI tile (pixels) WxH")
+    ap.add_argument("--pyramid", action="store_true",
+                    help="Fig. 4's three steps instead (256^2, 512^2, 1024^2 x 500 JI, HSPyramid): ms per step and total")
     args = ap.parse_args()
+    if args.pyramid:
+        return pyramid(args)
     import numpy as np
     import torch
 
@@ -67,6 +71,48 @@ def main():
                 print(json.dumps({"workload": wl, "cfg": cfg, "error": str(e)}), flush=True)
         del h
         torch.cuda.empty_cache()
+
+
+def pyramid(args):
+    """Fig. 4's JI part (the paper's ~25% gain is on this application,
+    98.5% of whose time is in these nodes): the three steps' chains executed in order,
+    untiled vs tiled, CUDA events around each step and around the whole."""
+    import torch
+
+    import __graft_entry__ as ge
+    from inputs import synth
+    from paper_conf_date_maghazeh0ep19_b200.hs import HSPyramid
+    ge.build()
+    s = torch.cuda.current_stream()
+    tw, th = (int(v) for v in args.tile.split("x"))
+    hp = HSPyramid(1024, 1024, 500, tile=(tw, th))
+    for i, h in enumerate(hp.steps):
+        hp.set_coef(i, synth.hs_fields(1234 + i, h.W, h.H, 1)[0])
+    cfgs = json.loads(args.configs) if args.configs else [
+        dict(kind="none", exec_mode="graph"),
+        dict(kind="chain", rows=4, l2_fraction=0.5, exec_mode="dag", discard=True, resident_budget=True),
+        dict(kind="chain", rows=4, l2_fraction=0.5, exec_mode="dag", discard=True, resident_budget=True, pdl=True)]
+    for cfg in cfgs:
+        plans = hp.plan(0, **cfg)
+        for _ in range(2):
+            hp.run(s.cuda_stream)
+        tot, per = [], [[] for _ in plans]
+        for _ in range(args.reps):
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(len(plans) + 1)]
+            ev[0].record(s)
+            for i, p in enumerate(plans):
+                p.execute(s.cuda_stream)
+                ev[i + 1].record(s)
+            ev[-1].synchronize()
+            for i in range(len(plans)):
+                per[i].append(ev[i].elapsed_time(ev[i + 1]))
+            tot.append(ev[0].elapsed_time(ev[-1]))
+        print(json.dumps({"workload": "fig4_steps_256_512_1024_x500", "tile": args.tile, "cfg": cfg,
+                          "ms": round(statistics.median(tot), 4),
+                          "ms_per_step": [round(statistics.median(x), 4) for x in per],
+                          "fragments": [p.stats()["n_fragments"] for p in plans],
+                          "launches": [p.stats()["n_launches"] for p in plans]}), flush=True)
+        del plans
 
 
 if __name__ == "__main__":
