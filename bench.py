@@ -590,12 +590,16 @@ def main():
         # the persistent executor driven by per-tile dependency flags (north star's variant,
         # KTILER_EXEC_FLOW, its measured-best defaults) on the same batch, for comparison
         try:
-            fl = p.b.g.plan(0, kind="rows", rows=1, exec_mode="flow", consumer_discard=True)
+            from paper_conf_date_maghazeh0ep19_b200.pipeline import FLOW_GEOMETRY
+            pf = Pipeline(W, H, per, T=args.T, internal=True, geometry=FLOW_GEOMETRY)  # FLOW's best tiles
+            pf.view("rgb").copy_(p.view("rgb"))
+            fl = pf.plan(0, kind="rows", rows=1, exec_mode="flow", consumer_discard=True)
             ms_fl = timed(lambda: fl.execute(s), max(3, args.steps // 4), 2)
             line["flow"] = {"value": pix / (ms_fl / 1000) / 1e6, "ms_per_step": ms_fl,
                             "vs_untiled": line["untiled"]["ms_per_step"] / ms_fl,
-                            "policy": "rows=1 fragments, 3 CTAs/SM one role, skew 32, consumer discard"}
-            del fl
+                            "policy": "rows=1 fragments, 3 CTAs/SM one role, skew 32, consumer discard; "
+                                      "pipeline.FLOW_GEOMETRY (thresh 256x32)"}
+            del fl, pf
         except Exception as e:  # diagnostics only
             line["flow"] = {"error": str(e)}
     if not args.no_trace and rank == 0:

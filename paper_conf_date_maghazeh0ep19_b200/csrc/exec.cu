@@ -1288,9 +1288,10 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 // L2 sector promotion of the TMA requests (KTILER_TMA_PROMOTION = 0 / 64 / 128 / 256 bytes;
-// default 256).
+// default 128: the DAG + PDL step 0.6-0.8% faster than with 256, 0 the same,
+// profiles/r02c_policy_sweep.txt).
 CUtensorMapL2promotion l2_promotion() {
-  static const int v = getenv("KTILER_TMA_PROMOTION") ? atoi(getenv("KTILER_TMA_PROMOTION")) : 256;
+  static const int v = getenv("KTILER_TMA_PROMOTION") ? atoi(getenv("KTILER_TMA_PROMOTION")) : 128;
   return v == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
                 : (v == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
                            : (v == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B));
@@ -1803,6 +1804,19 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
   }
   int nsm = 0;
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+  int slot = 0;
+  for (auto& n : g.nodes) {
+    const kt::Access& w = n.acc[n.wacc];
+    if (!n.scalar) slot = std::max(slot, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
+  }
+  int smem_sm = 0, smem_blk = 0;
+  cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
+  cudaDeviceGetAttribute(&smem_blk, cudaDevAttrMaxSharedMemoryPerBlockOptin, P->device);
+  cudaFuncAttributes fa{};
+  auto per_cta_of = [&](void (*f)(PParams), int minb) {
+    cudaFuncGetAttributes(&fa, (const void*)f);
+    return std::min(smem_sm / minb - 1024, smem_blk) - (int)fa.sharedSizeBytes;
+  };
   {
     // KTILER_PERSIST_GROUPS: compute groups per CTA (4 -> one CTA per SM; 2 -> two; 1 ->
     // three single-group CTAs)
@@ -1811,22 +1825,19 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
     if (ng >= 4) { P->pfn = persistent_kernel<4, 1>; P->pminb = 1; P->pgroups = 4; }
     else if (ng == 2) { P->pfn = persistent_kernel<2, 2>; P->pminb = 2; P->pgroups = 2; }
     else { P->pfn = persistent_kernel<1, 3>; P->pminb = 3; P->pgroups = 1; }
+    // tiles too large for two slots per compute group (e.g. 64 KB f32 thresh tiles): one
+    // single-group CTA per SM (the whole shared memory for its ring)
+    if (!ev && slot && per_cta_of(P->pfn, P->pminb) / slot < 2 * P->pgroups) {
+      P->pfn = persistent_kernel<1, 1>;
+      P->pminb = 1;
+      P->pgroups = 1;
+    }
     P->pthreads = P->pgroups * PCOMP_THREADS + 64;
-  }
-  int slot = 0;
-  for (auto& n : g.nodes) {
-    const kt::Access& w = n.acc[n.wacc];
-    if (!n.scalar) slot = std::max(slot, (ktd::stage_bytes(n.op, (int)w.ax, (int)w.ay) + 127) & ~127);
   }
   // ring depth: as many slots as fit the shared memory of MINB CTAs per SM, a multiple of
   // the compute groups (slot s always serves group s mod NG, so every waiter on a slot's
   // barrier has consumed the slot's previous use itself: no parity aliasing)
-  int smem_sm = 0, smem_blk = 0;
-  cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
-  cudaDeviceGetAttribute(&smem_blk, cudaDevAttrMaxSharedMemoryPerBlockOptin, P->device);
-  cudaFuncAttributes fa{};
-  cudaFuncGetAttributes(&fa, (const void*)P->pfn);
-  const int per_cta = std::min(smem_sm / P->pminb - 1024, smem_blk) - (int)fa.sharedSizeBytes;
+  const int per_cta = per_cta_of(P->pfn, P->pminb);
   const int ngr = P->pgroups;
   int nslots = slot ? std::min(PSTAGES_MAX, std::max(2 * ngr, per_cta / slot)) : 2 * ngr;
   if (const char* ev = getenv("KTILER_PERSIST_SLOTS")) nslots = std::min(PSTAGES_MAX, std::max(ngr, atoi(ev)));
@@ -2027,13 +2038,14 @@ ktiler_status setup_persistent(ktiler_plan_s* P) {
 typedef void (*ffn_t)(ktflow::FParams);
 ffn_t flow_variant(int k) {
   switch (k) {
+    case 1: return ktflow::flow_kernel<8, 1>;  // tiles too large for two slots at 2 CTAs / SM
     case 2: return ktflow::flow_kernel<8, 2>;
     case 3: return ktflow::flow_kernel<4, 3>;
     case 5: return ktflow::flow_kernel<3, 5>;
     default: return ktflow::flow_kernel<4, 4>;
   }
 }
-int flow_threads(int k) { return k == 5 ? 128 : (k == 2 ? 288 : 160); }
+int flow_threads(int k) { return k == 5 ? 128 : (k <= 2 ? 288 : 160); }
 
 // Automatic roles: ONE role serving every node, on K slots per SM.  Measured on 16 x 8K
 // (profiles/r02_flow_sweeps.txt): a CTA that can take any ready tile keeps its warps busy;
@@ -2117,14 +2129,14 @@ ktiler_status setup_flow(ktiler_plan_s* P) {
     }
     int smem_sm0 = 0;
     cudaDeviceGetAttribute(&smem_sm0, cudaDevAttrMaxSharedMemoryPerMultiprocessor, P->device);
-    K = 2;
-    for (int k = 5; k >= 3; --k)
+    K = 1;
+    for (int k = 5; k >= 2; --k)
       if (smem_sm0 / k - 1024 - 1024 >= 2 * maxst) {
         K = k;
         break;
       }
   }
-  if (K < 2 || K > 5) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: 2..5 slots (CTAs) per SM");
+  if (K < 1 || K > 5) return fail(KTILER_E_UNSUPPORTED, "FLOW mode: 1..5 slots (CTAs) per SM");
   P->ffn = flow_variant(K);
   P->fthreads = flow_threads(K);
   int nsm = 0, smem_sm = 0, smem_blk = 0;

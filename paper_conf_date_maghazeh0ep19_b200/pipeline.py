@@ -11,7 +11,7 @@ Buffers are torch CUDA tensors (PyTorch is only the allocator here); with
 planner can run without a GPU (planning never dereferences buffers).
 
 B200 geometry: per-op tiles, see B200_GEOMETRY (gray 256x32, blur5 512x64,
-half-resolution kernels 256x32); the planner derives the mixed-geometry
+half-resolution kernels down2 256x32, sobel3 / thresh 256x64); the planner derives the mixed-geometry
 block dependencies in closed form from the declared footprints.
 
 """
@@ -29,8 +29,14 @@ B200_GEOMETRY = {
     "blur": (512, 64, 128),    # 128 column strips x 16 rows; 37 KB staged halo tile
     "down": (256, 32, 128),    # 512 items (4 per thread); 32 KB staged blur rows
     "sobel": (256, 64, 128),   # 128 strips x 8 rows; 19 KB halo tile
-    "thresh": (256, 32, 128),  # 512 items (4 per thread); 32 KB staged f32
+    "thresh": (256, 64, 128),  # 1024 items (8 per thread); 64 KB staged f32 = one sobel tile
+                               # (DAG + PDL step 1.5% faster than 256x32, profiles/r02c_policy_sweep.txt)
 }
+
+# The persistent executors (FLOW, PERSISTENT) stage every op's tiles in one ring of slots of
+# the largest staged tile: with 64 KB thresh tiles FLOW fits one CTA per SM (9.2 ms on
+# 64 x 8K), with 32 KB ones three (6.9 ms; profiles/r02c_policy_sweep.txt).
+FLOW_GEOMETRY = dict(B200_GEOMETRY, thresh=(256, 32, 128))
 
 
 def _cdiv(a: int, b: int) -> int:
