@@ -432,9 +432,18 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # KTILER_BENCH_BACKEND=gloo (test only, echoed in config.env): ranks may share a GPU, so
+    # the multi-rank path (barriers, max over ranks, rank-0 line) runs on a 1-GPU box
+    backend = os.environ.get("KTILER_BENCH_BACKEND", "nccl")
+    if backend == "gloo":
+        local %= max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    coll_dev = "cuda" if backend == "nccl" else "cpu"
     W, H, Ftot, cfg_idx, shard = WORKLOADS[args.workload]
     import __graft_entry__ as ge
     ge.build()
@@ -495,7 +504,7 @@ def main():
         ms = e0.elapsed_time(e1) / steps
         if per_step:
             step_ms[:] = [(e0 if k == 0 else marks[k - 1]).elapsed_time(marks[k]) for k in range(steps)]
-        return FR.max_over_ranks(ms, world, device="cuda")
+        return FR.max_over_ranks(ms, world, device=coll_dev)
 
     comm = None
     if sp is not None and world > 1:
