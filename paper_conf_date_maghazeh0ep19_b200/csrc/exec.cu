@@ -1033,7 +1033,7 @@ ktiler_status ring_analysis(ktiler_plan_s* P) {
 // overlap (nfrag > 1: GRAPH_DAG, profiles/r02_dag_pdl_sweep.txt) or when `prod` is a small
 // launch of at most 2 CTAs per SM (a latency-bound chain of small kernels, where the
 // consumer's early CTAs take idle SMs — HS 256^2 / 512^2 x 500 JI, 64 / 256 CTAs: 2.15 /
-// 2.26 vs 2.39 / 2.50 ms, profiles/r02c_hs_pyramid.txt).  In a one-fragment plan larger
+// 2.26 vs 2.39 / 2.50 ms, profiles/r02c_hs_pyramid.jsonl).  In a one-fragment plan larger
 // producers lose (4096^2, 512-2048 CTAs: 52.5-54.5 vs 48-50 us; 64 x 8K untiled: 3.22 vs
 // 3.19 ms).  STREAM launches are host-latency bound, so there every producer edge is
 // programmatic (HS 1024^2 x 500: 3.86 vs 5.12 ms).  KTILER_PDL_ONE_FRAGMENT=1
