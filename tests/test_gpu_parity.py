@@ -145,6 +145,25 @@ def test_b200_geometry_tiled(mode):
     assert _eq(out["mask"], ref["mask"])
 
 
+BENCH_POLICY = dict(kind="budget", exec_mode="dag", window=2, resident_budget=True, consumer_discard=True, pdl=True)
+
+
+@pytest.mark.parametrize("W,H,F", [(2000, 1082, 3), (1538, 770, 2), (4100, 520, 1)])
+@pytest.mark.parametrize("mode", ["dag-bench", "flow", "persistent"])
+def test_b200_geometry_ragged(W, H, F, mode):
+    """The shipped geometry (thresh 256x64 tiles: one sobel tile) on ragged sizes (no axis a
+    multiple of any tile), tiled into several fragments: the bench's own policy, and FLOW /
+    PERSISTENT on their one-CTA-per-SM fallbacks for 64 KB tiles; intermediates too."""
+    rgb = synth.scene(W + H + F, W, H, F)
+    ref = O.pipeline(rgb, T=45.0)
+    pol = dict(BENCH_POLICY) if mode == "dag-bench" else dict(kind="rows", rows=1, exec_mode=mode)
+    cb = (2 << 20) if mode == "dag-bench" else (4 << 20)  # the resident budget counts intermediates only
+    out, plan = _run(W, H, F, rgb, T=45.0, cache_bytes=cb, geometry=None, internal=False, **pol)
+    assert plan.num_fragments() >= 3
+    for k in KEYS:
+        assert _eq(out[k], ref[k]), k
+
+
 REPLAY = [("graph", dict(discard=True)), ("persistent", dict(discard=True)), ("chain", dict(discard=True)),
           ("wave", dict(discard=True)),
           # bench.py's executor and its discard variants: the halo-reader counters persist
