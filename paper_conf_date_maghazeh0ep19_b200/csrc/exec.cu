@@ -52,11 +52,17 @@ struct DRect {  // whole 128-B lines: row r -> base + (z mod ring)*fs + y*pitch 
 __device__ __forceinline__ int64_t drect_zoff(const DRect& d, int64_t z) {
   return (d.ring ? (int64_t)((uint32_t)z % (uint32_t)d.ring) : z) * d.fstride;
 }
-// Device-side trace ring (ktiler_trace_enable): NULL rec = tracing off.
+// Device-side trace buffer (ktiler_trace_enable): NULL rec = tracing off.  Sharded by CTA
+// and SM (TRACE_SHARDS counters, each owning cap records), so a record costs an atomic on
+// one of many counters instead of one device-wide counter that every CTA of the step contends on
+// (that serialisation slowed a traced 64 x 8K step by ~1.7 ms and penalised plans with
+// many small CTAs).  ktiler_trace_read gathers the shards.
+constexpr int TRACE_SHARDS = 256;
+static_assert(TRACE_SHARDS == ktflow::FL_TRACE_SHARDS, "FLOW writes the same sharded trace layout");
 struct TraceBuf {
   ktiler_trace_record* rec;
-  unsigned long long* n;
-  int64_t cap;
+  unsigned long long* n;  // TRACE_SHARDS counters
+  int64_t cap;            // records per shard
 };
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
@@ -64,12 +70,14 @@ __device__ __forceinline__ uint64_t gtimer() {
   return t;
 }
 __device__ __forceinline__ void trace_put(const TraceBuf& tb, uint64_t id, uint32_t kind, uint64_t t0, uint64_t t1) {
-  const unsigned long long k = atomicAdd(tb.n, 1ull);
-  if ((int64_t)k < tb.cap) {
-    uint32_t sm;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
-    tb.rec[k] = ktiler_trace_record{id, sm, kind, t0, t1};
-  }
+  uint32_t sm;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+  // shard by a hash of (record id, CTA, SM): small launches fill the low SM ids with
+  // low CTA indices first, so SM or CTA alone would crowd a few shards
+  const uint32_t sh =
+      ((blockIdx.x * 0x9E3779B9u) ^ (sm * 0x85EBCA6Bu) ^ ((uint32_t)id * 0xC2B2AE35u)) >> 24 & (TRACE_SHARDS - 1);
+  const unsigned long long k = atomicAdd(tb.n + sh, 1ull);
+  if ((int64_t)k < tb.cap) tb.rec[(int64_t)sh * tb.cap + (int64_t)k] = ktiler_trace_record{id, sm, kind, t0, t1};
 }
 
 struct KParams {
@@ -866,6 +874,7 @@ struct Launch {
   int64_t grid = 0;      // CTAs of the last prepared launch (prep_launch)
   int sub = -1;          // schedule sub-kernel (kernel launches) / discard list (DAG discards)
   std::vector<int32_t> crects;  // OP_CUSTOM rect list
+  int cap_per_sm = 0;    // > 0: grid capped at this many CTAs per SM (grid-stride through the ring)
 };
 
 }  // namespace
@@ -1158,6 +1167,18 @@ void build_launches(ktiler_plan_s* P) {
           L.kp.nstage = std::min(stages_env, KMAXST);
           L.smem = (int)(L.kp.nstage * L.kp.stage_bytes);
         }
+        // KTILER_SRC_CTAS=K (experiment): the sub-kernels of a tiled plan that read a graph
+        // input (the HBM-streaming source node) run at most K CTAs per SM, grid-striding through
+        // a KTILER_SRC_STAGES-deep ring (default 3), so they stream without filling every SM
+        // slot ahead of the previous fragment's consumer sub-kernels
+        static const int src_ctas = getenv("KTILER_SRC_CTAS") ? atoi(getenv("KTILER_SRC_CTAS")) : 0;
+        static const int src_stages = getenv("KTILER_SRC_STAGES") ? atoi(getenv("KTILER_SRC_STAGES")) : 3;
+        if (src_ctas > 0 && !n.scalar && P->s.nfrag > 1 && !g.written_by_node(r.buf) &&
+            (src_stages <= 2 || deep_kernel(n.op))) {
+          L.kp.nstage = std::max(2, std::min(src_stages, KMAXST));
+          L.smem = (int)(L.kp.nstage * L.kp.stage_bytes);
+          L.cap_per_sm = src_ctas;
+        }
         P->launches.push_back(L);
       }
     }
@@ -1183,6 +1204,11 @@ void build_launches(ktiler_plan_s* P) {
 // GRAPH_DAG edges at sub-kernel level: exact sub-kernel dependencies (Schedule::sub_deps),
 // the previous sub-kernel of the same node, and the run-ahead window (a sub-kernel with no
 // producers in fragment f waits for the leaf sub-kernels of fragment f - window).
+int dag_prio_mode() {
+  static const int v = getenv("KTILER_DAG_PRIO") ? atoi(getenv("KTILER_DAG_PRIO")) : 0;
+  return v;
+}
+
 std::vector<std::vector<int>> dag_edges(const ktiler_plan_s* P) {
   const kt::Schedule& S = P->s;
   const kt::Graph& g = P->g;
@@ -1352,6 +1378,7 @@ ktiler_status cuda_fail(cudaError_t e, const char* what) {
 
 kfn_t deep_kernel(int op) {  // runtime ring depth (KParams::nstage > 2)
   switch (op) {
+    case 0: return op_kernel<0, false, 0>;
     case 2: return op_kernel<2, false, 0>;
     case 3: return op_kernel<3, false, 0>;
     case 4: return op_kernel<4, false, 0>;
@@ -1387,6 +1414,12 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
     L.resident = (int64_t)std::max(1, nsm) * std::max(1, occ);
   }
   int64_t grid = std::max<int64_t>(L.blocks, 1);
+  if (L.cap_per_sm > 0) {  // KTILER_SRC_CTAS: K CTAs per SM grid-striding through the ring
+    int nsm = 0;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, P->device);
+    *grid_out = std::min<int64_t>({grid, L.resident, (int64_t)L.cap_per_sm * std::max(1, nsm)});
+    return KTILER_OK;
+  }
   // deep staging ring (KTILER_STAGES, set at plan time): one resident wave of CTAs that
   // grid-stride over the sub-kernel's tiles
   if (L.kp.nstage > 2) {
@@ -1518,6 +1551,28 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
       return cuda_fail(ee, "cudaGraphAddDependencies_v2");
     return KTILER_OK;
   };
+  // CTA-dispatch priority per kernel node (KTILER_DAG_PRIO experiment; needs
+  // cudaGraphInstantiateFlagUseNodePriority at instantiation, dag_uses_priority): 1 = the
+  // deeper the node, the higher its priority, so a consumer sub-kernel's CTAs are dispatched
+  // before the next fragment's source CTAs that keep refilling the SMs; 2 = the reverse.
+  const int prio_mode = dag_prio_mode();
+  std::vector<int> ndepth(g.nodes.size(), 0);
+  for (int v : g.topo)
+    for (auto& c : g.in_ch[v]) ndepth[v] = std::max(ndepth[v], ndepth[c.u] + 1);
+  int prio_lo = 0, prio_hi = 0;  // least / greatest (numerically lower = higher priority)
+  if (prio_mode) cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  auto set_prio = [&](cudaGraphNode_t nd, int node) -> ktiler_status {
+    if (!prio_mode || node < 0) return KTILER_OK;
+    int d = ndepth[node], dmax = 0;
+    for (int x : ndepth) dmax = std::max(dmax, x);
+    if (prio_mode == 2) d = dmax - d;
+    if (prio_mode == 3) d = d > 0 ? dmax : 0;   // source nodes low, every consumer high
+    if (prio_mode == 4) d = d >= 3 ? dmax : 0;  // only the deep (quarter-resolution) consumers high
+    cudaKernelNodeAttrValue v = {};
+    v.priority = std::max(prio_hi, prio_lo - d);
+    cudaError_t ee = cudaGraphKernelNodeSetAttribute(nd, cudaLaunchAttributePriority, &v);
+    return ee == cudaSuccess ? KTILER_OK : cuda_fail(ee, "cudaGraphKernelNodeSetAttribute(priority)");
+  };
   size_t li = 0;
   std::vector<std::vector<size_t>> launch_of(nsub);  // P->launches index of each node in nodes_of
   for (int i = 0; i < nsub; ++i) {
@@ -1543,6 +1598,7 @@ ktiler_status build_dag(ktiler_plan_s* P, cudaGraph_t* out) {
     for (; li < P->launches.size() && P->launches[li].sub == i; ++li) {
       cudaGraphNode_t nd;
       ktiler_status st = add_node(P->launches[li], deps, prog, &nd);
+      if (!st && P->launches[li].node >= 0 && P->launches[li].n->op != KTILER_OP_CUSTOM) st = set_prio(nd, P->launches[li].node);
       if (st) {
         cudaGraphDestroy(gr);
         return st;
@@ -2570,7 +2626,8 @@ ktiler_status ktiler_execute(ktiler_plan_t p, void* stream) {
           return s;
         }
         p->graph = gr;
-        if ((e = cudaGraphInstantiate(&p->exec, gr, 0)) != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
+        const unsigned long long iflags = dag_prio_mode() ? cudaGraphInstantiateFlagUseNodePriority : 0;
+        if ((e = cudaGraphInstantiate(&p->exec, gr, iflags)) != cudaSuccess) return cuda_fail(e, "cudaGraphInstantiate");
       }
       if ((e = cudaGraphLaunch(p->exec, st)) != cudaSuccess) return cuda_fail(e, "cudaGraphLaunch");
       break;
@@ -2715,19 +2772,24 @@ ktiler_status ktiler_calibrate(ktiler_graph_t gh, int32_t node, int32_t npts, co
     return r;
   };
   // device-side spans (first CTA start -> last CTA end) through the tracer
-  const int64_t tcap = 1 << 18;
+  const int64_t tper = 1 << 10, tcap = tper * TRACE_SHARDS;  // per-SM shards (TraceBuf)
   void* tmem = nullptr;
-  if ((e = cudaMalloc(&tmem, (size_t)tcap * sizeof(ktiler_trace_record) + 256)) != cudaSuccess)
+  if ((e = cudaMalloc(&tmem, (size_t)tcap * sizeof(ktiler_trace_record) + TRACE_SHARDS * 8)) != cudaSuccess)
     return cuda_fail(e, "cudaMalloc (calibration trace)");
   TraceBuf tb{(ktiler_trace_record*)tmem, (unsigned long long*)((char*)tmem + (size_t)tcap * sizeof(ktiler_trace_record)),
-              tcap};
+              tper};
+  cudaMemset(tb.n, 0, TRACE_SHARDS * sizeof(unsigned long long));
   std::vector<ktiler_trace_record> rec;
   auto read_span = [&](uint64_t id, uint64_t* t0, uint64_t* t1) -> bool {  // after a sync
-    unsigned long long cnt = 0;
-    cudaMemcpy(&cnt, tb.n, sizeof(cnt), cudaMemcpyDeviceToHost);
-    const int64_t k = std::min<int64_t>((int64_t)cnt, tcap);
-    rec.resize((size_t)k);
-    if (k) cudaMemcpy(rec.data(), tb.rec, (size_t)k * sizeof(ktiler_trace_record), cudaMemcpyDeviceToHost);
+    unsigned long long cnt[TRACE_SHARDS];
+    cudaMemcpy(cnt, tb.n, sizeof(cnt), cudaMemcpyDeviceToHost);
+    rec.clear();
+    for (int sh = 0; sh < TRACE_SHARDS; ++sh) {
+      const int64_t k = std::min<int64_t>((int64_t)cnt[sh], tper);
+      const size_t at = rec.size();
+      rec.resize(at + (size_t)k);
+      if (k) cudaMemcpy(rec.data() + at, tb.rec + sh * tper, (size_t)k * sizeof(ktiler_trace_record), cudaMemcpyDeviceToHost);
+    }
     *t0 = ~0ull;
     *t1 = 0;
     for (auto& r : rec)
@@ -2776,7 +2838,7 @@ ktiler_status ktiler_calibrate(ktiler_graph_t gh, int32_t node, int32_t npts, co
     const std::vector<kt::Rect6> one = first_rects(n, std::min<int64_t>(n.nblocks, n.gx()));
     std::vector<double> gaps;
     for (int r = 0; r < reps + 1 && !rs; ++r) {
-      cudaMemsetAsync(tb.n, 0, sizeof(unsigned long long), st);
+      cudaMemsetAsync(tb.n, 0, TRACE_SHARDS * sizeof(unsigned long long), st);
       rs = launch_rects(node, one, 2, 2);  // trace ids 2 and 3
       cudaStreamSynchronize(st);
       uint64_t a0, a1, b0, b1;
@@ -2805,7 +2867,7 @@ ktiler_status ktiler_calibrate(ktiler_graph_t gh, int32_t node, int32_t npts, co
         if (hot)
           for (auto& pp : prod)
             if (!rs) rs = launch_rects(pp.first, pp.second, -1);
-        cudaMemsetAsync(tb.n, 0, sizeof(unsigned long long), st);
+        cudaMemsetAsync(tb.n, 0, TRACE_SHARDS * sizeof(unsigned long long), st);
         if (!rs) rs = launch_rects(node, rects, 1);
         cudaStreamSynchronize(st);
         uint64_t t0, t1;
@@ -3011,13 +3073,16 @@ ktiler_status ktiler_trace_enable(ktiler_plan_t p, int64_t capacity) {
   if (!p || capacity <= 0) return fail(KTILER_E_INVALID, "NULL plan or capacity <= 0");
   if (p->executed || p->tb.rec) return fail(KTILER_E_STATE, "ktiler_trace_enable must precede the first execute");
   void* d = nullptr;
-  cudaError_t e = cudaMalloc(&d, (size_t)capacity * sizeof(ktiler_trace_record) + 256);
+  // capacity records in TRACE_SHARDS per-SM shards (rounded up), then the shard counters
+  const int64_t per = (capacity + TRACE_SHARDS - 1) / TRACE_SHARDS;
+  const size_t rec_bytes = (size_t)per * TRACE_SHARDS * sizeof(ktiler_trace_record);
+  const size_t bytes = rec_bytes + TRACE_SHARDS * sizeof(unsigned long long);
+  cudaError_t e = cudaMalloc(&d, bytes);
   if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc (trace)");
-  if ((e = cudaMemset(d, 0, (size_t)capacity * sizeof(ktiler_trace_record) + 256)) != cudaSuccess)
-    return cuda_fail(e, "cudaMemset (trace)");
+  if ((e = cudaMemset(d, 0, bytes)) != cudaSuccess) return cuda_fail(e, "cudaMemset (trace)");
   p->tb.rec = (ktiler_trace_record*)d;
-  p->tb.n = (unsigned long long*)((char*)d + (size_t)capacity * sizeof(ktiler_trace_record));
-  p->tb.cap = capacity;
+  p->tb.n = (unsigned long long*)((char*)d + rec_bytes);
+  p->tb.cap = per;
   kt::clear_error();
   return KTILER_OK;
 }
@@ -3027,13 +3092,20 @@ ktiler_status ktiler_trace_read(ktiler_plan_t p, ktiler_trace_record* out, int64
   if (!p->tb.rec) return fail(KTILER_E_STATE, "tracing not enabled");
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceSynchronize");
-  unsigned long long cnt = 0;
-  if ((e = cudaMemcpy(&cnt, p->tb.n, sizeof(cnt), cudaMemcpyDeviceToHost)) != cudaSuccess) return cuda_fail(e, "cudaMemcpy");
-  *n = (int64_t)cnt;
+  unsigned long long cnt[TRACE_SHARDS];
+  if ((e = cudaMemcpy(cnt, p->tb.n, sizeof(cnt), cudaMemcpyDeviceToHost)) != cudaSuccess) return cuda_fail(e, "cudaMemcpy");
+  int64_t total = 0;
+  for (int sh = 0; sh < TRACE_SHARDS; ++sh) total += (int64_t)cnt[sh];
+  *n = total;
   if (out && cap > 0) {
-    int64_t k = std::min<int64_t>({cap, (int64_t)cnt, p->tb.cap});
-    if (k > 0 && (e = cudaMemcpy(out, p->tb.rec, (size_t)k * sizeof(ktiler_trace_record), cudaMemcpyDeviceToHost)) != cudaSuccess)
-      return cuda_fail(e, "cudaMemcpy");
+    int64_t k = 0;  // gather the shards' written records, shard by shard
+    for (int sh = 0; sh < TRACE_SHARDS && k < cap; ++sh) {
+      const int64_t m = std::min<int64_t>({(int64_t)cnt[sh], p->tb.cap, cap - k});
+      if (m > 0 && (e = cudaMemcpy(out + k, p->tb.rec + (int64_t)sh * p->tb.cap, (size_t)m * sizeof(ktiler_trace_record),
+                                   cudaMemcpyDeviceToHost)) != cudaSuccess)
+        return cuda_fail(e, "cudaMemcpy");
+      k += m;
+    }
     if ((e = cudaMemset(p->tb.n, 0, sizeof(cnt))) != cudaSuccess) return cuda_fail(e, "cudaMemset");
   }
   kt::clear_error();

@@ -69,18 +69,23 @@ struct FTrace {
   unsigned long long* n;
   int64_t cap;
 };
+constexpr int FL_TRACE_SHARDS = 256;  // == exec.cu TRACE_SHARDS
 __device__ __forceinline__ uint64_t fl_timer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
 __device__ __forceinline__ void fl_trace(const FTrace& tb, uint64_t id, uint32_t kind, uint64_t t0, uint64_t t1) {
-  const unsigned long long k = atomicAdd(tb.n, 1ull);
-  if ((int64_t)k < tb.cap) {
-    uint32_t sm;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
-    tb.rec[k] = ktiler_trace_record{id, sm, kind, t0, t1};
-  }
+  // the plan's per-SM sharded trace buffer (exec.cu TraceBuf): FL_TRACE_SHARDS counters,
+  // cap records per shard
+  uint32_t sm;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+  // shard by a hash of (record id, CTA, SM): small launches fill the low SM ids with
+  // low CTA indices first, so SM or CTA alone would crowd a few shards
+  const uint32_t sh =
+      ((blockIdx.x * 0x9E3779B9u) ^ (sm * 0x85EBCA6Bu) ^ ((uint32_t)id * 0xC2B2AE35u)) >> 24 & (FL_TRACE_SHARDS - 1);
+  const unsigned long long k = atomicAdd(tb.n + sh, 1ull);
+  if ((int64_t)k < tb.cap) tb.rec[(int64_t)sh * tb.cap + (int64_t)k] = ktiler_trace_record{id, sm, kind, t0, t1};
 }
 
 struct FCtrl {

@@ -370,7 +370,10 @@ class Plan:
         _check(lib().ktiler_trace_read(self._h, ctypes.cast(buf, ctypes.c_void_p), cap, ctypes.byref(n)))
         dt = np.dtype([("id", "<u8"), ("smid", "<u4"), ("kind", "<u4"), ("t0", "<u8"), ("t1", "<u8")])
         k = min(n.value, cap)
-        return np.frombuffer(bytes(buf)[:k * dt.itemsize], dtype=dt).copy(), n.value
+        rec = np.frombuffer(bytes(buf)[:k * dt.itemsize], dtype=dt).copy()
+        # the library gathers its shards; a full shard drops its excess records, so fewer
+        # than k may have been copied (the rest of buf stays zero: t1 is never 0 in a record)
+        return rec[rec["t1"] != 0], n.value
 
     def launches(self):
         """[(sub, node, tiles)] of the plan's launch list (trace ids index it)."""
