@@ -231,15 +231,26 @@ __device__ __forceinline__ void consumer_discard(const KParams& p, const ktd::Ti
   const int64_t y0 = OP == 2 ? 2 * t.y0 : t.y0, nrows = OP == 2 ? 2 * (t.y1 - t.y0) : t.y1 - t.y0;
   const uint8_t* base = p.in.p + ktd::zoff(p.in, t.z);
   const int64_t b0 = EB * t.x0, b1 = EB * t.x1;
-  for (int64_t i = tid;; i += nt) {
-    // lines of row r: [ceil(a / 128), floor(b / 128)) of absolute addresses a, b
-    const int64_t first = ((int64_t)(uintptr_t)(base + y0 * p.in.pitch + b0) + 127) >> 7;
-    const int64_t last = ((int64_t)(uintptr_t)(base + y0 * p.in.pitch + b1)) >> 7;
-    const int64_t per = last > first ? last - first : 0;  // same for every row (128-B pitch)
-    if (per == 0 || i >= per * nrows) break;
-    const int64_t r = i / per, l = i - r * per;
-    const uint8_t* row = base + (y0 + r) * p.in.pitch;
-    ktd::discard_line(reinterpret_cast<const void*>((((int64_t)(uintptr_t)(row + b0) + 127) >> 7 << 7) + 128 * l));
+  // lines of row r: [ceil(a / 128), floor(b / 128)) of absolute addresses a, b; the count is
+  // the same for every row (128-B pitch).  CTA-uniform set-up once, then 32-bit index math
+  // per line (a 64-bit division per line cost more instructions than the down2 tile itself)
+  const int64_t r0 = (int64_t)(uintptr_t)(base + y0 * p.in.pitch);
+  const int64_t first = (r0 + b0 + 127) >> 7, last = (r0 + b1) >> 7;
+  if (last <= first) return;
+  const unsigned per = (unsigned)(last - first), n = per * (unsigned)nrows;
+  const int64_t pitch = p.in.pitch;
+  auto line = [&](unsigned r, unsigned l) {
+    const int64_t row = r0 + (int64_t)r * pitch;
+    ktd::discard_line(reinterpret_cast<const void*>((((row + b0 + 127) >> 7) + (int64_t)l) << 7));
+  };
+  if ((per & (per - 1)) == 0) {
+    const int sh = __ffs(per) - 1;
+    for (unsigned i = tid; i < n; i += nt) line(i >> sh, i & (per - 1));
+  } else {
+    for (unsigned i = tid; i < n; i += nt) {
+      const unsigned r = i / per;
+      line(r, i - r * per);
+    }
   }
 }
 
