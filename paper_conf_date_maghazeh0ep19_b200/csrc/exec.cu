@@ -344,15 +344,8 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     __shared__ ktd::Tile s_tile[KMAXST];  // decoded once by warp 0, read by all after the mbarrier
     __shared__ uint64_t s_tw[KMAXST];     // trace (chain): producers ready
     const int S = NST ? NST : (p.nstage < 2 ? 2 : (p.nstage > KMAXST ? KMAXST : p.nstage));
-    if (tid == 0) {
-      for (int j = 0; j < S; ++j) ktd::mbar_init(&mbar[j], 1);
-      ktd::fence_proxy_async();
-    }
-    __syncthreads();
-    if (!p.chain) pdl_enter();
-    if (p.tb.rec && tid == 0) s_tr = gtimer();
-    const unsigned epoch = s_epoch;
     const int64_t i0 = blockIdx.x;
+    unsigned epoch = 0;
     auto issue = [&](int64_t i, int slot) {  // warp 0
       const ktd::Tile t = launch_tile(p, i);
       if (p.chain) {  // producers' tiles complete (acquire), then hand them to the async proxy
@@ -371,8 +364,27 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
         ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
       }
     };
+    // Tensor-map staging (one thread issues): thread 0 waits for the programmatic producers
+    // itself (griddepcontrol.wait orders the executing thread after every prerequisite
+    // grid's completion and memory flush) and requests the CTA's first tile at once,
+    // instead of after every warp of the CTA has reached the barrier (64 x 8K: -0.7% tiled
+    // and untiled).  The other threads still pass pdl_enter before touching
+    // anything a producer wrote; they read only the staged tile, after its mbarrier.
+    const bool early = p.use_tmap && !p.chain && i0 < ntiles;
+    if (tid == 0) {
+      for (int j = 0; j < S; ++j) ktd::mbar_init(&mbar[j], 1);
+      ktd::fence_proxy_async();
+      if (early) {
+        if (p.pdl) pdl_wait();
+        issue(i0, 0);
+      }
+    }
+    __syncthreads();
+    if (!p.chain) pdl_enter();
+    if (p.tb.rec && tid == 0) s_tr = gtimer();
+    epoch = s_epoch;
     if (tid < 32)
-      for (int j = 0; j < S && i0 + j * (int64_t)gridDim.x < ntiles; ++j) issue(i0 + j * (int64_t)gridDim.x, j);
+      for (int j = early ? 1 : 0; j < S && i0 + j * (int64_t)gridDim.x < ntiles; ++j) issue(i0 + j * (int64_t)gridDim.x, j);
     int b = 0;          // slot of the current tile
     unsigned par = 0;   // its mbarrier phase parity (flips each time the ring wraps)
     for (int64_t i = i0; i < ntiles; i += gridDim.x) {
