@@ -1483,7 +1483,10 @@ ktiler_status prep_launch(ktiler_plan_s* P, Launch& L, kfn_t fn, int64_t* grid_o
   // GRAPH_WAVE: one tile per CTA, so the hardware scheduler balances concurrent
   // sub-kernels tile by tile (64 x 8K, 0.5 x L2 resident budget: 4.03 ms vs 4.23 ms
   // grid-stride).  Measured on 64 x 8K; KTILER_TILES_PER_CTA overrides.
-  const bool concurrent = P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE;
+  // (a one-fragment plan has no concurrent sub-kernels: it is the untiled schedule and
+  // takes the GRAPH rule, so the two replay identical launches)
+  const bool concurrent =
+      (P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE) && P->s.nfrag > 1;
   int tpc = tpc_env >= 0 ? tpc_env : (L.blocks > 8 * L.resident ? 2 : ((chain || concurrent) ? 1 : 0));
   if (tpc_env < 0 && tpc == 2 && L.node >= 0 && !L.n->scalar && L.kp.stage_bytes && L.smem == (int)(2 * L.kp.stage_bytes)) {
     // double buffering halves the CTAs that fit by shared memory; when registers would
