@@ -137,8 +137,11 @@ def test_discover_user_kernel(boxlib):
     assert acc["hl"] >= 2 and acc["hr"] >= 2     # >= the 2-px reach (128-B line quantized)
 
 
-@pytest.mark.parametrize("mode", ["dag", "graph", "stream"])
+@pytest.mark.parametrize("mode", ["dag", "dag_pdl", "graph", "stream"])
 def test_user_kernel_tiled_after_discovery(boxlib, mode):
+    """dag_pdl: the bench's DAG policy (programmatic producer edges, dispatch-order edges from
+    the source's consumers, A50) with a user kernel as the source's consumer: the
+    order and PDL edges skip it (a child graph has no programmatic port)."""
     from paper_conf_date_maghazeh0ep19_b200 import footprint as FP
     from paper_conf_date_maghazeh0ep19_b200 import ktiler as K
     c0, reads, _ = _discover(boxlib)
@@ -148,7 +151,10 @@ def test_user_kernel_tiled_after_discovery(boxlib, mode):
     c.view("rgb").copy_(torch.from_numpy(rgb))
     for k in ("gray", "box", "down"):
         c.t[k].fill_(0xA5)
-    plan = c.g.plan(48 * 1024, kind="budget", exec_mode=mode)
+    if mode == "dag_pdl":
+        plan = c.g.plan(48 * 1024, kind="budget", exec_mode="dag", pdl=True, resident_budget=True, window=2)
+    else:
+        plan = c.g.plan(48 * 1024, kind="budget", exec_mode=mode)
     assert plan.num_fragments() >= 4
     for _ in range(2):  # replays (DAG: the captured callback runs again)
         plan.execute(torch.cuda.current_stream().cuda_stream)
