@@ -235,11 +235,16 @@ __device__ __forceinline__ void flow_consumer_discard(const FNode& nd, const ktd
   const int64_t b0 = eb * t.x0, b1 = eb * t.x1;
   const int64_t first = ((int64_t)(uintptr_t)(base + y0 * nd.in.pitch + b0) + 127) >> 7;
   const int64_t last = ((int64_t)(uintptr_t)(base + y0 * nd.in.pitch + b1)) >> 7;
-  const int64_t per = last > first ? last - first : 0;  // same for every row (128-B pitch)
-  for (int64_t i = tid; i < per * nrows; i += nt) {
-    const int64_t r = i / per, l = i - r * per;
-    const uint8_t* row = base + (y0 + r) * nd.in.pitch;
-    ktd::discard_line(reinterpret_cast<const void*>((((int64_t)(uintptr_t)(row + b0) + 127) >> 7 << 7) + 128 * l));
+  if (last <= first) return;
+  // same count for every row (128-B pitch); 32-bit index math per line (a 64-bit division
+  // per line cost more than the tile's own arithmetic)
+  const unsigned per = (unsigned)(last - first), n = per * (unsigned)nrows;
+  const bool pow2 = (per & (per - 1)) == 0;
+  const int sh = __ffs(per) - 1;
+  for (unsigned i = tid; i < n; i += nt) {
+    const unsigned r = pow2 ? i >> sh : i / per, l = i - r * per;
+    const uint8_t* row = base + (y0 + (int64_t)r) * nd.in.pitch;
+    ktd::discard_line(reinterpret_cast<const void*>((((int64_t)(uintptr_t)(row + b0) + 127) >> 7 << 7) + 128 * (int64_t)l));
   }
 }
 
