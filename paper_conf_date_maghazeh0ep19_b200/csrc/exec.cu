@@ -266,9 +266,11 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
   const int py0 = ry0 / p.way, py1 = min(p.pgy, (ry1 + p.way - 1) / p.way);
   const int pw = px1 - px0, n = pw * (py1 - py0);
   const uint8_t* fb = p.in.p + ktd::zoff(p.in, bz);
+  const unsigned upw = (unsigned)max(pw, 1);
   for (int i0 = 0; i0 < n; i0 += 32) {
     const int i = i0 + lane;
-    const int py = py0 + i / max(pw, 1), px = px0 + i % max(pw, 1);
+    const unsigned qd = (unsigned)i / upw;
+    const int py = py0 + (int)qd, px = px0 + (int)((unsigned)i - qd * upw);
     bool last = false;
     if (i < n) {
       const int64_t idx = ((int64_t)bz * p.pgy + py) * p.pgx + px;
@@ -283,10 +285,14 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
       const int64_t y0 = (int64_t)p.way * qy, y1 = min((int64_t)p.in.H, y0 + p.way);
       const int64_t a0 = (int64_t)(uintptr_t)(fb + y0 * p.in.pitch + x0);
       const int64_t l0 = (a0 + 127) >> 7, l1 = (a0 + (x1 - x0)) >> 7;  // whole lines of the first row
-      const int64_t per = l1 > l0 ? l1 - l0 : 0, tot = per * (y1 - y0);
-      for (int64_t k = lane; k < tot; k += 32) {
-        const int64_t r = k / per, l = k - r * per;
-        ktd::discard_line(reinterpret_cast<const void*>(((l0 + l) << 7) + r * p.in.pitch));
+      if (l1 <= l0) continue;
+      // 32-bit index math per line (as consumer_discard): shift / mask for power-of-two rows
+      const unsigned per = (unsigned)(l1 - l0), tot = per * (unsigned)(y1 - y0);
+      const bool pow2 = (per & (per - 1)) == 0;
+      const int sh = __ffs(per) - 1;
+      for (unsigned k = lane; k < tot; k += 32) {
+        const unsigned r = pow2 ? k >> sh : k / per, l = k - r * per;
+        ktd::discard_line(reinterpret_cast<const void*>(((l0 + (int64_t)l) << 7) + (int64_t)r * p.in.pitch));
       }
     }
   }
