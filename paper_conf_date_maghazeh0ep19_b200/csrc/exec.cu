@@ -301,7 +301,10 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
 // NST: staging ring depth; 2 (compile time, the default code path) or 0 = p.nstage at run
 // time (KTILER_STAGES variants of the L2-fed consumers, instantiated for down2 / sobel3 /
 // thresh only)
-template <int OP, bool SCALAR, int NST = 2>
+// LEAN: no GRAPH_CHAIN flags, no counted halo discards, no tracing (the launch has none of
+// them; launch_fn picks it): those paths are compiled out, which leaves the register
+// allocator more room (blur5 runs at its 80-register cap)
+template <int OP, bool SCALAR, int NST = 2, bool LEAN = false>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
   __shared__ uint64_t s_t0;  // trace: CTA start (kept out of registers)
   __shared__ uint64_t s_tr, s_tl;  // trace: producers ready (after PDL wait), first tile staged
@@ -309,8 +312,8 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
   const int nt = blockDim.x * blockDim.y * blockDim.z;
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
   if (tid == 0) {
-    if (p.tb.rec) s_t0 = gtimer();
-    if (p.chain) s_epoch = *(volatile const unsigned int*)p.epoch;
+    if ((!LEAN && p.tb.rec)) s_t0 = gtimer();
+    if ((!LEAN && p.chain)) s_epoch = *(volatile const unsigned int*)p.epoch;
   }
   // PDL (p.pdl): wait for the programmatic producers (griddepcontrol.wait), then let this
   // launch's dependents be scheduled (p.pdl == 1: right away; 2: only when CTAs exit).  The
@@ -322,7 +325,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     if (p.ndisc) do_discards(p);
     if (p.pdl == 1 || p.pdl == 3) pdl_launch();
   };
-  if (p.chain) {
+  if ((!LEAN && p.chain)) {
     pdl_launch();  // the next sub-kernel may become resident now: it waits on tile flags
   } else if (SCALAR) {
     pdl_enter();
@@ -333,12 +336,12 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     const unsigned epoch = s_epoch;
     for (int64_t i = blockIdx.x; i < ntiles; i += gridDim.x) {
       const ktd::Tile t = launch_tile(p, i);
-      if (p.chain) {
+      if ((!LEAN && p.chain)) {
         if (tid < 32) chain_wait(p, (int)(t.x0 / p.tw), (int)(t.y0 / p.th), (int)t.z, epoch, tid);
         __syncthreads();
       }
       ktd::scalar_tile(OP, p.in, p.out, t, p.T, nt, tid);
-      if (p.chain) {
+      if ((!LEAN && p.chain)) {
         __syncthreads();
         if (tid == 0) chain_publish(p, t, epoch);
       }
@@ -356,10 +359,10 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     unsigned epoch = 0;
     auto issue = [&](int64_t i, int slot) {  // warp 0
       const ktd::Tile t = launch_tile(p, i);
-      if (p.chain) {  // producers' tiles complete (acquire), then hand them to the async proxy
+      if ((!LEAN && p.chain)) {  // producers' tiles complete (acquire), then hand them to the async proxy
         chain_wait(p, (int)(t.x0 / p.tw), (int)(t.y0 / p.th), (int)t.z, epoch, tid);
         ktd::fence_proxy_async();
-        if (p.tb.rec && tid == 0) s_tw[slot] = gtimer();
+        if ((!LEAN && p.tb.rec) && tid == 0) s_tw[slot] = gtimer();
       }
       uint8_t* dst = ktsm + slot * p.stage_bytes;
       if (p.use_tmap) {
@@ -378,7 +381,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     // instead of after every warp of the CTA has reached the barrier (64 x 8K: -0.7% tiled
     // and untiled).  The other threads still pass pdl_enter before touching
     // anything a producer wrote; they read only the staged tile, after its mbarrier.
-    const bool early = p.use_tmap && !p.chain && i0 < ntiles;
+    const bool early = p.use_tmap && !(!LEAN && p.chain) && i0 < ntiles;
     if (tid == 0) {
       for (int j = 0; j < S; ++j) ktd::mbar_init(&mbar[j], 1);
       ktd::fence_proxy_async();
@@ -388,8 +391,8 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       }
     }
     __syncthreads();
-    if (!p.chain) pdl_enter();
-    if (p.tb.rec && tid == 0) s_tr = gtimer();
+    if (!(!LEAN && p.chain)) pdl_enter();
+    if ((!LEAN && p.tb.rec) && tid == 0) s_tr = gtimer();
     epoch = s_epoch;
     if (tid < 32)
       for (int j = early ? 1 : 0; j < S && i0 + j * (int64_t)gridDim.x < ntiles; ++j) issue(i0 + j * (int64_t)gridDim.x, j);
@@ -398,13 +401,13 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     for (int64_t i = i0; i < ntiles; i += gridDim.x) {
       uint8_t* buf = ktsm + b * p.stage_bytes;
       ktd::mbar_wait(&mbar[b], par);
-      if (p.tb.rec && tid == 0 && i == i0) s_tl = gtimer();
+      if ((!LEAN && p.tb.rec) && tid == 0 && i == i0) s_tl = gtimer();
       const ktd::Tile t = s_tile[b];
       if constexpr (OP == 2 || OP == 4) {
         if (p.cdisc) consumer_discard<OP>(p, t, nt, tid);
       }
       if constexpr (OP == 1 || OP == 3) {  // as soon as staged: the earlier, the fewer write-backs
-        if (p.hcnt && tid < 32) halo_discard(p, t, tid);
+        if ((!LEAN && p.hcnt) && tid < 32) halo_discard(p, t, tid);
       }
 
       if ((OP == 1 || OP == 3 || OP == 6 || OP == 7) && ktd::needs_fix(OP, p.in, t)) {
@@ -413,12 +416,12 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       }
       ktd::compute_tile(OP, p.out, t, buf, p.T, nt, tid, &p.aux, p.taps, p.radius);
       const int64_t nx = i + (int64_t)S * gridDim.x;
-      if (p.chain) {
+      if ((!LEAN && p.chain)) {
         __syncthreads();  // tile written (and buffer b consumed)
         if (tid == 0) {
-          const uint64_t tc = p.tb.rec ? gtimer() : 0;
+          const uint64_t tc = (!LEAN && p.tb.rec) ? gtimer() : 0;
           chain_publish(p, t, epoch);
-          if (p.tb.rec) {
+          if ((!LEAN && p.tb.rec)) {
             trace_put(p.tb, p.lid, 3, s_tw[b], tc);  // producers ready -> tile computed
             trace_put(p.tb, p.lid, 4, tc, gtimer());  // publish (fence + release)
           }
@@ -436,7 +439,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       }
     }
   }
-  if (p.chain) {
+  if ((!LEAN && p.chain)) {
     __syncthreads();
     if (tid == 0) chain_finish(p, s_epoch, p.chain == 2);
     if (p.ndisc) {  // lines dead after an earlier launch: wait until it and all before it finished
@@ -446,11 +449,11 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
       do_discards(p);
     }
   }
-  if (p.tb.rec) {
+  if ((!LEAN && p.tb.rec)) {
     __syncthreads();
     if (tid == 0) {
       trace_put(p.tb, p.lid, 0, s_t0, gtimer());
-      if (!SCALAR && !p.chain && blockIdx.x < ntiles) {  // CTA phases: start -> ready -> first tile staged
+      if (!SCALAR && !(!LEAN && p.chain) && blockIdx.x < ntiles) {  // CTA phases: start -> ready -> first tile staged
         trace_put(p.tb, p.lid, 5, s_t0, s_tr);
         trace_put(p.tb, p.lid, 6, s_tr, s_tl);
       }
@@ -882,6 +885,16 @@ kfn_t vec_kernel(int op) {
     case 6: return op_kernel<6, false>;
     case 7: return op_kernel<7, false>;
     default: return op_kernel<4, false>;
+  }
+}
+kfn_t vec_kernel_lean(int op) {
+  switch (op) {
+    case 0: return op_kernel<0, false, 2, true>;
+    case 1: return op_kernel<1, false, 2, true>;
+    case 2: return op_kernel<2, false, 2, true>;
+    case 3: return op_kernel<3, false, 2, true>;
+    case 4: return op_kernel<4, false, 2, true>;
+    default: return nullptr;
   }
 }
 kfn_t scalar_kernel(int op) {
@@ -1438,6 +1451,10 @@ kfn_t deep_kernel(int op) {  // runtime ring depth (KParams::nstage > 2)
   }
 }
 kfn_t launch_fn(const Launch& L) {
+  static const bool lean_off = getenv("KTILER_LEAN") && atoi(getenv("KTILER_LEAN")) == 0;  // experiment knob
+  if (!lean_off && L.node >= 0 && !L.n->scalar && L.kp.nstage <= 2 && !L.kp.chain && !L.kp.hcnt && !L.kp.tb.rec &&
+      vec_kernel_lean(L.n->op))
+    return vec_kernel_lean(L.n->op);
   if (L.node >= 0 && !L.n->scalar && L.kp.nstage > 2 && deep_kernel(L.n->op)) return deep_kernel(L.n->op);
   return L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
 }
