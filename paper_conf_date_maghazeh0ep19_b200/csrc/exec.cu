@@ -887,13 +887,13 @@ kfn_t vec_kernel(int op) {
     default: return op_kernel<4, false>;
   }
 }
-kfn_t vec_kernel_lean(int op) {
+kfn_t vec_kernel_lean(int op, bool one) {  // one: a one-slot staging ring (one tile per CTA)
   switch (op) {
-    case 0: return op_kernel<0, false, 2, true>;
-    case 1: return op_kernel<1, false, 2, true>;
-    case 2: return op_kernel<2, false, 2, true>;
-    case 3: return op_kernel<3, false, 2, true>;
-    case 4: return op_kernel<4, false, 2, true>;
+    case 0: return one ? op_kernel<0, false, 1, true> : op_kernel<0, false, 2, true>;
+    case 1: return one ? op_kernel<1, false, 1, true> : op_kernel<1, false, 2, true>;
+    case 2: return one ? op_kernel<2, false, 1, true> : op_kernel<2, false, 2, true>;
+    case 3: return one ? op_kernel<3, false, 1, true> : op_kernel<3, false, 2, true>;
+    case 4: return one ? op_kernel<4, false, 1, true> : op_kernel<4, false, 2, true>;
     default: return nullptr;
   }
 }
@@ -919,6 +919,7 @@ struct Launch {
   int sub = -1;          // schedule sub-kernel (kernel launches) / discard list (DAG discards)
   std::vector<int32_t> crects;  // OP_CUSTOM rect list
   int cap_per_sm = 0;    // > 0: grid capped at this many CTAs per SM (grid-stride through the ring)
+  bool one = false;      // one tile per CTA by construction (tiled GRAPH_DAG / WAVE): one-slot ring kernel
 };
 
 }  // namespace
@@ -1229,6 +1230,10 @@ void build_launches(ktiler_plan_s* P) {
           L.smem = (int)(L.kp.nstage * L.kp.stage_bytes);
           L.cap_per_sm = src_ctas;
         }
+        // tiled GRAPH_DAG / WAVE launches run one tile per CTA (prep_launch) unless overridden
+        static const bool tpc_set = getenv("KTILER_TILES_PER_CTA") != nullptr;
+        L.one = !tpc_set && L.kp.nstage <= 2 && L.cap_per_sm == 0 && P->s.nfrag > 1 &&
+                (P->pol.exec_mode == KTILER_EXEC_GRAPH_DAG || P->pol.exec_mode == KTILER_EXEC_GRAPH_WAVE);
         P->launches.push_back(L);
       }
     }
@@ -1451,10 +1456,12 @@ kfn_t deep_kernel(int op) {  // runtime ring depth (KParams::nstage > 2)
   }
 }
 kfn_t launch_fn(const Launch& L) {
-  static const bool lean_off = getenv("KTILER_LEAN") && atoi(getenv("KTILER_LEAN")) == 0;  // experiment knob
-  if (!lean_off && L.node >= 0 && !L.n->scalar && L.kp.nstage <= 2 && !L.kp.chain && !L.kp.hcnt && !L.kp.tb.rec &&
-      vec_kernel_lean(L.n->op))
-    return vec_kernel_lean(L.n->op);
+  // KTILER_LEAN (experiment knob): 0 = full kernels, 1 = lean two-slot only, unset = lean, and
+  // one-slot where the launch runs one tile per CTA (L.one, GRAPH_DAG / WAVE tiled plans)
+  static const int lean_env = getenv("KTILER_LEAN") ? atoi(getenv("KTILER_LEAN")) : 2;
+  if (lean_env && L.node >= 0 && !L.n->scalar && L.kp.nstage <= 2 && !L.kp.chain && !L.kp.hcnt && !L.kp.tb.rec &&
+      vec_kernel_lean(L.n->op, false))
+    return vec_kernel_lean(L.n->op, lean_env == 2 && L.one);
   if (L.node >= 0 && !L.n->scalar && L.kp.nstage > 2 && deep_kernel(L.n->op)) return deep_kernel(L.n->op);
   return L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
 }
