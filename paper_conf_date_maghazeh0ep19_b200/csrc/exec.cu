@@ -301,8 +301,8 @@ __device__ __forceinline__ void halo_discard(const KParams& p, const ktd::Tile& 
 // NST: staging ring depth; 2 (compile time, the default code path) or 0 = p.nstage at run
 // time (KTILER_STAGES variants of the L2-fed consumers, instantiated for down2 / sobel3 /
 // thresh only)
-// LEAN: no GRAPH_CHAIN flags, no counted halo discards, no tracing (the launch has none of
-// them; launch_fn picks it): those paths are compiled out, which leaves the register
+// LEAN: no GRAPH_CHAIN flags, no counted halo discards, no tracing, no discard lists, tensor-
+// map staging (the launch has none of the former; launch_fn picks it): those paths are compiled out, which leaves the register
 // allocator more room (blur5 runs at its 80-register cap)
 template <int OP, bool SCALAR, int NST = 2, bool LEAN = false>
 __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP == 1 ? 3 : 4)) op_kernel(const __grid_constant__ KParams p) {
@@ -322,7 +322,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
   // (dag_order_node): it reads no producer's output, so it does not wait for one
   auto pdl_enter = [&]() {
     if (p.pdl && (p.pdl != 3 || p.ndisc)) pdl_wait();
-    if (p.ndisc) do_discards(p);
+    if (!LEAN && p.ndisc) do_discards(p);  // LEAN launches carry no discard lists
     if (p.pdl == 1 || p.pdl == 3) pdl_launch();
   };
   if ((!LEAN && p.chain)) {
@@ -365,12 +365,12 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
         if ((!LEAN && p.tb.rec) && tid == 0) s_tw[slot] = gtimer();
       }
       uint8_t* dst = ktsm + slot * p.stage_bytes;
-      if (p.use_tmap) {
+      if (LEAN || p.use_tmap) {  // LEAN launches always stage by tensor map
         if (tid == 0) {
           s_tile[slot] = t;
           ktd::stage_issue_tmap(OP, &p.tmap, p.box_bytes, p.in, t, dst, &mbar[slot], p.in_stream != 0);
         }
-      } else {
+      } else if constexpr (!LEAN) {
         if (tid == 0) s_tile[slot] = t;
         ktd::stage_issue(OP, p.in, t, dst, &mbar[slot], tid);
       }
@@ -381,7 +381,7 @@ __global__ void __launch_bounds__(256, (OP == 3 || OP == 6 || OP == 7) ? 2 : (OP
     // instead of after every warp of the CTA has reached the barrier (64 x 8K: -0.7% tiled
     // and untiled).  The other threads still pass pdl_enter before touching
     // anything a producer wrote; they read only the staged tile, after its mbarrier.
-    const bool early = p.use_tmap && !(!LEAN && p.chain) && i0 < ntiles;
+    const bool early = (LEAN || p.use_tmap) && !(!LEAN && p.chain) && i0 < ntiles;
     if (tid == 0) {
       for (int j = 0; j < S; ++j) ktd::mbar_init(&mbar[j], 1);
       ktd::fence_proxy_async();
@@ -1460,7 +1460,7 @@ kfn_t launch_fn(const Launch& L) {
   // one-slot where the launch runs one tile per CTA (L.one, GRAPH_DAG / WAVE tiled plans)
   static const int lean_env = getenv("KTILER_LEAN") ? atoi(getenv("KTILER_LEAN")) : 2;
   if (lean_env && L.node >= 0 && !L.n->scalar && L.kp.nstage <= 2 && !L.kp.chain && !L.kp.hcnt && !L.kp.tb.rec &&
-      vec_kernel_lean(L.n->op, false))
+      L.kp.use_tmap && !L.kp.ndisc && vec_kernel_lean(L.n->op, false))
     return vec_kernel_lean(L.n->op, lean_env == 2 && L.one);
   if (L.node >= 0 && !L.n->scalar && L.kp.nstage > 2 && deep_kernel(L.n->op)) return deep_kernel(L.n->op);
   return L.node < 0 ? (kfn_t)discard_kernel : (L.n->scalar ? scalar_kernel(L.n->op) : vec_kernel(L.n->op));
