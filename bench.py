@@ -625,7 +625,7 @@ def main():
                 ach = d["bytes"] / d["launches"] / (d["span_ns"] / d["launches"])  # B/ns = GB/s
                 dtraffic = None
                 try:
-                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02h_dominant_traffic.json")))
+                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02i_dominant_traffic.json")))
                     if dom in dt["kernels"] and all(line["config"].get(k) == v for k, v in dt["config"].items()):
                         kd = dt["kernels"][dom]
                         dtraffic = {"bytes": kd["dram_bytes_per_launch_mean"], "source": kd["source"]}
