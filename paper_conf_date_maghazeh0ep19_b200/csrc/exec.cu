@@ -894,6 +894,8 @@ kfn_t vec_kernel_lean(int op, bool one) {  // one: a one-slot staging ring (one 
     case 2: return one ? op_kernel<2, false, 1, true> : op_kernel<2, false, 2, true>;
     case 3: return one ? op_kernel<3, false, 1, true> : op_kernel<3, false, 2, true>;
     case 4: return one ? op_kernel<4, false, 1, true> : op_kernel<4, false, 2, true>;
+    case 6: return one ? op_kernel<6, false, 1, true> : op_kernel<6, false, 2, true>;
+    case 7: return one ? op_kernel<7, false, 1, true> : op_kernel<7, false, 2, true>;
     default: return nullptr;
   }
 }
