@@ -65,7 +65,7 @@ def parse(argv=None):
     ap.add_argument("--mode", default="dag", choices=["stream", "graph", "persist_l2", "persistent", "dag", "chain", "wave", "flow"])
     ap.add_argument("--kind", default="budget", choices=["budget", "rows", "balanced", "none"])
     ap.add_argument("--rows", type=int, default=2)
-    ap.add_argument("--l2-fraction", type=float, default=0.94)
+    ap.add_argument("--l2-fraction", type=float, default=1.0)
     ap.add_argument("--no-resident", action="store_true",
                     help="paper-literal budget (count graph input/output lines too; SURVEY A11)")
     ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
@@ -625,7 +625,7 @@ def main():
                 ach = d["bytes"] / d["launches"] / (d["span_ns"] / d["launches"])  # B/ns = GB/s
                 dtraffic = None
                 try:
-                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02i_dominant_traffic.json")))
+                    dt = json.load(open(os.path.join(ROOT, "profiles", "r02j_dominant_traffic.json")))
                     if dom in dt["kernels"] and all(line["config"].get(k) == v for k, v in dt["config"].items()):
                         kd = dt["kernels"][dom]
                         dtraffic = {"bytes": kd["dram_bytes_per_launch_mean"], "source": kd["source"]}

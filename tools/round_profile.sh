@@ -15,7 +15,7 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/$
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 4000 --csv --log-file gpurun_out/${TAG}_launches_bench.csv \
   python bench.py --steps 2 --warmup 1 --no-cpu --no-e2e --no-trace --no-untiled --no-ncu > gpurun_out/${TAG}_launches_bench.log 2>&1
 echo "launches rc=$?"
-C='[{"kind":"budget","l2_fraction":0.94,"exec_mode":"dag","discard":false,"window":2,"resident_budget":true,"consumer_discard":true,"pdl":true}]'
+C='[{"kind":"budget","l2_fraction":1.0,"exec_mode":"dag","discard":false,"window":2,"resident_budget":true,"consumer_discard":true,"pdl":true}]'
 for K in 0 1; do
   timeout 900 ncu --set full --import-source on --cache-control none --clock-control none --kernel-name-base mangled \
     -k regex:"op_kernelILi${K}ELb0" --launch-skip 120 -c 4 -f -o gpurun_out/${TAG}_dag_op${K}_full \
